@@ -1,0 +1,625 @@
+// api.cu -- C ABI (include/bzk.h), batch scheduler (waves, ping-pong scratch, tail cut-off) and
+// stream loader (host -> device waves on a side stream, "dynamic loading").
+//
+// a1 input residency/loading, a8 batch scheduler; the kernels for rows
+// a2-a7 live in sumcheck.cuh.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "bzk.h"
+#include "field.cuh"
+#include "gen.cuh"
+#include "sha256.cuh"
+#include "sumcheck.cuh"
+
+using namespace bzk;
+
+namespace {
+
+constexpr uint32_t kThreads = 256;
+constexpr uint32_t kTailLog = 8;          // rounds with h <= 2^kTailLog pairs run in k_tail
+constexpr uint32_t kSMs = 148;
+
+struct ProfRec { int kind; cudaEvent_t a, b; };
+
+}  // namespace
+
+struct bzk_ctx {
+    int device = 0;
+    size_t workspace_limit = 0;
+    void *ws = nullptr;
+    size_t ws_size = 0;
+    cudaStream_t copy_stream = nullptr;
+    cudaEvent_t ev_copied[2] = {nullptr, nullptr};
+    cudaEvent_t ev_consumed[2] = {nullptr, nullptr};
+    uint32_t *d_flag = nullptr;
+    std::string last_error;
+    bool prof = false;
+    std::vector<ProfRec> recs;
+    std::vector<cudaEvent_t> ev_pool;
+    uint64_t launches = 0;
+    int num_sms = kSMs;
+};
+
+namespace {
+
+bzk_status fail(bzk_ctx *c, bzk_status s, const std::string &msg) {
+    if (c) c->last_error = msg;
+    return s;
+}
+
+bzk_status cuda_fail(bzk_ctx *c, cudaError_t e, const char *where) {
+    return fail(c, BZK_ECUDA, std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(call)                                                   \
+    do {                                                           \
+        cudaError_t _e = (call);                                   \
+        if (_e != cudaSuccess) return cuda_fail(ctx, _e, #call);   \
+    } while (0)
+
+cudaEvent_t pool_event(bzk_ctx *ctx) {
+    if (!ctx->ev_pool.empty()) {
+        cudaEvent_t e = ctx->ev_pool.back();
+        ctx->ev_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    return e;
+}
+
+struct ProfScope {
+    bzk_ctx *ctx; cudaStream_t s; int kind; cudaEvent_t a = nullptr;
+    ProfScope(bzk_ctx *c, cudaStream_t st, int k) : ctx(c), s(st), kind(k) {
+        if (ctx->prof) { a = pool_event(ctx); cudaEventRecord(a, s); }
+    }
+    ~ProfScope() {
+        if (ctx->prof) {
+            cudaEvent_t b = pool_event(ctx);
+            cudaEventRecord(b, s);
+            ctx->recs.push_back({kind, a, b});
+        }
+    }
+};
+
+// ---------------------------------------------------------------- planning
+
+struct Plan {
+    uint32_t k, D, order;
+    uint64_t B, Bw, nwaves;
+    uint32_t i0;          // first tail round (k >= 1)
+    uint32_t log_h0;      // pairs of the first tail round
+    uint64_t N;
+    size_t elem_table;    // bytes of one table set (D * N * 32)
+    // per-wave workspace layout (bytes)
+    size_t off_ps, off_tick, off_part, off_bufX, off_bufY, off_stage0, off_stage1, off_out, off_seed;
+    size_t total;
+    uint32_t cmax;
+    bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
+    size_t out_bytes_per_proof;
+};
+
+uint32_t ctas_for(uint64_t h, uint64_t nb) {
+    // enough CTAs to fill 148 SMs x 2 resident CTAs x 4 waves, at most 16 pairs per thread
+    const uint64_t target = (uint64_t)kSMs * 2 * 4;
+    uint64_t ppt = (nb * h) / ((uint64_t)kThreads * target);
+    ppt = std::max<uint64_t>(1, std::min<uint64_t>(16, ppt));
+    uint64_t c = (h + kThreads * ppt - 1) / (kThreads * ppt);
+    return (uint32_t)std::max<uint64_t>(1, c);
+}
+
+size_t align_up(size_t x) { return (x + 255) & ~(size_t)255; }
+
+bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
+    if (!b) return fail(ctx, BZK_EINVAL, "batch is NULL");
+    if (b->num_vars > 30) return fail(ctx, BZK_EINVAL, "num_vars must be <= 30");
+    if (b->degree < 1 || b->degree > 4) return fail(ctx, BZK_EINVAL, "degree must be in 1..4");
+    if (b->order > 1) return fail(ctx, BZK_EINVAL, "order must be BZK_ORDER_LSB or BZK_ORDER_MSB");
+    if (b->batch == 0) return fail(ctx, BZK_EINVAL, "batch must be >= 1");
+    if (!b->seed) return fail(ctx, BZK_EINVAL, "seed is NULL");
+    if (!b->tables) return fail(ctx, BZK_EINVAL, "tables is NULL");
+    if (b->num_vars > 0 && (!b->round_evals || !b->challenges))
+        return fail(ctx, BZK_EINVAL, "round_evals/challenges is NULL");
+    if (!b->final_evals) return fail(ctx, BZK_EINVAL, "final_evals is NULL");
+    if (b->tables_mem > 1 || b->outputs_mem > 1) return fail(ctx, BZK_EINVAL, "bad *_mem value");
+    if (b->first_index + b->batch > (1ull << 28)) return fail(ctx, BZK_EINVAL, "global index must be < 2^28");
+    return BZK_OK;
+}
+
+bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
+    P.k = b->num_vars; P.D = b->degree; P.order = b->order; P.B = b->batch;
+    P.N = 1ull << P.k;
+    P.elem_table = (size_t)P.D * P.N * 32;
+    P.host_tables = b->tables_mem == BZK_MEM_HOST;
+    P.host_outputs = b->outputs_mem == BZK_MEM_HOST;
+    if (P.k == 0) { P.i0 = 1; P.log_h0 = 0; }
+    else if (P.k - 1 <= kTailLog) { P.i0 = 1; P.log_h0 = P.k - 1; }
+    else { P.i0 = P.k - kTailLog; P.log_h0 = kTailLog; }
+    const bool preserve = (b->flags & BZK_F_PRESERVE_INPUT) != 0;
+    P.need_bufX = P.i0 > 2;
+    P.need_bufY = P.i0 > 3;
+    // consume mode (or host tables staged into our own buffers): round 3+ may overwrite the input
+    P.bufY_alias_input = P.need_bufY && (P.host_tables || !preserve);
+    P.out_bytes_per_proof = (size_t)32 * ((size_t)P.k * (P.D + 1) + P.k + P.D + 1);
+
+    size_t limit = ctx->workspace_limit;
+    if (limit == 0) {
+        size_t fr = 0, tot = 0;
+        cudaMemGetInfo(&fr, &tot);
+        fr += ctx->ws_size;  // our own current allocation is reusable
+        limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
+    }
+    auto per_proof = [&](uint64_t bw) -> size_t {
+        (void)bw;
+        size_t s = sizeof(ProofState) + 4;
+        uint32_t c = P.k ? ctas_for(1ull << (P.k - 1), bw) : 1;
+        s += (size_t)c * (P.D + 1) * 32;
+        if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * 32;
+        if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * 32;
+        if (P.host_tables) s += 2 * P.elem_table;
+        return s;
+    };
+    const size_t fixed = 4096 + (P.host_outputs ? align_up(P.B * P.out_bytes_per_proof) : 0);
+    uint64_t bw = std::min<uint64_t>(P.B, 65535);
+    while (bw > 1 && fixed + per_proof(bw) * bw + 8 * 256 > limit) bw = (bw + 1) / 2;
+    if (fixed + per_proof(bw) * bw + 8 * 256 > limit)
+        return fail(ctx, BZK_ENOMEM, "workspace_limit too small for one proof");
+    // balance the waves
+    uint64_t nw = (P.B + bw - 1) / bw;
+    bw = (P.B + nw - 1) / nw;
+    P.Bw = bw; P.nwaves = nw;
+    P.cmax = P.k ? std::max(ctas_for(1ull << (P.k - 1), bw),
+                            ctas_for(1ull << (P.k - 1), P.B - (nw - 1) * bw)) : 1;
+
+    size_t off = 0;
+    P.off_seed = off; off += 256;
+    P.off_ps = off; off = align_up(off + bw * sizeof(ProofState));
+    P.off_tick = off; off = align_up(off + bw * 4);
+    P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * (P.D + 1) * 32);
+    P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * 32);
+    P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * 32);
+    P.off_stage0 = off; if (P.host_tables) off = align_up(off + bw * P.elem_table);
+    P.off_stage1 = off; if (P.host_tables) off = align_up(off + bw * P.elem_table);
+    P.off_out = off; if (P.host_outputs) off = align_up(off + P.B * P.out_bytes_per_proof);
+    P.total = off;
+    return BZK_OK;
+}
+
+bzk_status ensure_ws(bzk_ctx *ctx, size_t bytes) {
+    if (ctx->ws_size >= bytes) return BZK_OK;
+    if (ctx->ws) { cudaFree(ctx->ws); ctx->ws = nullptr; ctx->ws_size = 0; }
+    cudaError_t e = cudaMalloc(&ctx->ws, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ctx, BZK_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(e));
+    }
+    ctx->ws_size = bytes;
+    return BZK_OK;
+}
+
+// ---------------------------------------------------------------- kernel dispatch
+
+cudaError_t dispatch_round(uint32_t D, uint32_t order, bool first, dim3 grid, cudaStream_t s,
+                           const RoundParams &p) {
+    switch (D) {
+        case 1: return launch_round<1>(order, first, grid, kThreads, s, p);
+        case 2: return launch_round<2>(order, first, grid, kThreads, s, p);
+        case 3: return launch_round<3>(order, first, grid, kThreads, s, p);
+        case 4: return launch_round<4>(order, first, grid, kThreads, s, p);
+    }
+    return cudaErrorInvalidValue;
+}
+
+cudaError_t dispatch_tail(uint32_t D, uint32_t order, uint32_t grid, size_t smem, cudaStream_t s,
+                          const TailParams &p) {
+    switch (D) {
+        case 1: return launch_tail<1>(order, grid, kThreads, smem, s, p);
+        case 2: return launch_tail<2>(order, grid, kThreads, smem, s, p);
+        case 3: return launch_tail<3>(order, grid, kThreads, smem, s, p);
+        case 4: return launch_tail<4>(order, grid, kThreads, smem, s, p);
+    }
+    return cudaErrorInvalidValue;
+}
+
+__global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        fe v = ld_fe(t + i);
+        if (!fe_is_canon(v)) atomicOr(flag, 1u);
+    }
+}
+
+// ---------------------------------------------------------------- one wave
+
+struct WaveIO {
+    fe *tables;        // device tables of this wave [nb][D][N]
+    fe *round_evals, *challenges, *final_evals, *claims;   // device outputs of this wave
+    uint64_t nb, first_index;
+};
+
+bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
+    char *ws = (char *)ctx->ws;
+    ProofState *ps = (ProofState *)(ws + P.off_ps);
+    uint32_t *tick = (uint32_t *)(ws + P.off_tick);
+    fe *part = (fe *)(ws + P.off_part);
+    fe *bufX = (fe *)(ws + P.off_bufX);
+    fe *bufY = P.bufY_alias_input ? io.tables : (fe *)(ws + P.off_bufY);
+    const uint8_t *seed = (const uint8_t *)(ws + P.off_seed);
+    const uint32_t D = P.D, k = P.k;
+    {
+        ProfScope ps_(ctx, s, 3);
+        k_transcript_init<<<(uint32_t)((io.nb + 127) / 128), 128, 0, s>>>(ps, (uint32_t)io.nb, seed,
+                                                                          io.first_index, k, D, P.order);
+        ++ctx->launches;
+        CK(cudaGetLastError());
+    }
+    for (uint32_t i = 1; i < P.i0; ++i) {
+        RoundParams rp;
+        memset(&rp, 0, sizeof rp);
+        rp.log_h = k - i;
+        rp.round = i; rp.k = k; rp.order = P.order;
+        const uint64_t h = 1ull << rp.log_h;
+        rp.ctas = ctas_for(h, io.nb);
+        rp.partials = part; rp.tickets = tick; rp.ps = ps;
+        rp.round_evals = io.round_evals; rp.challenges = io.challenges; rp.claims = io.claims;
+        rp.seed = seed; rp.first_index = io.first_index;
+        if (i == 1) { rp.src = io.tables; rp.dst = nullptr; }
+        else {
+            rp.src = (i == 2) ? io.tables : ((i - 1) % 2 == 0 ? bufX : bufY);
+            rp.dst = (i % 2 == 0) ? bufX : bufY;
+        }
+        dim3 grid(rp.ctas, (uint32_t)io.nb);
+        ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
+        cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp);
+        ++ctx->launches;
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
+    }
+    {
+        TailParams tp;
+        memset(&tp, 0, sizeof tp);
+        tp.i0 = P.i0; tp.log_h0 = P.log_h0; tp.k = k; tp.order = P.order; tp.ps = ps;
+        tp.round_evals = io.round_evals; tp.challenges = io.challenges;
+        tp.final_evals = io.final_evals; tp.claims = io.claims;
+        if (P.i0 <= 2) tp.src = io.tables;
+        else tp.src = ((P.i0 - 1) % 2 == 0) ? bufX : bufY;
+        size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 32;
+        ProfScope ps_(ctx, s, 2);
+        cudaError_t e = dispatch_tail(D, P.order, (uint32_t)io.nb, smem, s, tp);
+        ++ctx->launches;
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "k_tail launch");
+    }
+    return BZK_OK;
+}
+
+bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
+    bzk_status st = validate_args(ctx, b);
+    if (st) return st;
+    Plan P;
+    st = make_plan(ctx, b, P);
+    if (st) return st;
+    st = ensure_ws(ctx, P.total);
+    if (st) return st;
+    char *ws = (char *)ctx->ws;
+    CK(cudaMemcpyAsync(ws + P.off_seed, b->seed, 32, cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(ws + P.off_tick, 0, P.Bw * 4, s));
+    const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
+    if (validate) CK(cudaMemsetAsync(ctx->d_flag, 0, 4, s));
+
+    const size_t opp = P.out_bytes_per_proof;
+    const size_t ev_pp = (size_t)P.k * (P.D + 1), ch_pp = P.k, fi_pp = P.D;
+    fe *o_ev, *o_ch, *o_fi, *o_cl;
+    if (P.host_outputs) {
+        fe *base = (fe *)(ws + P.off_out);
+        o_ev = base; o_ch = o_ev + P.B * ev_pp; o_fi = o_ch + P.B * ch_pp; o_cl = o_fi + P.B * fi_pp;
+    } else {
+        o_ev = (fe *)b->round_evals; o_ch = (fe *)b->challenges; o_fi = (fe *)b->final_evals;
+        o_cl = (fe *)b->claims;
+    }
+    (void)opp;
+    for (uint64_t w = 0; w < P.nwaves; ++w) {
+        WaveIO io;
+        const uint64_t b0 = w * P.Bw;
+        io.nb = std::min<uint64_t>(P.Bw, P.B - b0);
+        io.first_index = b->first_index + b0;
+        io.round_evals = o_ev + b0 * ev_pp;
+        io.challenges = o_ch + b0 * ch_pp;
+        io.final_evals = o_fi + b0 * fi_pp;
+        io.claims = (P.host_outputs || o_cl) ? o_cl + b0 : nullptr;
+        if (P.host_tables) {
+            // loader: wave w's tables -> staging[w % 2] on the copy stream, overlapping wave w-1
+            const int slot = (int)(w % 2);
+            fe *stage = (fe *)(ws + (slot ? P.off_stage1 : P.off_stage0));
+            if (w >= 2) CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
+
+            {
+                ProfScope ps_(ctx, ctx->copy_stream, 5);
+                CK(cudaMemcpyAsync(stage, (const char *)b->tables + b0 * P.elem_table, io.nb * P.elem_table,
+                                   cudaMemcpyHostToDevice, ctx->copy_stream));
+            }
+            CK(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
+            CK(cudaStreamWaitEvent(s, ctx->ev_copied[slot], 0));
+            io.tables = stage;
+        } else {
+            io.tables = (fe *)((char *)b->tables + b0 * P.elem_table);
+        }
+        if (validate) {
+            ProfScope ps_(ctx, s, 4);
+            k_validate<<<kSMs * 8, 256, 0, s>>>(io.tables, io.nb * P.D * P.N, ctx->d_flag);
+            ++ctx->launches;
+            CK(cudaGetLastError());
+        }
+        st = run_wave(ctx, P, io, s);
+        if (st) return st;
+        if (P.host_tables) CK(cudaEventRecord(ctx->ev_consumed[w % 2], s));
+    }
+    if (P.host_outputs) {
+        if (P.k) {
+            CK(cudaMemcpyAsync(b->round_evals, o_ev, P.B * ev_pp * 32, cudaMemcpyDeviceToHost, s));
+            CK(cudaMemcpyAsync(b->challenges, o_ch, P.B * ch_pp * 32, cudaMemcpyDeviceToHost, s));
+        }
+        CK(cudaMemcpyAsync(b->final_evals, o_fi, P.B * fi_pp * 32, cudaMemcpyDeviceToHost, s));
+        if (b->claims) CK(cudaMemcpyAsync(b->claims, o_cl, P.B * 32, cudaMemcpyDeviceToHost, s));
+    }
+    if (validate) {
+        uint32_t flag = 0;
+        CK(cudaMemcpyAsync(&flag, ctx->d_flag, 4, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (flag) return fail(ctx, BZK_ENONCANON, "an input element is >= p");
+    }
+    if ((b->flags & BZK_F_SYNC) || P.host_outputs || P.host_tables) CK(cudaStreamSynchronize(s));
+    return BZK_OK;
+}
+
+// ---------------------------------------------------------------- debug kernels
+
+__global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *out) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        fe x = ld_fe(a + i), r;
+        switch (op) {
+            case 0: r = fe_add(x, ld_fe(b + i)); break;
+            case 1: r = fe_sub(x, ld_fe(b + i)); break;
+            case 2: r = mont_mul(x, ld_fe(b + i)); break;
+            case 3: r = mont_mul(mont_mul(x, ld_fe(b + i)), fe_const(2)); break;
+            default: r = fe_reduce_256(x); break;
+        }
+        st_fe(out + i, r);
+    }
+}
+
+__global__ void k_debug_sha256(const uint8_t *msgs, uint32_t len, uint64_t n, uint8_t *out) {
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint8_t *m = msgs + i * len;
+    sha256_words sh;
+    sh.init();
+    for (uint32_t w = 0; w < len / 4; ++w)
+        sh.push(((uint32_t)m[4 * w] << 24) | ((uint32_t)m[4 * w + 1] << 16) | ((uint32_t)m[4 * w + 2] << 8) |
+                (uint32_t)m[4 * w + 3]);
+    uint32_t h[8];
+    sh.finish(h);
+    for (int j = 0; j < 8; ++j) {
+        out[i * 32 + 4 * j] = (uint8_t)(h[j] >> 24);
+        out[i * 32 + 4 * j + 1] = (uint8_t)(h[j] >> 16);
+        out[i * 32 + 4 * j + 2] = (uint8_t)(h[j] >> 8);
+        out[i * 32 + 4 * j + 3] = (uint8_t)h[j];
+    }
+}
+
+// 8 independent IMAD chains per thread; returns cycles in out[block]
+__global__ void k_imad_rate(uint32_t iters, uint32_t seed, unsigned long long *cycles, uint32_t *sink) {
+    uint32_t a0 = seed ^ threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5,
+             a6 = a0 + 6, a7 = a0 + 7;
+    const uint32_t x = seed | 1, y = seed >> 3;
+    __syncthreads();
+    unsigned long long t0 = clock64();
+    for (uint32_t it = 0; it < iters; ++it) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            asm volatile("mad.lo.u32 %0, %0, %8, %9;\n\t"
+                         "mad.lo.u32 %1, %1, %8, %9;\n\t"
+                         "mad.lo.u32 %2, %2, %8, %9;\n\t"
+                         "mad.lo.u32 %3, %3, %8, %9;\n\t"
+                         "mad.lo.u32 %4, %4, %8, %9;\n\t"
+                         "mad.lo.u32 %5, %5, %8, %9;\n\t"
+                         "mad.lo.u32 %6, %6, %8, %9;\n\t"
+                         "mad.lo.u32 %7, %7, %8, %9;"
+                         : "+r"(a0), "+r"(a1), "+r"(a2), "+r"(a3), "+r"(a4), "+r"(a5), "+r"(a6), "+r"(a7)
+                         : "r"(x), "r"(y));
+        }
+    }
+    __syncthreads();
+    unsigned long long t1 = clock64();
+    if (threadIdx.x == 0) cycles[blockIdx.x] = t1 - t0;
+    sink[blockIdx.x * blockDim.x + threadIdx.x] = a0 ^ a1 ^ a2 ^ a3 ^ a4 ^ a5 ^ a6 ^ a7;
+}
+
+}  // namespace
+
+// ==================================================================== C ABI
+
+extern "C" {
+
+const char *bzk_version(void) { return "bzk 0.1 sm_100a (BN254 Fr, SHA-256 Fiat-Shamir)"; }
+
+const char *bzk_strerror(bzk_status s) {
+    switch (s) {
+        case BZK_OK: return "ok";
+        case BZK_EINVAL: return "invalid argument";
+        case BZK_ENOMEM: return "out of device memory / workspace limit";
+        case BZK_ECUDA: return "CUDA error";
+        case BZK_ENONCANON: return "non-canonical input element";
+        case BZK_EUNSUPPORTED: return "unsupported";
+    }
+    return "unknown status";
+}
+
+const char *bzk_last_error(const bzk_ctx *ctx) { return ctx ? ctx->last_error.c_str() : ""; }
+
+bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
+    if (!out) return BZK_EINVAL;
+    *out = nullptr;
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0) return BZK_ECUDA;
+    if (device < 0 || device >= n) return BZK_EINVAL;
+    e = cudaSetDevice(device);
+    if (e != cudaSuccess) return BZK_ECUDA;
+    bzk_ctx *ctx = new bzk_ctx();
+    ctx->device = device;
+    ctx->workspace_limit = workspace_limit;
+    cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device);
+    if (cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaMalloc(&ctx->d_flag, 4) != cudaSuccess) {
+        delete ctx;
+        return BZK_ECUDA;
+    }
+    for (int i = 0; i < 2; ++i) {
+        cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&ctx->ev_consumed[i], cudaEventDisableTiming);
+    }
+    *out = ctx;
+    return BZK_OK;
+}
+
+void bzk_destroy(bzk_ctx *ctx) {
+    if (!ctx) return;
+    cudaSetDevice(ctx->device);
+    cudaDeviceSynchronize();
+    if (ctx->ws) cudaFree(ctx->ws);
+    if (ctx->d_flag) cudaFree(ctx->d_flag);
+    for (int i = 0; i < 2; ++i) {
+        if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+        if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
+    }
+    for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+    if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
+    delete ctx;
+}
+
+bzk_status bzk_workspace_size(bzk_ctx *ctx, const bzk_batch *batch, size_t *bytes) {
+    if (!ctx || !bytes) return BZK_EINVAL;
+    bzk_status st = validate_args(ctx, batch);
+    if (st) return st;
+    Plan P;
+    st = make_plan(ctx, batch, P);
+    if (st) return st;
+    *bytes = P.total;
+    return BZK_OK;
+}
+
+bzk_status bzk_prove(bzk_ctx *ctx, const bzk_batch *batch, void *cuda_stream) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    return prove_impl(ctx, batch, (cudaStream_t)cuda_stream);
+}
+
+bzk_status bzk_prove_ragged(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, void *cuda_stream) {
+    if (!ctx || (!jobs && njobs)) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    for (size_t j = 0; j < njobs; ++j) {
+        bzk_status st = validate_args(ctx, &jobs[j]);
+        if (st) return fail(ctx, st, "job " + std::to_string(j) + ": " + ctx->last_error);
+    }
+    for (size_t j = 0; j < njobs; ++j) {
+        bzk_status st = prove_impl(ctx, &jobs[j], (cudaStream_t)cuda_stream);
+        if (st) return st;
+    }
+    return BZK_OK;
+}
+
+bzk_status bzk_sync(bzk_ctx *ctx) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "bzk_sync");
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "bzk_sync");
+    return BZK_OK;
+}
+
+bzk_status bzk_generate(uint64_t *dst, uint64_t batch, uint32_t d, uint32_t k, uint64_t first_index,
+                        uint32_t dist, uint64_t data_seed, void *cuda_stream) {
+    if (!dst || k > 30 || d < 1 || d > 15 || dist > 2 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
+    k_generate<<<kSMs * 16, 256, 0, (cudaStream_t)cuda_stream>>>(dst, batch, d, k, first_index, dist, data_seed);
+    return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+}
+
+bzk_status bzk_profile_enable(bzk_ctx *ctx, int on) {
+    if (!ctx) return BZK_EINVAL;
+    ctx->prof = on != 0;
+    return BZK_OK;
+}
+
+bzk_status bzk_profile_read(bzk_ctx *ctx, double ms[BZK_PROF_KINDS], uint64_t count[BZK_PROF_KINDS], int reset) {
+    if (!ctx || !ms || !count) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "bzk_profile_read");
+    for (int i = 0; i < BZK_PROF_KINDS; ++i) { ms[i] = 0; count[i] = 0; }
+    for (auto &r : ctx->recs) {
+        float t = 0;
+        cudaEventElapsedTime(&t, r.a, r.b);
+        if (r.kind >= 0 && r.kind < BZK_PROF_KINDS) { ms[r.kind] += t; count[r.kind] += 1; }
+    }
+    if (reset) {
+        for (auto &r : ctx->recs) { ctx->ev_pool.push_back(r.a); ctx->ev_pool.push_back(r.b); }
+        ctx->recs.clear();
+    }
+    return BZK_OK;
+}
+
+uint64_t bzk_launch_count(bzk_ctx *ctx, int reset) {
+    if (!ctx) return 0;
+    uint64_t n = ctx->launches;
+    if (reset) ctx->launches = 0;
+    return n;
+}
+
+bzk_status bzk_debug_field(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out,
+                           void *cuda_stream) {
+    if (op < 0 || op > 4 || !a || !out || (op < 4 && !b)) return BZK_EINVAL;
+    if (n == 0) return BZK_OK;
+    k_debug_field<<<kSMs * 8, 256, 0, (cudaStream_t)cuda_stream>>>(op, n, (const fe *)a, (const fe *)b, (fe *)out);
+    return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+}
+
+bzk_status bzk_debug_sha256(const uint8_t *msgs, uint32_t msg_len, uint64_t n, uint8_t *out, void *cuda_stream) {
+    if (!msgs || !out || msg_len % 4) return BZK_EINVAL;
+    if (n == 0) return BZK_OK;
+    k_debug_sha256<<<(uint32_t)((n + 127) / 128), 128, 0, (cudaStream_t)cuda_stream>>>(msgs, msg_len, n, out);
+    return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+}
+
+bzk_status bzk_debug_imad_rate(uint32_t iters, double *rate, void *cuda_stream) {
+    if (!rate || iters == 0) return BZK_EINVAL;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    int nsm = kSMs;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+    const int blocks = nsm * 2, threads = 512;
+    unsigned long long *cyc = nullptr;
+    uint32_t *sink = nullptr;
+    if (cudaMalloc(&cyc, blocks * sizeof(unsigned long long)) != cudaSuccess) return BZK_ENOMEM;
+    if (cudaMalloc(&sink, (size_t)blocks * threads * 4) != cudaSuccess) { cudaFree(cyc); return BZK_ENOMEM; }
+    k_imad_rate<<<blocks, threads, 0, s>>>(iters, 12345u, cyc, sink);
+    std::vector<unsigned long long> h(blocks);
+    cudaMemcpyAsync(h.data(), cyc, blocks * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s);
+    cudaError_t e = cudaStreamSynchronize(s);
+    cudaFree(cyc);
+    cudaFree(sink);
+    if (e != cudaSuccess) return BZK_ECUDA;
+    std::sort(h.begin(), h.end());
+    const double med = (double)h[blocks / 2];
+    // 2 co-resident blocks per SM, each threads x iters x 32 IMAD
+    *rate = 2.0 * threads * (double)iters * 32.0 / med;
+    return BZK_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,311 @@
+// field.cuh -- BN254 scalar field F_p on sm_100a: 8 x 32-bit limbs, Montgomery CIOS on
+// 32-bit IMAD carry chains (mad.lo.cc / madc.hi.cc).
+//
+// Reading R1: the paper fixes 256-bit elements (PAPER.md:187 Sec. 3.3, :320
+// Sec. 6.2) but never names the prime; we take BN254 Fr.
+//
+// Representation conventions used by the kernels:
+//   * tables and every value that leaves the library are in STANDARD form, canonical (< p);
+//   * challenges are held in MONTGOMERY form (r*R mod p, R = 2^256) so that
+//     mont_mul(r*R, x) = r*x: the fold T' = a + r(b - a) stays in standard form with ONE
+//     mont_mul and no conversion pass;
+//   * a product of d standard values through d-1 mont_muls carries R^{-(d-1)}; round sums
+//     are fixed once per round by mont_mul(S, R^d mod p).
+#pragma once
+#include <stdint.h>
+
+namespace bzk {
+
+struct fe { uint32_t l[8]; };
+
+// p = 0x30644e72e131a029b85045b68181585d2833e84879b9709143e1f593f0000001 (LE 32-bit limbs)
+#define BZK_P0 0xf0000001u
+#define BZK_P1 0x43e1f593u
+#define BZK_P2 0x79b97091u
+#define BZK_P3 0x2833e848u
+#define BZK_P4 0x8181585du
+#define BZK_P5 0xb85045b6u
+#define BZK_P6 0xe131a029u
+#define BZK_P7 0x30644e72u
+#define BZK_NP0 0xefffffffu   // -p^{-1} mod 2^32
+
+// Constants in standard form (LE limbs), derived in DESIGN.md App. A and checked on the host
+// by tests/test_abi.py against Python integers (bzk_debug_constants).
+//   R mod p, R^2 mod p, R^3 mod p, R^4 mod p, R^5 mod p
+__device__ __forceinline__ fe fe_const(int which);
+
+__device__ __forceinline__ fe fe_zero() { fe r; _Pragma("unroll") for (int i = 0; i < 8; ++i) r.l[i] = 0; return r; }
+
+__device__ __forceinline__ bool fe_is_zero(const fe &a) {
+    uint32_t x = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x |= a.l[i];
+    return x == 0;
+}
+
+// r = a - p (with borrow out); returns borrow (1 if a < p)
+__device__ __forceinline__ uint32_t sub_p(fe &r, const fe &a) {
+    uint32_t borrow;
+    asm("sub.cc.u32  %0, %9,  %17;\n\t"
+        "subc.cc.u32 %1, %10, %18;\n\t"
+        "subc.cc.u32 %2, %11, %19;\n\t"
+        "subc.cc.u32 %3, %12, %20;\n\t"
+        "subc.cc.u32 %4, %13, %21;\n\t"
+        "subc.cc.u32 %5, %14, %22;\n\t"
+        "subc.cc.u32 %6, %15, %23;\n\t"
+        "subc.cc.u32 %7, %16, %24;\n\t"
+        "subc.u32    %8, 0, 0;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]),
+          "=r"(r.l[6]), "=r"(r.l[7]), "=r"(borrow)
+        : "r"(a.l[0]), "r"(a.l[1]), "r"(a.l[2]), "r"(a.l[3]), "r"(a.l[4]), "r"(a.l[5]), "r"(a.l[6]),
+          "r"(a.l[7]), "n"(BZK_P0), "n"(BZK_P1), "n"(BZK_P2), "n"(BZK_P3), "n"(BZK_P4), "n"(BZK_P5),
+          "n"(BZK_P6), "n"(BZK_P7));
+    return borrow;   // 0xffffffff if a < p, else 0
+}
+
+// a mod p for a < 2p
+__device__ __forceinline__ fe fe_reduce_once(const fe &a) {
+    fe s;
+    uint32_t borrow = sub_p(s, a);
+    fe r;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) r.l[i] = borrow ? a.l[i] : s.l[i];
+    return r;
+}
+
+// (a + b) mod p for canonical a, b (a + b < 2p < 2^255: no carry out of 256 bits)
+__device__ __forceinline__ fe fe_add(const fe &a, const fe &b) {
+    fe s;
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(s.l[0]), "=r"(s.l[1]), "=r"(s.l[2]), "=r"(s.l[3]), "=r"(s.l[4]), "=r"(s.l[5]),
+          "=r"(s.l[6]), "=r"(s.l[7])
+        : "r"(a.l[0]), "r"(a.l[1]), "r"(a.l[2]), "r"(a.l[3]), "r"(a.l[4]), "r"(a.l[5]), "r"(a.l[6]),
+          "r"(a.l[7]), "r"(b.l[0]), "r"(b.l[1]), "r"(b.l[2]), "r"(b.l[3]), "r"(b.l[4]), "r"(b.l[5]),
+          "r"(b.l[6]), "r"(b.l[7]));
+    return fe_reduce_once(s);
+}
+
+// (a - b) mod p for canonical a, b
+__device__ __forceinline__ fe fe_sub(const fe &a, const fe &b) {
+    fe s;
+    uint32_t borrow;
+    asm("sub.cc.u32  %0, %9,  %17;\n\t"
+        "subc.cc.u32 %1, %10, %18;\n\t"
+        "subc.cc.u32 %2, %11, %19;\n\t"
+        "subc.cc.u32 %3, %12, %20;\n\t"
+        "subc.cc.u32 %4, %13, %21;\n\t"
+        "subc.cc.u32 %5, %14, %22;\n\t"
+        "subc.cc.u32 %6, %15, %23;\n\t"
+        "subc.cc.u32 %7, %16, %24;\n\t"
+        "subc.u32    %8, 0, 0;"
+        : "=r"(s.l[0]), "=r"(s.l[1]), "=r"(s.l[2]), "=r"(s.l[3]), "=r"(s.l[4]), "=r"(s.l[5]),
+          "=r"(s.l[6]), "=r"(s.l[7]), "=r"(borrow)
+        : "r"(a.l[0]), "r"(a.l[1]), "r"(a.l[2]), "r"(a.l[3]), "r"(a.l[4]), "r"(a.l[5]), "r"(a.l[6]),
+          "r"(a.l[7]), "r"(b.l[0]), "r"(b.l[1]), "r"(b.l[2]), "r"(b.l[3]), "r"(b.l[4]), "r"(b.l[5]),
+          "r"(b.l[6]), "r"(b.l[7]));
+    // add back p masked by the borrow
+    uint32_t m0 = BZK_P0 & borrow, m1 = BZK_P1 & borrow, m2 = BZK_P2 & borrow, m3 = BZK_P3 & borrow;
+    uint32_t m4 = BZK_P4 & borrow, m5 = BZK_P5 & borrow, m6 = BZK_P6 & borrow, m7 = BZK_P7 & borrow;
+    asm("add.cc.u32  %0, %0, %8;\n\t"
+        "addc.cc.u32 %1, %1, %9;\n\t"
+        "addc.cc.u32 %2, %2, %10;\n\t"
+        "addc.cc.u32 %3, %3, %11;\n\t"
+        "addc.cc.u32 %4, %4, %12;\n\t"
+        "addc.cc.u32 %5, %5, %13;\n\t"
+        "addc.cc.u32 %6, %6, %14;\n\t"
+        "addc.u32    %7, %7, %15;"
+        : "+r"(s.l[0]), "+r"(s.l[1]), "+r"(s.l[2]), "+r"(s.l[3]), "+r"(s.l[4]), "+r"(s.l[5]),
+          "+r"(s.l[6]), "+r"(s.l[7])
+        : "r"(m0), "r"(m1), "r"(m2), "r"(m3), "r"(m4), "r"(m5), "r"(m6), "r"(m7));
+    return s;
+}
+
+// t[0..9] += a[0..7] * b   (even-index products on one carry chain, odd on another)
+__device__ __forceinline__ void mad_row(uint32_t t[10], const uint32_t a[8], uint32_t b) {
+    asm("mad.lo.cc.u32  %0, %10, %18, %0;\n\t"
+        "madc.hi.cc.u32 %1, %10, %18, %1;\n\t"
+        "madc.lo.cc.u32 %2, %12, %18, %2;\n\t"
+        "madc.hi.cc.u32 %3, %12, %18, %3;\n\t"
+        "madc.lo.cc.u32 %4, %14, %18, %4;\n\t"
+        "madc.hi.cc.u32 %5, %14, %18, %5;\n\t"
+        "madc.lo.cc.u32 %6, %16, %18, %6;\n\t"
+        "madc.hi.cc.u32 %7, %16, %18, %7;\n\t"
+        "addc.cc.u32    %8, %8, 0;\n\t"
+        "addc.u32       %9, %9, 0;\n\t"
+        "mad.lo.cc.u32  %1, %11, %18, %1;\n\t"
+        "madc.hi.cc.u32 %2, %11, %18, %2;\n\t"
+        "madc.lo.cc.u32 %3, %13, %18, %3;\n\t"
+        "madc.hi.cc.u32 %4, %13, %18, %4;\n\t"
+        "madc.lo.cc.u32 %5, %15, %18, %5;\n\t"
+        "madc.hi.cc.u32 %6, %15, %18, %6;\n\t"
+        "madc.lo.cc.u32 %7, %17, %18, %7;\n\t"
+        "madc.hi.cc.u32 %8, %17, %18, %8;\n\t"
+        "addc.u32       %9, %9, 0;"
+        : "+r"(t[0]), "+r"(t[1]), "+r"(t[2]), "+r"(t[3]), "+r"(t[4]), "+r"(t[5]), "+r"(t[6]),
+          "+r"(t[7]), "+r"(t[8]), "+r"(t[9])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(a[4]), "r"(a[5]), "r"(a[6]), "r"(a[7]),
+          "r"(b));
+}
+
+// t[0..9] += p * m
+__device__ __forceinline__ void mad_row_p(uint32_t t[10], uint32_t m) {
+    asm("mad.lo.cc.u32  %0, %11, %10, %0;\n\t"
+        "madc.hi.cc.u32 %1, %11, %10, %1;\n\t"
+        "madc.lo.cc.u32 %2, %13, %10, %2;\n\t"
+        "madc.hi.cc.u32 %3, %13, %10, %3;\n\t"
+        "madc.lo.cc.u32 %4, %15, %10, %4;\n\t"
+        "madc.hi.cc.u32 %5, %15, %10, %5;\n\t"
+        "madc.lo.cc.u32 %6, %17, %10, %6;\n\t"
+        "madc.hi.cc.u32 %7, %17, %10, %7;\n\t"
+        "addc.cc.u32    %8, %8, 0;\n\t"
+        "addc.u32       %9, %9, 0;\n\t"
+        "mad.lo.cc.u32  %1, %12, %10, %1;\n\t"
+        "madc.hi.cc.u32 %2, %12, %10, %2;\n\t"
+        "madc.lo.cc.u32 %3, %14, %10, %3;\n\t"
+        "madc.hi.cc.u32 %4, %14, %10, %4;\n\t"
+        "madc.lo.cc.u32 %5, %16, %10, %5;\n\t"
+        "madc.hi.cc.u32 %6, %16, %10, %6;\n\t"
+        "madc.lo.cc.u32 %7, %18, %10, %7;\n\t"
+        "madc.hi.cc.u32 %8, %18, %10, %8;\n\t"
+        "addc.u32       %9, %9, 0;"
+        : "+r"(t[0]), "+r"(t[1]), "+r"(t[2]), "+r"(t[3]), "+r"(t[4]), "+r"(t[5]), "+r"(t[6]),
+          "+r"(t[7]), "+r"(t[8]), "+r"(t[9])
+        : "r"(m), "r"(BZK_P0), "r"(BZK_P1), "r"(BZK_P2), "r"(BZK_P3), "r"(BZK_P4), "r"(BZK_P5),
+          "r"(BZK_P6), "r"(BZK_P7));
+}
+
+// Montgomery product a*b*R^{-1} mod p (CIOS), a, b canonical -> canonical.
+__device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
+    uint32_t t[10];
+#pragma unroll
+    for (int i = 0; i < 10; ++i) t[i] = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        mad_row(t, a.l, b.l[i]);
+        uint32_t m = t[0] * BZK_NP0;
+        mad_row_p(t, m);
+        // t[0] == 0 now; shift down one limb
+#pragma unroll
+        for (int j = 0; j < 9; ++j) t[j] = t[j + 1];
+        t[9] = 0;
+    }
+    fe r;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) r.l[i] = t[i];
+    return fe_reduce_once(r);   // t < 2p for canonical inputs
+}
+
+__device__ __forceinline__ fe fe_const(int which) {
+    fe r;
+    switch (which) {
+        case 1: {  // R mod p
+            const uint32_t v[8] = {0x4ffffffbu, 0xac96341cu, 0x9f60cd29u, 0x36fc7695u,
+                                   0x7879462eu, 0x666ea36fu, 0x9a07df2fu, 0x0e0a77c1u};
+            _Pragma("unroll") for (int i = 0; i < 8; ++i) r.l[i] = v[i];
+            break;
+        }
+        case 2: {  // R^2 mod p
+            const uint32_t v[8] = {0xae216da7u, 0x1bb8e645u, 0xe35c59e3u, 0x53fe3ab1u,
+                                   0x53bb8085u, 0x8c49833du, 0x7f4e44a5u, 0x0216d0b1u};
+            _Pragma("unroll") for (int i = 0; i < 8; ++i) r.l[i] = v[i];
+            break;
+        }
+        case 3: {  // R^3 mod p
+            const uint32_t v[8] = {0xb4bf0040u, 0x5e94d8e1u, 0x1cfbb6b8u, 0x2a489cbeu,
+                                   0xa19fcfedu, 0x893cc664u, 0x7fcc657cu, 0x0cf8594bu};
+            _Pragma("unroll") for (int i = 0; i < 8; ++i) r.l[i] = v[i];
+            break;
+        }
+        default: r = fe_zero(); r.l[0] = 1; break;
+    }
+    return r;
+}
+
+// x^e for small fixed powers of R: R^d mod p = mont_mul chain of R^2 and R^3 (computed once per use)
+//   R^4 = mont_mul(R^3, R^2);  R^5 = mont_mul(R^4, R^2)  (mont_mul(R^a, R^b) = R^{a+b-1})
+__device__ __forceinline__ fe fe_R_pow(int d) {
+    if (d <= 1) return fe_const(1);
+    if (d == 2) return fe_const(2);
+    if (d == 3) return fe_const(3);
+    fe r = fe_const(3);
+    for (int e = 3; e < d; ++e) r = mont_mul(r, fe_const(2));
+    return r;
+}
+
+// canonicalise an arbitrary 256-bit value (< 2^256 < 6p): subtract p up to 5 times
+__device__ __forceinline__ fe fe_reduce_256(const fe &a) {
+    fe r = a;
+#pragma unroll 1
+    for (int it = 0; it < 6; ++it) {
+        fe s;
+        uint32_t borrow = sub_p(s, r);
+        if (borrow) break;
+        r = s;
+    }
+    return r;
+}
+
+__device__ __forceinline__ bool fe_is_canon(const fe &a) {
+    fe s;
+    return sub_p(s, a) != 0;
+}
+
+// ---------------------------------------------------------------- memory helpers
+
+// 32-byte element load/store as two 128-bit accesses (coalesced across a warp)
+__device__ __forceinline__ fe ld_fe(const fe *p) {
+    const uint4 *q = reinterpret_cast<const uint4 *>(p);
+    uint4 x = __ldg(q), y = __ldg(q + 1);
+    fe r;
+    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
+    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+    return r;
+}
+
+// streaming (evict-first) load for data read exactly once
+__device__ __forceinline__ fe ld_fe_stream(const fe *p) {
+    const uint4 *q = reinterpret_cast<const uint4 *>(p);
+    uint4 x = __ldcs(q), y = __ldcs(q + 1);
+    fe r;
+    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
+    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+    return r;
+}
+
+// L2-coherent load (data written by other CTAs of the same launch)
+__device__ __forceinline__ fe ld_fe_cg(const fe *p) {
+    const uint4 *q = reinterpret_cast<const uint4 *>(p);
+    uint4 x = __ldcg(q), y = __ldcg(q + 1);
+    fe r;
+    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
+    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+    return r;
+}
+
+__device__ __forceinline__ void st_fe(fe *p, const fe &v) {
+    uint4 *q = reinterpret_cast<uint4 *>(p);
+    q[0] = make_uint4(v.l[0], v.l[1], v.l[2], v.l[3]);
+    q[1] = make_uint4(v.l[4], v.l[5], v.l[6], v.l[7]);
+}
+
+__device__ __forceinline__ void st_fe_cg(fe *p, const fe &v) {
+    uint4 *q = reinterpret_cast<uint4 *>(p);
+    __stcg(q, make_uint4(v.l[0], v.l[1], v.l[2], v.l[3]));
+    __stcg(q + 1, make_uint4(v.l[4], v.l[5], v.l[6], v.l[7]));
+}
+
+__device__ __forceinline__ fe shfl_down_fe(const fe &v, int delta) {
+    fe r;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) r.l[i] = __shfl_down_sync(0xffffffffu, v.l[i], delta);
+    return r;
+}
+
+}  // namespace bzk

@@ -1,0 +1,33 @@
+// k_impl.cuh -- per-degree kernel instantiation; included by k_d1.cu .. k_d4.cu with BZK_D set.
+#include "sumcheck.cuh"
+
+namespace bzk {
+
+template <>
+cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
+                                const RoundParams &p) {
+    if (order == 0) {
+        if (first) k_round<BZK_D, 0, true><<<grid, threads, 0, s>>>(p);
+        else       k_round<BZK_D, 0, false><<<grid, threads, 0, s>>>(p);
+    } else {
+        if (first) k_round<BZK_D, 1, true><<<grid, threads, 0, s>>>(p);
+        else       k_round<BZK_D, 1, false><<<grid, threads, 0, s>>>(p);
+    }
+    return cudaGetLastError();
+}
+
+template <>
+cudaError_t launch_tail<BZK_D>(uint32_t order, uint32_t grid, uint32_t threads, size_t smem, cudaStream_t s,
+                               const TailParams &p) {
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        attr_set = true;
+    }
+    if (order == 0) k_tail<BZK_D, 0><<<grid, threads, smem, s>>>(p);
+    else            k_tail<BZK_D, 1><<<grid, threads, smem, s>>>(p);
+    return cudaGetLastError();
+}
+
+}  // namespace bzk
