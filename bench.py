@@ -1,0 +1,360 @@
+#!/usr/bin/env python
+"""bench.py -- batched sum-check proofs/s on B200 (BASELINE.json metric), one JSON line.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c1|c3|m0] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (N > 1: one rank per GPU)
+
+A "step" is one bzk_prove call over the whole batch (every round of every proof: round-1 eval,
+fused fold+eval rounds, transcript hashing, on-chip tail, final fold).  Default workload =
+BASELINE.json configs[1]: 1024 proofs of a degree-2 product of two multilinear tables with 2^20
+BN254-Fr entries each (64 GiB of input, resident in HBM; PRESERVE mode so every step proves the
+same tables).  Multi-GPU: rank r proves global proofs [r*B, (r+1)*B) (weak scaling, no data-path
+collective; NCCL only gathers timings and output digests afterwards).
+
+Timing: W untimed warm-up steps, then K steps bracketed by barrier + cuda synchronize, CUDA events
+on the launch stream, max over ranks.  Inputs (64 GiB) are far larger than the 126 MB L2, so no
+flush is needed between steps.
+"""
+from __future__ import annotations
+
+import argparse
+import hashlib
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "sum-check proofs/s @2^20-entry tables, 1/2/4/8 B200; % of HBM/int roofline"
+
+CONFIGS = {
+    # name: (B per GPU, d, k, order, dist, description)
+    "c2": (1024, 2, 20, 0, "uniform", "configs[1]: 1024 proofs x product of 2 multilinears, k=20, BN254 Fr, "
+                                      "LSB order, tables resident in HBM"),
+    "c1": (16, 2, 12, 0, "uniform", "configs[0]: 16 proofs x d=2, k=12 (oracle-size case)"),
+    "c3": (256, 3, 22, 0, "uniform", "configs[2]: 256 GKR-layer-style proofs, degree-3 product f*g*h, k=22, "
+                                     "consume mode"),
+    "m0": (1024, 1, 20, 1, "uniform", "paper shape (Table 4 analogue): 1024 proofs x single multilinear (d=1), "
+                                      "k=20, MSB order = Alg. 1 pairing"),
+}
+
+# integer roof: 148 SMs x 64 IMAD/clk/SM (fma-heavy pipe, B300_MICROARCH.md
+# rt_SMSP = 2) x 1.965 GHz max SM clock; 272 IMAD per 256-bit Montgomery product (8-limb CIOS:
+# 2 n^2 + n = 136 32x32 products, lo + hi each)
+IMAD_PER_CLK_SM = 64
+SMS = 148
+IMAD_PER_MULMOD = 272
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            m = json.load(f)
+        return m.get("hbm_gbs", 6551.0), m.get("sm_max_mhz", 1965.0), "measured"
+    except OSError:
+        return 6650.0, 1965.0, "fallback"
+
+
+def alg_mulmods(d: int, k: int, kind: str) -> int:
+    """Algorithmic modular products per proof.
+
+    round 1 (eval only): (d+1)(d-1) per pair (all points t = 0..d; the claim is unknown);
+    fused round i >= 2: d * 2h fold products + d(d-1) per pair (g_i(1) = claim - g_i(0) derived);
+    the tail kernel covers the remaining rounds plus the final fold."""
+    tail_log = 8
+    i0 = 1 if k - 1 <= tail_log else k - tail_log
+    if kind == "round1":
+        return (d + 1) * (d - 1) * (1 << (k - 1)) if i0 > 1 else 0
+    if kind == "fused":
+        return sum(2 * d * (1 << (k - i)) + d * (d - 1) * (1 << (k - i)) for i in range(2, i0))
+    if kind == "total":
+        return d * d * ((1 << k) - 1)
+    raise ValueError(kind)
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region (B200_PROFILING.md recipe)."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        sm.sort()
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx or None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(cfg, max_proofs=8):
+    """The oracle as it stands on this box's host cores: a bounded sample of the same workload."""
+    import numpy as np  # noqa: F401
+
+    import oracle
+    from paper_conf_asplos_lucw0cz25_b200 import inputs
+    B, d, k, order, dist, _ = CONFIGS[cfg]
+    cores = len(os.sched_getaffinity(0))
+    n = max(1, min(max_proofs, cores, B))
+    tabs = inputs.gen_tables(n, d, k, 0, dist)
+    oracle.build()
+    t0 = time.perf_counter()
+    oracle.prove_batch(tabs, k, d, order, inputs.DEFAULT_SEED, 0, nthreads=n)
+    dt = time.perf_counter() - t0
+    return {"value": n / dt, "unit": "proofs/s", "cores": n, "kind": "oracle",
+            "sample": f"{n} proofs of {cfg} (d={d}, k={k}), one per thread, {dt:.1f} s wall"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle (this tier's reference arm), rank 0 only."""
+    if rank != 0:
+        return
+    B, d, k, order, dist, desc = CONFIGS[args.config]
+    for _ in range(args.warmup):
+        pass  # the oracle has no warm-up state; warm-up steps are not timed and not run
+    times = []
+    cb = None
+    for _ in range(args.steps):
+        cb = cpu_baseline(args.config, max_proofs=args.ref_proofs)
+        times.append(cb["cores"] / cb["value"])
+    nproofs = cb["cores"]
+    value = nproofs * len(times) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "proofs/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * sum(times) / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic", "config": {"workload": desc, "batch_sampled": nproofs, "d": d, "k": k},
+            "cpu_baseline": {"value": value, "unit": "proofs/s", "cores": nproofs, "kind": "oracle",
+                             "sample": cb["sample"]},
+            "e2e": {"value": value, "unit": "proofs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--batch", type=int, default=None, help="override proofs per GPU")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--ref-proofs", type=int, default=8)
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import numpy as np
+    import torch
+
+    from paper_conf_asplos_lucw0cz25_b200 import bzk
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    B, d, k, order, gen_dist, desc = CONFIGS[args.config]
+    if args.batch:
+        B = args.batch
+    first = rank * B
+    consume = args.config == "c3"
+    flags = 0 if consume else bzk.BZK_F_PRESERVE_INPUT
+    stream = torch.cuda.Stream()
+    tables = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
+    prover = bzk.Prover(local)
+    out = bzk.Prover.alloc_outputs(B, k, d)
+    batch = prover.batch(tables, k, d, order, None, first, flags, out)
+
+    def step():
+        if consume:
+            # consume mode destroys the input: regenerate it (untimed) before every step
+            bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
+        bzk.bzk_prove(prover.ctx, batch, stream)
+
+    for _ in range(args.warmup):
+        step()
+    stream.synchronize()
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    bzk.bzk_profile_enable(prover.ctx, True)
+    bzk.bzk_profile_read(prover.ctx, reset=True)
+    bzk.bzk_launch_count(prover.ctx, reset=True)
+    barrier()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            if consume:
+                bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
+            ev[i][0].record(stream)
+            bzk.bzk_prove(prover.ctx, batch, stream)
+            ev[i][1].record(stream)
+        stream.synchronize()
+        barrier()
+    launches = bzk.bzk_launch_count(prover.ctx, reset=True)
+    prof = bzk.bzk_profile_read(prover.ctx, reset=True)
+    bzk.bzk_profile_enable(prover.ctx, False)
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    my_ms = float(sum(step_ms))
+
+    # output digest (for cross-GPU-count comparisons) -- outside the timed region
+    h = hashlib.sha256()
+    for key in ("round_evals", "challenges", "final_evals", "claims"):
+        h.update(out[key].cpu().numpy().tobytes())
+    digest = h.hexdigest()
+
+    if dist:
+        t = torch.tensor([my_ms], dtype=torch.float64, device="cuda")
+        allt = [torch.zeros_like(t) for _ in range(world)]
+        dist.all_gather(allt, t)
+        max_ms = max(float(x.item()) for x in allt)
+        dg = torch.tensor(list(bytes.fromhex(digest)), dtype=torch.uint8, device="cuda")
+        alld = [torch.zeros_like(dg) for _ in range(world)]
+        dist.all_gather(alld, dg)
+        digests = [bytes(x.cpu().numpy()).hex() for x in alld]
+    else:
+        max_ms, digests = my_ms, [digest]
+
+    total_proofs = B * world * args.steps
+    value = total_proofs / (max_ms / 1000.0)
+    ms_per_step = max_ms / args.steps
+
+    # ---------------- roofline of the dominant kernel (ALU-bound: integer pipe)
+    hbm_peak, sm_max_mhz, peak_src = peaks()
+    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused"}
+    dom = max(kinds, key=lambda n: prof[n][0])
+    dom_ms, dom_cnt = prof[dom]
+    mulmods_per_launch = alg_mulmods(d, k, kinds[dom]) * B / max(1, dom_cnt / args.steps)
+    avg_launch_s = dom_ms / max(1, dom_cnt) / 1000.0
+    achieved = mulmods_per_launch / avg_launch_s / 1e9
+    int_peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6 / IMAD_PER_MULMOD / 1e9
+    total_alg = alg_mulmods(d, k, "total") * B
+    step_gmulmod = total_alg / (ms_per_step / 1000.0) / 1e9
+    # HBM: algorithmic bytes (read each input once) and the streaming schedule's bytes
+    alg_bytes = d * (1 << k) * 32 * B
+    roofline = {"bound": "alu", "kernel": dom, "achieved": round(achieved, 2), "peak": round(int_peak, 2),
+                "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": None,
+                "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} MHz "
+                               f"({peak_src} max clock) / {IMAD_PER_MULMOD} IMAD per mulmod",
+                "step_frac": round(step_gmulmod / int_peak, 4),
+                "hbm_alg_frac": round(alg_bytes / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
+                "hbm_peak_gbs": hbm_peak}
+
+    kernel_ms = {n: round(v[0] / args.steps, 3) for n, v in prof.items() if v[1]}
+    line = {"metric": METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": desc, "batch_per_gpu": B, "global_batch": B * world, "d": d, "k": k,
+                       "order": "LSB" if order == 0 else "MSB", "field": "BN254 Fr",
+                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * d * (1 << k) * 32 / 2**30)},
+            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
+            "kernel_ms_per_step": kernel_ms, "roofline": roofline, "clocks": clk.summary(),
+            "digest": digests[0], "digests_agree": len(set(digests)) == 1}
+
+    # ---------------- e2e: host (pinned) tables in, host outputs out, through bzk_prove
+    if not args.no_e2e and not consume:
+        del tables
+        torch.cuda.empty_cache()
+        host_t = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, pin_memory=True)
+        chunk = max(1, B // 16)
+        tmp = torch.empty((chunk, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+        for c0 in range(0, B, chunk):
+            n = min(chunk, B - c0)
+            bzk.bzk_generate(tmp, n, d, k, first + c0, gen_dist, stream=stream)
+            stream.synchronize()
+            host_t[c0:c0 + n].copy_(tmp[:n])
+        del tmp
+        torch.cuda.empty_cache()
+        out_h = bzk.Prover.alloc_outputs(B, k, d, device="cpu", pin=True)
+        hb = prover.batch(host_t, k, d, order, None, first, 0, out_h)
+        bzk.bzk_prove(prover.ctx, hb, stream)   # warm-up (allocates staging)
+        barrier()
+        t0 = time.perf_counter()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            bzk.bzk_prove(prover.ctx, hb, stream)   # host tables + host outputs: returns after D2H
+        e1.record(stream)
+        stream.synchronize()
+        barrier()
+        wall = time.perf_counter() - t0
+        e2e_ms = e0.elapsed_time(e1)
+        if dist:
+            t = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
+            allt = [torch.zeros_like(t) for _ in range(world)]
+            dist.all_gather(allt, t)
+            e2e_ms = max(float(x.item()) for x in allt)
+        out_bytes = sum(v.numel() * 8 for v in out_h.values())
+        same = all(torch.equal(out_h[key], out[key].cpu()) for key in out_h)
+        line["e2e"] = {"value": round(B * world * args.e2e_steps / (e2e_ms / 1000.0), 2), "unit": "proofs/s",
+                       "h2d_bytes_per_step": int(host_t.numel() * 8), "d2h_bytes_per_step": int(out_bytes),
+                       "steps": args.e2e_steps, "wall_s": round(wall, 3), "matches_device_run": bool(same),
+                       "path": "bzk_prove(tables_mem=HOST pinned, outputs_mem=HOST): side-stream H2D waves "
+                               "overlapping compute"}
+    if rank == 0 and world == 1 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(args.config)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    prover.close()
+    if dist:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

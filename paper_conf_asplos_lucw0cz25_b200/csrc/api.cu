@@ -167,6 +167,8 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     };
     const size_t fixed = 4096 + (P.host_outputs ? align_up(P.B * P.out_bytes_per_proof) : 0);
     uint64_t bw = std::min<uint64_t>(P.B, 65535);
+    // host tables: at least 8 loader waves so the H2D of wave w+1 overlaps the compute of wave w
+    if (P.host_tables && P.B >= 8) bw = std::min<uint64_t>(bw, (P.B + 7) / 8);
     while (bw > 1 && fixed + per_proof(bw) * bw + 8 * 256 > limit) bw = (bw + 1) / 2;
     if (fixed + per_proof(bw) * bw + 8 * 256 > limit)
         return fail(ctx, BZK_ENOMEM, "workspace_limit too small for one proof");
