@@ -28,7 +28,7 @@ PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", 
 
 EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
            "bzk_strerror", "bzk_last_error", "bzk_generate", "bzk_profile_enable", "bzk_profile_read",
-           "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_imad_rate", "bzk_version"]
+           "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version"]
 
 
 class BzkError(RuntimeError):
@@ -75,11 +75,11 @@ def lib():
         L.bzk_launch_count.restype = u64
         L.bzk_debug_field.argtypes = [i32, u64, vp, vp, vp, vp]
         L.bzk_debug_sha256.argtypes = [vp, u32, u64, vp, vp]
-        L.bzk_debug_imad_rate.argtypes = [u32, ctypes.POINTER(ctypes.c_double), vp]
+        L.bzk_debug_bench.argtypes = [i32, u32, ctypes.POINTER(ctypes.c_double), vp]
         L.bzk_version.restype = ctypes.c_char_p
         for name in ("bzk_create", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
                      "bzk_generate", "bzk_profile_enable", "bzk_profile_read", "bzk_debug_field",
-                     "bzk_debug_sha256", "bzk_debug_imad_rate"):
+                     "bzk_debug_sha256", "bzk_debug_bench"):
             getattr(L, name).restype = i32
         _lib = L
     return _lib
@@ -193,9 +193,10 @@ def bzk_debug_sha256(msgs, msg_len: int, n: int, out, stream=None) -> None:
     _check(lib().bzk_debug_sha256(ptr(msgs), msg_len, n, ptr(out), _stream_handle(stream)))
 
 
-def bzk_debug_imad_rate(iters: int = 4096, stream=None) -> float:
+def bzk_debug_bench(kind: int, iters: int = 4096, stream=None) -> float:
+    """ops per SM per clock: kind 0 IMAD, 1 IMAD.WIDE, 2 reference mont_mul, 3 hot-path mont_mul."""
     r = ctypes.c_double()
-    _check(lib().bzk_debug_imad_rate(iters, ctypes.byref(r), _stream_handle(stream)))
+    _check(lib().bzk_debug_bench(kind, iters, ctypes.byref(r), _stream_handle(stream)))
     return r.value
 
 

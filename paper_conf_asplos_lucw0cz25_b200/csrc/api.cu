@@ -38,6 +38,7 @@ struct bzk_ctx {
     cudaEvent_t ev_copied[2] = {nullptr, nullptr};
     cudaEvent_t ev_consumed[2] = {nullptr, nullptr};
     uint32_t *d_flag = nullptr;
+    fe *consts = nullptr;            // Lagrange / node constants (k_init_consts)
     std::string last_error;
     bool prof = false;
     std::vector<ProfRec> recs;
@@ -270,7 +271,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.ctas = ctas_for(h, io.nb);
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = io.round_evals; rp.challenges = io.challenges; rp.claims = io.claims;
-        rp.seed = seed; rp.first_index = io.first_index;
+        rp.consts = ctx->consts;
         if (i == 1) { rp.src = io.tables; rp.dst = nullptr; }
         else {
             rp.src = (i == 2) ? io.tables : ((i - 1) % 2 == 0 ? bufX : bufY);
@@ -288,6 +289,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         tp.i0 = P.i0; tp.log_h0 = P.log_h0; tp.k = k; tp.order = P.order; tp.ps = ps;
         tp.round_evals = io.round_evals; tp.challenges = io.challenges;
         tp.final_evals = io.final_evals; tp.claims = io.claims;
+        tp.consts = ctx->consts;
         if (P.i0 <= 2) tp.src = io.tables;
         else tp.src = ((P.i0 - 1) % 2 == 0) ? bufX : bufY;
         size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 32;
@@ -414,34 +416,98 @@ __global__ void k_debug_sha256(const uint8_t *msgs, uint32_t len, uint64_t n, ui
     }
 }
 
-// 8 independent IMAD chains per thread; returns cycles in out[block]
-__global__ void k_imad_rate(uint32_t iters, uint32_t seed, unsigned long long *cycles, uint32_t *sink) {
-    uint32_t a0 = seed ^ threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5,
-             a6 = a0 + 6, a7 = a0 + 7;
-    const uint32_t x = seed | 1, y = seed >> 3;
-    __syncthreads();
-    unsigned long long t0 = clock64();
-    for (uint32_t it = 0; it < iters; ++it) {
+// Micro-benchmarks that calibrate the integer roof (bzk_debug_bench).
+//   kind 0: mad.lo.u32 (IMAD)      kind 1: mul.wide.u32 (IMAD.WIDE.U32)
+//   kind 2: mont_mul_v1            kind 3: mont_mul (hot path)
+template <int KIND>
+__global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, uint32_t *sink) {
+    const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
+    if (KIND == 4) {   // DFMA throughput (FP64 pipe)
+        double a[8];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            asm volatile("mad.lo.u32 %0, %0, %8, %9;\n\t"
-                         "mad.lo.u32 %1, %1, %8, %9;\n\t"
-                         "mad.lo.u32 %2, %2, %8, %9;\n\t"
-                         "mad.lo.u32 %3, %3, %8, %9;\n\t"
-                         "mad.lo.u32 %4, %4, %8, %9;\n\t"
-                         "mad.lo.u32 %5, %5, %8, %9;\n\t"
-                         "mad.lo.u32 %6, %6, %8, %9;\n\t"
-                         "mad.lo.u32 %7, %7, %8, %9;"
-                         : "+r"(a0), "+r"(a1), "+r"(a2), "+r"(a3), "+r"(a4), "+r"(a5), "+r"(a6), "+r"(a7)
-                         : "r"(x), "r"(y));
+        for (int i = 0; i < 8; ++i) a[i] = 1.0 + 1e-9 * (tid + i);
+        const double x = 0.999999, y = 1e-7 * (seed & 7);
+        for (uint32_t it = 0; it < iters; ++it) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) asm volatile("fma.rn.f64 %0, %0, %1, %2;" : "+d"(a[i]) : "d"(x), "d"(y));
         }
+        double acc = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc += a[i];
+        sink[tid] = (uint32_t)__double2loint(acc);
+        return;
     }
-    __syncthreads();
-    unsigned long long t1 = clock64();
-    if (threadIdx.x == 0) cycles[blockIdx.x] = t1 - t0;
-    sink[blockIdx.x * blockDim.x + threadIdx.x] = a0 ^ a1 ^ a2 ^ a3 ^ a4 ^ a5 ^ a6 ^ a7;
+    if (KIND <= 1) {
+        uint32_t a[8];
+        uint64_t w[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) { a[i] = seed ^ (tid + i); w[i] = a[i]; }
+        const uint32_t x = seed | 1, y = seed >> 3;
+        for (uint32_t it = 0; it < iters; ++it) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    if (KIND == 0) asm volatile("mad.lo.u32 %0, %0, %1, %2;" : "+r"(a[i]) : "r"(x), "r"(y));
+                    else asm volatile("mad.wide.u32 %0, %1, %2, %0;" : "+l"(w[i]) : "r"((uint32_t)w[i]), "r"(x));
+                }
+        }
+        uint32_t acc = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc ^= a[i] ^ (uint32_t)w[i] ^ (uint32_t)(w[i] >> 32);
+        sink[tid] = acc;
+    } else {
+        fe x[4], y;
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) x[c].l[i] = (seed * (i + 1) + tid * 7 + c) & (i == 7 ? 0x0fffffffu : ~0u);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) y.l[i] = (seed ^ (0x9e3779b9u * (i + 3))) & (i == 7 ? 0x0fffffffu : ~0u);
+        for (uint32_t it = 0; it < iters; ++it)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) x[c] = KIND == 2 ? mont_mul_v1(x[c], y) : mont_mul(x[c], y);
+        uint32_t acc = 0;
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+#pragma unroll
+            for (int i = 0; i < 8; ++i) acc ^= x[c].l[i];
+        sink[tid] = acc;
+    }
 }
 
+}  // namespace
+
+// ==== (see below)
+namespace {
+template <int KIND>
+cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
+    int nsm = kSMs, clk_khz = 1965000;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
+    cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, 0);
+    const int threads = 256, blocks = nsm * 8;
+    uint32_t *sink = nullptr;
+    cudaError_t e = cudaMalloc(&sink, (size_t)blocks * threads * 4);
+    if (e != cudaSuccess) return e;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    k_bench<KIND><<<blocks, threads, 0, s>>>(iters / 8 + 1, 12345u, sink);   // warm-up
+    cudaEventRecord(e0, s);
+    k_bench<KIND><<<blocks, threads, 0, s>>>(iters, 12345u, sink);
+    cudaEventRecord(e1, s);
+    e = cudaEventSynchronize(e1);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(sink);
+    const double ops = (double)blocks * threads * iters * ((KIND <= 1 || KIND == 4) ? 32.0 : 4.0);
+    *rate = ops / (ms * 1e-3) / ((double)clk_khz * 1e3) / nsm;   // per SM per clock (at the max clock)
+    return e;
+}
 }  // namespace
 
 // ==================================================================== C ABI
@@ -478,7 +544,13 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
     ctx->workspace_limit = workspace_limit;
     cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device);
     if (cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaMalloc(&ctx->d_flag, 4) != cudaSuccess) {
+        cudaMalloc(&ctx->d_flag, 4) != cudaSuccess ||
+        cudaMalloc(&ctx->consts, sizeof(fe) * kNumConsts) != cudaSuccess) {
+        delete ctx;
+        return BZK_ECUDA;
+    }
+    k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
+    if (cudaStreamSynchronize(ctx->copy_stream) != cudaSuccess) {
         delete ctx;
         return BZK_ECUDA;
     }
@@ -496,6 +568,7 @@ void bzk_destroy(bzk_ctx *ctx) {
     cudaDeviceSynchronize();
     if (ctx->ws) cudaFree(ctx->ws);
     if (ctx->d_flag) cudaFree(ctx->d_flag);
+    if (ctx->consts) cudaFree(ctx->consts);
     for (int i = 0; i < 2; ++i) {
         if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
         if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
@@ -600,28 +673,18 @@ bzk_status bzk_debug_sha256(const uint8_t *msgs, uint32_t msg_len, uint64_t n, u
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }
 
-bzk_status bzk_debug_imad_rate(uint32_t iters, double *rate, void *cuda_stream) {
-    if (!rate || iters == 0) return BZK_EINVAL;
+bzk_status bzk_debug_bench(int kind, uint32_t iters, double *rate, void *cuda_stream) {
+    if (!rate || iters == 0 || kind < 0 || kind > 4) return BZK_EINVAL;
     cudaStream_t s = (cudaStream_t)cuda_stream;
-    int nsm = kSMs;
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
-    const int blocks = nsm * 2, threads = 512;
-    unsigned long long *cyc = nullptr;
-    uint32_t *sink = nullptr;
-    if (cudaMalloc(&cyc, blocks * sizeof(unsigned long long)) != cudaSuccess) return BZK_ENOMEM;
-    if (cudaMalloc(&sink, (size_t)blocks * threads * 4) != cudaSuccess) { cudaFree(cyc); return BZK_ENOMEM; }
-    k_imad_rate<<<blocks, threads, 0, s>>>(iters, 12345u, cyc, sink);
-    std::vector<unsigned long long> h(blocks);
-    cudaMemcpyAsync(h.data(), cyc, blocks * sizeof(unsigned long long), cudaMemcpyDeviceToHost, s);
-    cudaError_t e = cudaStreamSynchronize(s);
-    cudaFree(cyc);
-    cudaFree(sink);
-    if (e != cudaSuccess) return BZK_ECUDA;
-    std::sort(h.begin(), h.end());
-    const double med = (double)h[blocks / 2];
-    // 2 co-resident blocks per SM, each threads x iters x 32 IMAD
-    *rate = 2.0 * threads * (double)iters * 32.0 / med;
-    return BZK_OK;
+    cudaError_t e = cudaErrorInvalidValue;
+    switch (kind) {
+        case 0: e = run_bench<0>(iters, rate, s); break;
+        case 1: e = run_bench<1>(iters, rate, s); break;
+        case 2: e = run_bench<2>(iters, rate, s); break;
+        case 3: e = run_bench<3>(iters, rate, s); break;
+        case 4: e = run_bench<4>(iters, rate, s); break;
+    }
+    return e == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }
 
 }  // extern "C"

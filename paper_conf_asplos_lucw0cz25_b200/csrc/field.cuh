@@ -181,8 +181,9 @@ __device__ __forceinline__ void mad_row_p(uint32_t t[10], uint32_t m) {
           "r"(BZK_P6), "r"(BZK_P7));
 }
 
-// Montgomery product a*b*R^{-1} mod p (CIOS), a, b canonical -> canonical.
-__device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
+// Montgomery product a*b*R^{-1} mod p (CIOS, row-wise), reference version kept for the
+// micro-benchmark (bzk_debug_bench kind 2): a single 10-word accumulator, even/odd product chains.
+__device__ __forceinline__ fe mont_mul_v1(const fe &a, const fe &b) {
     uint32_t t[10];
 #pragma unroll
     for (int i = 0; i < 10; ++i) t[i] = 0;
@@ -191,7 +192,6 @@ __device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
         mad_row(t, a.l, b.l[i]);
         uint32_t m = t[0] * BZK_NP0;
         mad_row_p(t, m);
-        // t[0] == 0 now; shift down one limb
 #pragma unroll
         for (int j = 0; j < 9; ++j) t[j] = t[j + 1];
         t[9] = 0;
@@ -199,7 +199,218 @@ __device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
     fe r;
 #pragma unroll
     for (int i = 0; i < 8; ++i) r.l[i] = t[i];
-    return fe_reduce_once(r);   // t < 2p for canonical inputs
+    return fe_reduce_once(r);
+}
+
+// ---------------------------------------------------------------- Montgomery product (hot path)
+//
+// CIOS with two parity-aligned accumulators so that every 32x32->64 product lands in an aligned
+// register pair and ptxas can emit one IMAD.WIDE.U32(.X) per product with no register moves:
+//   A[q] holds relative column q (pairs (A0,A1),(A2,A3),...,(A6,A7), A8 single),
+//   B[q] holds relative column q+1 (pairs (B0,B1) at columns (1,2), ..., B8 at column 9),
+//   L    holds a pending word at column 0.
+// Row i: A += a_even * b_i, B += a_odd * b_i (L is folded in at the head of the B chain, whose
+// carry enters column 1 = B0), m = A0 * (-p^{-1}), A += p_even * m, B += p_odd * m, then divide by
+// W = 2^32: the new A is the old B (columns 1..9), the new B is old A2..A8, and old A1 (column 1)
+// becomes the new pending L.  After 8 rows: result = A + L + (B << 32).
+
+// B chain of a row: A0 += L (carry to column 1), B[0..7] += a_odd * bi, carry into B8
+__device__ __forceinline__ void row_b(uint32_t A[9], uint32_t B[9], uint32_t L, const uint32_t a[8], uint32_t bi) {
+    asm("add.cc.u32     %0, %0, %10;\n\t"
+        "madc.lo.cc.u32 %1, %11, %15, %1;\n\t"
+        "madc.hi.cc.u32 %2, %11, %15, %2;\n\t"
+        "madc.lo.cc.u32 %3, %12, %15, %3;\n\t"
+        "madc.hi.cc.u32 %4, %12, %15, %4;\n\t"
+        "madc.lo.cc.u32 %5, %13, %15, %5;\n\t"
+        "madc.hi.cc.u32 %6, %13, %15, %6;\n\t"
+        "madc.lo.cc.u32 %7, %14, %15, %7;\n\t"
+        "madc.hi.cc.u32 %8, %14, %15, %8;\n\t"
+        "addc.u32       %9, %9, 0;"
+        : "+r"(A[0]), "+r"(B[0]), "+r"(B[1]), "+r"(B[2]), "+r"(B[3]), "+r"(B[4]), "+r"(B[5]), "+r"(B[6]),
+          "+r"(B[7]), "+r"(B[8])
+        : "r"(L), "r"(a[1]), "r"(a[3]), "r"(a[5]), "r"(a[7]), "r"(bi));
+}
+
+// A chain of a row: A[0..7] += a_even * bi, carry into A8
+__device__ __forceinline__ void row_a(uint32_t A[9], const uint32_t a[8], uint32_t bi) {
+    asm("mad.lo.cc.u32  %0, %9,  %13, %0;\n\t"
+        "madc.hi.cc.u32 %1, %9,  %13, %1;\n\t"
+        "madc.lo.cc.u32 %2, %10, %13, %2;\n\t"
+        "madc.hi.cc.u32 %3, %10, %13, %3;\n\t"
+        "madc.lo.cc.u32 %4, %11, %13, %4;\n\t"
+        "madc.hi.cc.u32 %5, %11, %13, %5;\n\t"
+        "madc.lo.cc.u32 %6, %12, %13, %6;\n\t"
+        "madc.hi.cc.u32 %7, %12, %13, %7;\n\t"
+        "addc.u32       %8, %8, 0;"
+        : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
+          "+r"(A[8])
+        : "r"(a[0]), "r"(a[2]), "r"(a[4]), "r"(a[6]), "r"(bi));
+}
+
+// reduction chains: A += p_even * m (A0 -> 0), B += p_odd * m
+__device__ __forceinline__ void red_a(uint32_t A[9], uint32_t m) {
+    asm("mad.lo.cc.u32  %0, %9, %10, %0;\n\t"
+        "madc.hi.cc.u32 %1, %9, %10, %1;\n\t"
+        "madc.lo.cc.u32 %2, %9, %11, %2;\n\t"
+        "madc.hi.cc.u32 %3, %9, %11, %3;\n\t"
+        "madc.lo.cc.u32 %4, %9, %12, %4;\n\t"
+        "madc.hi.cc.u32 %5, %9, %12, %5;\n\t"
+        "madc.lo.cc.u32 %6, %9, %13, %6;\n\t"
+        "madc.hi.cc.u32 %7, %9, %13, %7;\n\t"
+        "addc.u32       %8, %8, 0;"
+        : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
+          "+r"(A[8])
+        : "r"(m), "n"(BZK_P0), "n"(BZK_P2), "n"(BZK_P4), "n"(BZK_P6));
+}
+
+__device__ __forceinline__ void red_b(uint32_t B[9], uint32_t m) {
+    asm("mad.lo.cc.u32  %0, %9, %10, %0;\n\t"
+        "madc.hi.cc.u32 %1, %9, %10, %1;\n\t"
+        "madc.lo.cc.u32 %2, %9, %11, %2;\n\t"
+        "madc.hi.cc.u32 %3, %9, %11, %3;\n\t"
+        "madc.lo.cc.u32 %4, %9, %12, %4;\n\t"
+        "madc.hi.cc.u32 %5, %9, %12, %5;\n\t"
+        "madc.lo.cc.u32 %6, %9, %13, %6;\n\t"
+        "madc.hi.cc.u32 %7, %9, %13, %7;\n\t"
+        "addc.u32       %8, %8, 0;"
+        : "+r"(B[0]), "+r"(B[1]), "+r"(B[2]), "+r"(B[3]), "+r"(B[4]), "+r"(B[5]), "+r"(B[6]), "+r"(B[7]),
+          "+r"(B[8])
+        : "r"(m), "n"(BZK_P1), "n"(BZK_P3), "n"(BZK_P5), "n"(BZK_P7));
+}
+
+// Montgomery product a*b*R^{-1} mod p; a, b canonical -> canonical.
+__device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
+    uint32_t A[9], B[9], L = 0;
+    // row 0: plain products (no accumulation)
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]), "=r"(A[4]), "=r"(A[5]), "=r"(A[6]), "=r"(A[7]),
+          "=r"(A[8])
+        : "r"(a.l[0]), "r"(a.l[2]), "r"(a.l[4]), "r"(a.l[6]), "r"(b.l[0]));
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(B[0]), "=r"(B[1]), "=r"(B[2]), "=r"(B[3]), "=r"(B[4]), "=r"(B[5]), "=r"(B[6]), "=r"(B[7]),
+          "=r"(B[8])
+        : "r"(a.l[1]), "r"(a.l[3]), "r"(a.l[5]), "r"(a.l[7]), "r"(b.l[0]));
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        if (i > 0) {
+            row_b(A, B, L, a.l, b.l[i]);
+            row_a(A, a.l, b.l[i]);
+        }
+        uint32_t m = A[0] * BZK_NP0;
+        red_a(A, m);
+        red_b(B, m);
+        // divide by W: L = A1; A <- B; B <- A2..A8, 0, 0
+        L = A[1];
+        uint32_t nA[9], nB[9];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) nA[q] = B[q];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) nB[q] = A[q + 2];
+        nB[7] = 0;
+        nB[8] = 0;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) { A[q] = nA[q]; B[q] = nB[q]; }
+    }
+    // result = A + L + (B << 32)   (< 2p < 2^255, so A8 and B7, B8 end up zero)
+    fe r;
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
+          "=r"(r.l[7])
+        : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
+          "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
+    return fe_reduce_once(r);
+}
+
+// (x*y + u*v) * R^{-1} mod p with ONE Montgomery reduction (lazy sum of two products).
+// Each row adds x*y_i and u*v_i before the reduction row; with x, u < p the CIOS accumulator stays
+// below 3p + 1 (< 2^256 since 4p < 2^256), so the result needs at most two subtractions of p.
+__device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, const fe &v) {
+    uint32_t A[9], B[9], L = 0;
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]), "=r"(A[4]), "=r"(A[5]), "=r"(A[6]), "=r"(A[7]),
+          "=r"(A[8])
+        : "r"(x.l[0]), "r"(x.l[2]), "r"(x.l[4]), "r"(x.l[6]), "r"(y.l[0]));
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(B[0]), "=r"(B[1]), "=r"(B[2]), "=r"(B[3]), "=r"(B[4]), "=r"(B[5]), "=r"(B[6]), "=r"(B[7]),
+          "=r"(B[8])
+        : "r"(x.l[1]), "r"(x.l[3]), "r"(x.l[5]), "r"(x.l[7]), "r"(y.l[0]));
+    row_a(A, u.l, v.l[0]);
+    row_b(A, B, 0u, u.l, v.l[0]);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        if (i > 0) {
+            row_b(A, B, L, x.l, y.l[i]);
+            row_a(A, x.l, y.l[i]);
+            row_b(A, B, 0u, u.l, v.l[i]);
+            row_a(A, u.l, v.l[i]);
+        }
+        uint32_t m = A[0] * BZK_NP0;
+        red_a(A, m);
+        red_b(B, m);
+        L = A[1];
+        uint32_t nA[9], nB[9];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) nA[q] = B[q];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) nB[q] = A[q + 2];
+        nB[7] = 0;
+        nB[8] = 0;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) { A[q] = nA[q]; B[q] = nB[q]; }
+    }
+    fe r;
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
+          "=r"(r.l[7])
+        : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
+          "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
+    return fe_reduce_once(fe_reduce_once(r));   // r <= 3p
 }
 
 __device__ __forceinline__ fe fe_const(int which) {
