@@ -37,6 +37,11 @@ struct bzk_ctx {
     cudaStream_t copy_stream = nullptr;
     cudaEvent_t ev_copied[2] = {nullptr, nullptr};
     cudaEvent_t ev_consumed[2] = {nullptr, nullptr};
+    // loader ring: two device staging slots for host tables, reused across waves, jobs and calls
+    void *stage[2] = {nullptr, nullptr};
+    size_t stage_size = 0;
+    int next_slot = 0;
+    bool slot_used[2] = {false, false};
     uint32_t *d_flag = nullptr;
     fe *consts = nullptr;            // Lagrange / node constants (k_init_consts)
     std::string last_error;
@@ -99,8 +104,9 @@ struct Plan {
     uint64_t N;
     size_t elem_table;    // bytes of one table set (D * N * 32)
     // per-wave workspace layout (bytes)
-    size_t off_ps, off_tick, off_part, off_bufX, off_bufY, off_stage0, off_stage1, off_out, off_seed;
-    size_t total;
+    size_t off_ps, off_tick, off_part, off_bufX, off_bufY, off_out, off_seed;
+    size_t total;        // device workspace bytes (excluding the loader's staging slots)
+    size_t stage_bytes;  // bytes of one staging slot (host tables), 0 otherwise
     uint32_t cmax;
     bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
     size_t out_bytes_per_proof;
@@ -153,7 +159,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     if (limit == 0) {
         size_t fr = 0, tot = 0;
         cudaMemGetInfo(&fr, &tot);
-        fr += ctx->ws_size;  // our own current allocation is reusable
+        fr += ctx->ws_size + 2 * ctx->stage_size;  // our own current allocations are reusable
         limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
     }
     auto per_proof = [&](uint64_t bw) -> size_t {
@@ -168,8 +174,9 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     };
     const size_t fixed = 4096 + (P.host_outputs ? align_up(P.B * P.out_bytes_per_proof) : 0);
     uint64_t bw = std::min<uint64_t>(P.B, 65535);
-    // host tables: at least 8 loader waves so the H2D of wave w+1 overlaps the compute of wave w
-    if (P.host_tables && P.B >= 8) bw = std::min<uint64_t>(bw, (P.B + 7) / 8);
+    // large host-table jobs: at least 8 loader waves so the H2D of wave w+1 overlaps the compute
+    // of wave w (small jobs overlap with the neighbouring jobs instead)
+    if (P.host_tables && P.B >= 8 && P.B * P.elem_table > (2ull << 30)) bw = std::min<uint64_t>(bw, (P.B + 7) / 8);
     while (bw > 1 && fixed + per_proof(bw) * bw + 8 * 256 > limit) bw = (bw + 1) / 2;
     if (fixed + per_proof(bw) * bw + 8 * 256 > limit)
         return fail(ctx, BZK_ENOMEM, "workspace_limit too small for one proof");
@@ -187,10 +194,9 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * (P.D + 1) * 32);
     P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * 32);
     P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * 32);
-    P.off_stage0 = off; if (P.host_tables) off = align_up(off + bw * P.elem_table);
-    P.off_stage1 = off; if (P.host_tables) off = align_up(off + bw * P.elem_table);
     P.off_out = off; if (P.host_outputs) off = align_up(off + P.B * P.out_bytes_per_proof);
     P.total = off;
+    P.stage_bytes = P.host_tables ? align_up(bw * P.elem_table) : 0;
     return BZK_OK;
 }
 
@@ -203,6 +209,26 @@ bzk_status ensure_ws(bzk_ctx *ctx, size_t bytes) {
         return fail(ctx, BZK_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(e));
     }
     ctx->ws_size = bytes;
+    return BZK_OK;
+}
+
+bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
+    if (bytes == 0 || ctx->stage_size >= bytes) return BZK_OK;
+    cudaDeviceSynchronize();   // slots may still be in use by earlier work
+    for (int i = 0; i < 2; ++i) {
+        if (ctx->stage[i]) cudaFree(ctx->stage[i]);
+        ctx->stage[i] = nullptr;
+    }
+    ctx->stage_size = 0;
+    ctx->slot_used[0] = ctx->slot_used[1] = false;
+    for (int i = 0; i < 2; ++i) {
+        cudaError_t e = cudaMalloc(&ctx->stage[i], bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ctx, BZK_ENOMEM, std::string("cudaMalloc staging: ") + cudaGetErrorString(e));
+        }
+    }
+    ctx->stage_size = bytes;
     return BZK_OK;
 }
 
@@ -301,21 +327,18 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
     return BZK_OK;
 }
 
-bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
-    bzk_status st = validate_args(ctx, b);
-    if (st) return st;
-    Plan P;
-    st = make_plan(ctx, b, P);
-    if (st) return st;
-    st = ensure_ws(ctx, P.total);
-    if (st) return st;
+// Enqueue one job (all its waves) on stream s.  Host tables go through the loader ring: wave w's
+// tables are copied into the next staging slot on the copy stream as soon as that slot's
+// previous user (possibly a wave of the previous job or call) has been consumed, so copies run
+// ahead of compute across waves AND jobs.  Returns after enqueueing (no synchronisation) unless
+// validation is requested.
+bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStream_t s) {
     char *ws = (char *)ctx->ws;
     CK(cudaMemcpyAsync(ws + P.off_seed, b->seed, 32, cudaMemcpyHostToDevice, s));
     CK(cudaMemsetAsync(ws + P.off_tick, 0, P.Bw * 4, s));
     const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
     if (validate) CK(cudaMemsetAsync(ctx->d_flag, 0, 4, s));
 
-    const size_t opp = P.out_bytes_per_proof;
     const size_t ev_pp = (size_t)P.k * (P.D + 1), ch_pp = P.k, fi_pp = P.D;
     fe *o_ev, *o_ch, *o_fi, *o_cl;
     if (P.host_outputs) {
@@ -325,7 +348,6 @@ bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
         o_ev = (fe *)b->round_evals; o_ch = (fe *)b->challenges; o_fi = (fe *)b->final_evals;
         o_cl = (fe *)b->claims;
     }
-    (void)opp;
     for (uint64_t w = 0; w < P.nwaves; ++w) {
         WaveIO io;
         const uint64_t b0 = w * P.Bw;
@@ -335,20 +357,19 @@ bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
         io.challenges = o_ch + b0 * ch_pp;
         io.final_evals = o_fi + b0 * fi_pp;
         io.claims = (P.host_outputs || o_cl) ? o_cl + b0 : nullptr;
+        int slot = -1;
         if (P.host_tables) {
-            // loader: wave w's tables -> staging[w % 2] on the copy stream, overlapping wave w-1
-            const int slot = (int)(w % 2);
-            fe *stage = (fe *)(ws + (slot ? P.off_stage1 : P.off_stage0));
-            if (w >= 2) CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
-
+            slot = ctx->next_slot;
+            ctx->next_slot ^= 1;
+            if (ctx->slot_used[slot]) CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
             {
                 ProfScope ps_(ctx, ctx->copy_stream, 5);
-                CK(cudaMemcpyAsync(stage, (const char *)b->tables + b0 * P.elem_table, io.nb * P.elem_table,
-                                   cudaMemcpyHostToDevice, ctx->copy_stream));
+                CK(cudaMemcpyAsync(ctx->stage[slot], (const char *)b->tables + b0 * P.elem_table,
+                                   io.nb * P.elem_table, cudaMemcpyHostToDevice, ctx->copy_stream));
             }
             CK(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
             CK(cudaStreamWaitEvent(s, ctx->ev_copied[slot], 0));
-            io.tables = stage;
+            io.tables = (fe *)ctx->stage[slot];
         } else {
             io.tables = (fe *)((char *)b->tables + b0 * P.elem_table);
         }
@@ -358,9 +379,12 @@ bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
             ++ctx->launches;
             CK(cudaGetLastError());
         }
-        st = run_wave(ctx, P, io, s);
+        bzk_status st = run_wave(ctx, P, io, s);
         if (st) return st;
-        if (P.host_tables) CK(cudaEventRecord(ctx->ev_consumed[w % 2], s));
+        if (slot >= 0) {
+            CK(cudaEventRecord(ctx->ev_consumed[slot], s));
+            ctx->slot_used[slot] = true;
+        }
     }
     if (P.host_outputs) {
         if (P.k) {
@@ -376,7 +400,33 @@ bzk_status prove_impl(bzk_ctx *ctx, const bzk_batch *b, cudaStream_t s) {
         CK(cudaStreamSynchronize(s));
         if (flag) return fail(ctx, BZK_ENONCANON, "an input element is >= p");
     }
-    if ((b->flags & BZK_F_SYNC) || P.host_outputs || P.host_tables) CK(cudaStreamSynchronize(s));
+    return BZK_OK;
+}
+
+// Plan every job, size the workspace for the largest, enqueue all of them, then synchronise
+// when the caller asked for it or host memory is involved (outputs must be readable on return).
+bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStream_t s) {
+    std::vector<Plan> plans(njobs);
+    size_t ws_need = 0, stage_need = 0;
+    bool need_sync = false;
+    for (size_t j = 0; j < njobs; ++j) {
+        bzk_status st = validate_args(ctx, &jobs[j]);
+        if (st) return njobs > 1 ? fail(ctx, st, "job " + std::to_string(j) + ": " + ctx->last_error) : st;
+        st = make_plan(ctx, &jobs[j], plans[j]);
+        if (st) return st;
+        ws_need = std::max(ws_need, plans[j].total);
+        stage_need = std::max(stage_need, plans[j].stage_bytes);
+        need_sync |= (jobs[j].flags & BZK_F_SYNC) || plans[j].host_outputs || plans[j].host_tables;
+    }
+    bzk_status st = ensure_ws(ctx, ws_need);
+    if (st) return st;
+    st = ensure_stage(ctx, stage_need);
+    if (st) return st;
+    for (size_t j = 0; j < njobs; ++j) {
+        st = enqueue_job(ctx, &jobs[j], plans[j], s);
+        if (st) return st;
+    }
+    if (need_sync) CK(cudaStreamSynchronize(s));
     return BZK_OK;
 }
 
@@ -569,6 +619,8 @@ void bzk_destroy(bzk_ctx *ctx) {
     if (ctx->ws) cudaFree(ctx->ws);
     if (ctx->d_flag) cudaFree(ctx->d_flag);
     if (ctx->consts) cudaFree(ctx->consts);
+    for (int i = 0; i < 2; ++i)
+        if (ctx->stage[i]) cudaFree(ctx->stage[i]);
     for (int i = 0; i < 2; ++i) {
         if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
         if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
@@ -593,21 +645,14 @@ bzk_status bzk_workspace_size(bzk_ctx *ctx, const bzk_batch *batch, size_t *byte
 bzk_status bzk_prove(bzk_ctx *ctx, const bzk_batch *batch, void *cuda_stream) {
     if (!ctx) return BZK_EINVAL;
     cudaSetDevice(ctx->device);
-    return prove_impl(ctx, batch, (cudaStream_t)cuda_stream);
+    if (!batch) return fail(ctx, BZK_EINVAL, "batch is NULL");
+    return prove_jobs(ctx, batch, 1, (cudaStream_t)cuda_stream);
 }
 
 bzk_status bzk_prove_ragged(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, void *cuda_stream) {
     if (!ctx || (!jobs && njobs)) return BZK_EINVAL;
     cudaSetDevice(ctx->device);
-    for (size_t j = 0; j < njobs; ++j) {
-        bzk_status st = validate_args(ctx, &jobs[j]);
-        if (st) return fail(ctx, st, "job " + std::to_string(j) + ": " + ctx->last_error);
-    }
-    for (size_t j = 0; j < njobs; ++j) {
-        bzk_status st = prove_impl(ctx, &jobs[j], (cudaStream_t)cuda_stream);
-        if (st) return st;
-    }
-    return BZK_OK;
+    return prove_jobs(ctx, jobs, njobs, (cudaStream_t)cuda_stream);
 }
 
 bzk_status bzk_sync(bzk_ctx *ctx) {
