@@ -5,6 +5,7 @@
 // a2-a7 live in sumcheck.cuh.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -50,6 +51,11 @@ struct bzk_ctx {
     std::vector<cudaEvent_t> ev_pool;
     uint64_t launches = 0;
     int num_sms = kSMs;
+    size_t auto_limit = 0;           // cached default workspace limit (0 = recompute)
+    // CUDA graph of the last BZK_F_GRAPH call, replayed while the submitted jobs are identical
+    cudaGraphExec_t graph_exec = nullptr;
+    std::vector<unsigned char> graph_key;
+    uint64_t graph_launches = 0;      // kernel launches inside the cached graph
 };
 
 namespace {
@@ -112,11 +118,24 @@ struct Plan {
     size_t out_bytes_per_proof;
 };
 
+// tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
+// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round, default on)
+struct Knobs {
+    uint64_t ppt_max = 16, waves = 4;
+    uint32_t prefetch = 1;
+    Knobs() {
+        if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
+        if (const char *e = getenv("BZK_CTA_WAVES")) waves = std::max(1, atoi(e));
+        if (const char *e = getenv("BZK_PREFETCH")) prefetch = atoi(e) ? 1 : 0;
+    }
+};
+const Knobs &knobs() { static Knobs k; return k; }
+
 uint32_t ctas_for(uint64_t h, uint64_t nb) {
-    // enough CTAs to fill 148 SMs x 2 resident CTAs x 4 waves, at most 16 pairs per thread
-    const uint64_t target = (uint64_t)kSMs * 2 * 4;
+    // enough CTAs to fill 148 SMs x 2 resident CTAs x `waves` waves, at most ppt_max pairs per thread
+    const uint64_t target = (uint64_t)kSMs * 2 * knobs().waves;
     uint64_t ppt = (nb * h) / ((uint64_t)kThreads * target);
-    ppt = std::max<uint64_t>(1, std::min<uint64_t>(16, ppt));
+    ppt = std::max<uint64_t>(1, std::min<uint64_t>(knobs().ppt_max, ppt));
     uint64_t c = (h + kThreads * ppt - 1) / (kThreads * ppt);
     return (uint32_t)std::max<uint64_t>(1, c);
 }
@@ -157,10 +176,14 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
 
     size_t limit = ctx->workspace_limit;
     if (limit == 0) {
-        size_t fr = 0, tot = 0;
-        cudaMemGetInfo(&fr, &tot);
-        fr += ctx->ws_size + 2 * ctx->stage_size;  // our own current allocations are reusable
-        limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
+        // free device memory + our own reusable allocations - 2 GiB; cached until we (re)allocate
+        if (ctx->auto_limit == 0) {
+            size_t fr = 0, tot = 0;
+            cudaMemGetInfo(&fr, &tot);
+            fr += ctx->ws_size + 2 * ctx->stage_size;
+            ctx->auto_limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
+        }
+        limit = ctx->auto_limit;
     }
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
@@ -202,6 +225,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
 
 bzk_status ensure_ws(bzk_ctx *ctx, size_t bytes) {
     if (ctx->ws_size >= bytes) return BZK_OK;
+    ctx->auto_limit = 0;
     if (ctx->ws) { cudaFree(ctx->ws); ctx->ws = nullptr; ctx->ws_size = 0; }
     cudaError_t e = cudaMalloc(&ctx->ws, bytes);
     if (e != cudaSuccess) {
@@ -215,6 +239,7 @@ bzk_status ensure_ws(bzk_ctx *ctx, size_t bytes) {
 bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
     if (bytes == 0 || ctx->stage_size >= bytes) return BZK_OK;
     cudaDeviceSynchronize();   // slots may still be in use by earlier work
+    ctx->auto_limit = 0;
     for (int i = 0; i < 2; ++i) {
         if (ctx->stage[i]) cudaFree(ctx->stage[i]);
         ctx->stage[i] = nullptr;
@@ -267,6 +292,7 @@ __global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
 // ---------------------------------------------------------------- one wave
 
 struct WaveIO {
+    Seed32 seed;       // transcript seed, passed to the kernel by value
     fe *tables;        // device tables of this wave [nb][D][N]
     fe *round_evals, *challenges, *final_evals, *claims;   // device outputs of this wave
     uint64_t nb, first_index;
@@ -279,11 +305,10 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
     fe *part = (fe *)(ws + P.off_part);
     fe *bufX = (fe *)(ws + P.off_bufX);
     fe *bufY = P.bufY_alias_input ? io.tables : (fe *)(ws + P.off_bufY);
-    const uint8_t *seed = (const uint8_t *)(ws + P.off_seed);
     const uint32_t D = P.D, k = P.k;
     {
         ProfScope ps_(ctx, s, 3);
-        k_transcript_init<<<(uint32_t)((io.nb + 127) / 128), 128, 0, s>>>(ps, (uint32_t)io.nb, seed,
+        k_transcript_init<<<(uint32_t)((io.nb + 127) / 128), 128, 0, s>>>(ps, (uint32_t)io.nb, io.seed,
                                                                           io.first_index, k, D, P.order);
         ++ctx->launches;
         CK(cudaGetLastError());
@@ -298,6 +323,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = io.round_evals; rp.challenges = io.challenges; rp.claims = io.claims;
         rp.consts = ctx->consts;
+        rp.prefetch = knobs().prefetch;
         if (i == 1) { rp.src = io.tables; rp.dst = nullptr; }
         else {
             rp.src = (i == 2) ? io.tables : ((i - 1) % 2 == 0 ? bufX : bufY);
@@ -334,7 +360,6 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
 // validation is requested.
 bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStream_t s) {
     char *ws = (char *)ctx->ws;
-    CK(cudaMemcpyAsync(ws + P.off_seed, b->seed, 32, cudaMemcpyHostToDevice, s));
     CK(cudaMemsetAsync(ws + P.off_tick, 0, P.Bw * 4, s));
     const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
     if (validate) CK(cudaMemsetAsync(ctx->d_flag, 0, 4, s));
@@ -350,6 +375,7 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     }
     for (uint64_t w = 0; w < P.nwaves; ++w) {
         WaveIO io;
+        memcpy(io.seed.b, b->seed, 32);
         const uint64_t b0 = w * P.Bw;
         io.nb = std::min<uint64_t>(P.Bw, P.B - b0);
         io.first_index = b->first_index + b0;
@@ -418,13 +444,52 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
         stage_need = std::max(stage_need, plans[j].stage_bytes);
         need_sync |= (jobs[j].flags & BZK_F_SYNC) || plans[j].host_outputs || plans[j].host_tables;
     }
+    bool graph = !need_sync && !ctx->prof && s != nullptr;   // no capture on the legacy stream
+    for (size_t j = 0; j < njobs; ++j)
+        graph = graph && (jobs[j].flags & BZK_F_GRAPH) && !(jobs[j].flags & BZK_F_VALIDATE);
+    std::vector<unsigned char> key;
+    if (graph) {
+        // identical job descriptions (pointers, sizes, seed bytes) on the same stream -> replay
+        key.resize(njobs * (sizeof(bzk_batch) + 32) + sizeof(cudaStream_t));
+        unsigned char *kp = key.data();
+        memcpy(kp, &s, sizeof(s));
+        kp += sizeof(s);
+        for (size_t j = 0; j < njobs; ++j) {
+            memcpy(kp, &jobs[j], sizeof(bzk_batch));
+            memcpy(kp + sizeof(bzk_batch), jobs[j].seed, 32);
+            kp += sizeof(bzk_batch) + 32;
+        }
+    }
     bzk_status st = ensure_ws(ctx, ws_need);
     if (st) return st;
     st = ensure_stage(ctx, stage_need);
     if (st) return st;
+    if (graph && ctx->graph_exec && ctx->graph_key == key) {
+        CK(cudaGraphLaunch(ctx->graph_exec, s));
+        ctx->launches += ctx->graph_launches;
+        return BZK_OK;
+    }
+    if (graph) {
+        if (ctx->graph_exec) { cudaGraphExecDestroy(ctx->graph_exec); ctx->graph_exec = nullptr; }
+        CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    }
+    const uint64_t l0 = ctx->launches;
     for (size_t j = 0; j < njobs; ++j) {
         st = enqueue_job(ctx, &jobs[j], plans[j], s);
-        if (st) return st;
+        if (st) {
+            if (graph) { cudaGraph_t g; cudaStreamEndCapture(s, &g); if (g) cudaGraphDestroy(g); }
+            return st;
+        }
+    }
+    if (graph) {
+        cudaGraph_t g = nullptr;
+        CK(cudaStreamEndCapture(s, &g));
+        cudaError_t e = cudaGraphInstantiate(&ctx->graph_exec, g, 0);
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) { ctx->graph_exec = nullptr; return cuda_fail(ctx, e, "cudaGraphInstantiate"); }
+        ctx->graph_key = key;
+        ctx->graph_launches = ctx->launches - l0;
+        CK(cudaGraphLaunch(ctx->graph_exec, s));
     }
     if (need_sync) CK(cudaStreamSynchronize(s));
     return BZK_OK;
@@ -599,6 +664,10 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
         delete ctx;
         return BZK_ECUDA;
     }
+    set_kernel_attrs<1>();
+    set_kernel_attrs<2>();
+    set_kernel_attrs<3>();
+    set_kernel_attrs<4>();
     k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
     if (cudaStreamSynchronize(ctx->copy_stream) != cudaSuccess) {
         delete ctx;
@@ -625,6 +694,7 @@ void bzk_destroy(bzk_ctx *ctx) {
         if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
         if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
     }
+    if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
     for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
     for (auto e : ctx->ev_pool) cudaEventDestroy(e);
     if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);

@@ -17,14 +17,14 @@ cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t 
 }
 
 template <>
+cudaError_t set_kernel_attrs<BZK_D>() {
+    cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    return cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+}
+
+template <>
 cudaError_t launch_tail<BZK_D>(uint32_t order, uint32_t grid, uint32_t threads, size_t smem, cudaStream_t s,
                                const TailParams &p) {
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-        cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-        attr_set = true;
-    }
     if (order == 0) k_tail<BZK_D, 0><<<grid, threads, smem, s>>>(p);
     else            k_tail<BZK_D, 1><<<grid, threads, smem, s>>>(p);
     return cudaGetLastError();

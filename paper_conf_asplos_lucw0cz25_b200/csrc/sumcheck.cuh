@@ -25,6 +25,10 @@
 #pragma once
 #include <stdint.h>
 #include "field.cuh"
+
+#ifndef BZK_ROUND_OCC
+#define BZK_ROUND_OCC 2   // resident CTAs per SM requested for k_round (d <= 2)
+#endif
 #include "sha256.cuh"
 
 namespace bzk {
@@ -56,6 +60,7 @@ struct RoundParams {
     fe *challenges;       // [Bw][k]
     fe *claims;           // [Bw] (may be null)
     const fe *consts;     // kNumConsts
+    uint32_t prefetch;    // 1: bulk-prefetch the next iteration's tiles into L2
 };
 
 // ---------------------------------------------------------------- reductions
@@ -229,15 +234,14 @@ static __global__ void k_init_consts(fe *c) {
     }
 }
 
-static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, const uint8_t *seed,
-                                         uint64_t first_index, uint32_t k, uint32_t d, uint32_t order) {
+struct Seed32 { uint8_t b[32]; };
+
+static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed32 seed, uint64_t first_index,
+                                         uint32_t k, uint32_t d, uint32_t order) {
     uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
     if (b >= nproofs) return;
-    uint8_t s[32];
-#pragma unroll
-    for (int i = 0; i < 32; ++i) s[i] = seed[i];
     uint32_t st[8];
-    transcript_init(st, s, first_index + b, k, d, order);
+    transcript_init(st, seed.b, first_index + b, k, d, order);
 #pragma unroll
     for (int i = 0; i < 8; ++i) ps[b].st[i] = st[i];
 }
@@ -279,8 +283,39 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
     }
 }
 
+// L2 bulk prefetch of a contiguous byte range (cp.async.bulk.prefetch, sm_90+; no registers, no smem)
+__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// Lane 0 of a warp prefetches into L2 the table ranges that the warp's 32 lanes will load for the
+// pairs j0 .. j0+31 (j0 = the warp's first pair index): one contiguous range per table for LSB,
+// two for MSB.
 template <int D, int ORDER, bool FIRST>
-__global__ void __launch_bounds__(256, (D <= 2 ? 2 : 1)) k_round(RoundParams P) {
+__device__ __forceinline__ void prefetch_pairs(const fe *src, uint64_t h, uint64_t j0) {
+    if (j0 >= h) return;
+    const uint64_t n = (h - j0) < 32 ? (h - j0) : 32;
+#pragma unroll
+    for (int m = 0; m < D; ++m) {
+        if (FIRST) {
+            const fe *T = src + (size_t)m * (2 * h);
+            if (ORDER == 0) prefetch_l2(T + 2 * j0, (uint32_t)(n * 64));
+            else { prefetch_l2(T + j0, (uint32_t)(n * 32)); prefetch_l2(T + j0 + h, (uint32_t)(n * 32)); }
+        } else {
+            const fe *T = src + (size_t)m * (4 * h);
+            if (ORDER == 0) prefetch_l2(T + 4 * j0, (uint32_t)(n * 128));
+            else {
+                prefetch_l2(T + j0, (uint32_t)(n * 32));
+                prefetch_l2(T + j0 + h, (uint32_t)(n * 32));
+                prefetch_l2(T + j0 + 2 * h, (uint32_t)(n * 32));
+                prefetch_l2(T + j0 + 3 * h, (uint32_t)(n * 32));
+            }
+        }
+    }
+}
+
+template <int D, int ORDER, bool FIRST>
+__global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
     constexpr bool DERIVE = !FIRST;
     constexpr int NV = Pts<D, DERIVE>::NV;
     __shared__ fe s_red[32 * NV];
@@ -295,7 +330,12 @@ __global__ void __launch_bounds__(256, (D <= 2 ? 2 : 1)) k_round(RoundParams P) 
     fe *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const fe rm = FIRST ? fe_zero() : P.ps[b].rmont;
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
+    const uint32_t lane = threadIdx.x & 31;
     for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += 2 * stride) {
+        if (P.prefetch && lane == 0) {
+            prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
+            prefetch_pairs<D, ORDER, FIRST>(src, h, j + 3 * stride);
+        }
         fe a[D], da[D], a2[D], da2[D];
         load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, da);
         const uint64_t j2 = j + stride;
@@ -447,5 +487,7 @@ cudaError_t launch_round(uint32_t order, bool first, dim3 grid, uint32_t threads
 template <int D>
 cudaError_t launch_tail(uint32_t order, uint32_t grid, uint32_t threads, size_t smem, cudaStream_t s,
                         const TailParams &p);
+template <int D>
+cudaError_t set_kernel_attrs();   // once per process, before any launch or graph capture
 
 }  // namespace bzk

@@ -254,3 +254,29 @@ def test_outputs_verify_with_reference_verifier(prover, orc):
     for b in range(B):
         assert orc.verify(k, d, 1, SEED, 40 + b, np64(out["round_evals"][b]), np64(out["challenges"][b]),
                           np64(out["final_evals"][b]), np64(out["claims"][b])) == 0
+
+
+def test_cuda_graph_replay_and_recapture(prover):
+    B, d, k = 4, 2, 14
+    t = dev_tables(B, d, k)
+    ref = prover.prove(t, k, d, 0, flags=bzk.BZK_F_PRESERVE_INPUT)
+    out = bzk.Prover.alloc_outputs(B, k, d)
+    s = torch.cuda.Stream()
+    b = prover.batch(t, k, d, 0, None, 0, bzk.BZK_F_PRESERVE_INPUT | bzk.BZK_F_GRAPH, out)
+    for rep in range(3):                       # capture, then replays
+        for key in out:
+            out[key].zero_()
+        bzk.bzk_prove(prover.ctx, b, s)
+        s.synchronize()
+        for key in ref:
+            assert torch.equal(out[key], ref[key]), (rep, key)
+    # a different seed must not replay the old graph
+    seed2 = bytes([7]) + bytes(range(1, 32))
+    b2 = prover.batch(t, k, d, 0, seed2, 0, bzk.BZK_F_PRESERVE_INPUT | bzk.BZK_F_GRAPH, out)
+    bzk.bzk_prove(prover.ctx, b2, s)
+    s.synchronize()
+    ref2 = prover.prove(t, k, d, 0, seed=seed2, flags=bzk.BZK_F_PRESERVE_INPUT)
+    torch.cuda.synchronize()
+    for key in ref2:
+        assert torch.equal(out[key], ref2[key]), key
+    assert not torch.equal(ref2["challenges"], ref["challenges"])
