@@ -121,7 +121,7 @@ struct Plan {
 // tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
 // (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round, default on)
 struct Knobs {
-    uint64_t ppt_max = 16, waves = 4;
+    uint64_t ppt_max = 64, waves = 4;
     uint32_t prefetch = 1;
     Knobs() {
         if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
@@ -574,6 +574,7 @@ __global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, ui
         for (int i = 0; i < 8; ++i) acc ^= a[i] ^ (uint32_t)w[i] ^ (uint32_t)(w[i] >> 32);
         sink[tid] = acc;
     } else {
+        constexpr int CH = KIND == 5 ? 1 : (KIND == 6 ? 2 : 4);
         fe x[4], y;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
@@ -583,7 +584,11 @@ __global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, ui
         for (int i = 0; i < 8; ++i) y.l[i] = (seed ^ (0x9e3779b9u * (i + 3))) & (i == 7 ? 0x0fffffffu : ~0u);
         for (uint32_t it = 0; it < iters; ++it)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) x[c] = KIND == 2 ? mont_mul_v1(x[c], y) : mont_mul(x[c], y);
+            for (int c = 0; c < CH; ++c) {
+                if (KIND == 2) x[c] = mont_mul_v1(x[c], y);
+                else if (KIND == 8) x[c] = mont_mul2(x[c], y, x[(c + 1) & 3], y);
+                else x[c] = mont_mul(x[c], y);
+            }
         uint32_t acc = 0;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
@@ -602,7 +607,8 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
     int nsm = kSMs, clk_khz = 1965000;
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0);
     cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, 0);
-    const int threads = 256, blocks = nsm * 8;
+    // kinds 5-7: 2 CTAs of 256 threads per SM (the occupancy of k_round) with 1 / 2 / 4 chains per thread
+    const int threads = 256, blocks = (KIND >= 5 && KIND <= 7) ? nsm * 2 : nsm * 8;
     uint32_t *sink = nullptr;
     cudaError_t e = cudaMalloc(&sink, (size_t)blocks * threads * 4);
     if (e != cudaSuccess) return e;
@@ -619,7 +625,8 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     cudaFree(sink);
-    const double ops = (double)blocks * threads * iters * ((KIND <= 1 || KIND == 4) ? 32.0 : 4.0);
+    const double per = (KIND <= 1 || KIND == 4) ? 32.0 : (KIND == 5 ? 1.0 : (KIND == 6 ? 2.0 : 4.0));
+    const double ops = (double)blocks * threads * iters * per;   // kind 8 counts mont_mul2 calls
     *rate = ops / (ms * 1e-3) / ((double)clk_khz * 1e3) / nsm;   // per SM per clock (at the max clock)
     return e;
 }
@@ -789,7 +796,7 @@ bzk_status bzk_debug_sha256(const uint8_t *msgs, uint32_t msg_len, uint64_t n, u
 }
 
 bzk_status bzk_debug_bench(int kind, uint32_t iters, double *rate, void *cuda_stream) {
-    if (!rate || iters == 0 || kind < 0 || kind > 4) return BZK_EINVAL;
+    if (!rate || iters == 0 || kind < 0 || kind > 8) return BZK_EINVAL;
     cudaStream_t s = (cudaStream_t)cuda_stream;
     cudaError_t e = cudaErrorInvalidValue;
     switch (kind) {
@@ -798,6 +805,10 @@ bzk_status bzk_debug_bench(int kind, uint32_t iters, double *rate, void *cuda_st
         case 2: e = run_bench<2>(iters, rate, s); break;
         case 3: e = run_bench<3>(iters, rate, s); break;
         case 4: e = run_bench<4>(iters, rate, s); break;
+        case 5: e = run_bench<5>(iters, rate, s); break;
+        case 6: e = run_bench<6>(iters, rate, s); break;
+        case 7: e = run_bench<7>(iters, rate, s); break;
+        case 8: e = run_bench<8>(iters, rate, s); break;
     }
     return e == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }

@@ -247,8 +247,28 @@ __device__ __forceinline__ void row_a(uint32_t A[9], const uint32_t a[8], uint32
         : "r"(a[0]), "r"(a[2]), "r"(a[4]), "r"(a[6]), "r"(bi));
 }
 
-// reduction chains: A += p_even * m (A0 -> 0), B += p_odd * m
+// reduction chains: A += p_even * m (A0 -> 0), B += p_odd * m.
+// BN254 has p0 = 2^32 - 2^28 + 1 and -p^{-1} = -(2^28 + 1) mod 2^32, so the column-0 product
+// needs no multiplier: m = -(A0 + (A0 << 28)) and hi(A0 + m p0) = m - (m >> 4) + carry(A0 + m)
+// (exact: A0 + m p0 = 2^32 (m - (m >> 4)) + (A0 + m - (m << 28) mod 2^32), the last term being
+// 0 or 2^32 exactly as A0 + m carries).  Saves one IMAD and one IMAD.HI per row on the IMAD pipe.
+#ifndef BZK_M_ALU
+#define BZK_M_ALU 0      // 1: m via shift+add on the ALU pipe (fewer IMADs, longer dependency)
+#endif
+#ifndef BZK_P0_TRICK
+#define BZK_P0_TRICK 0   // 1: column-0 reduction product without IMAD.HI
+#endif
+__device__ __forceinline__ uint32_t mont_m(uint32_t a0) {
+#if !BZK_M_ALU
+    return a0 * BZK_NP0;
+#endif
+    uint32_t m;   // -(a0 + (a0 << 28)) on the ALU pipe (shift + add), kept out of the IMAD pipe
+    asm("{\n\t.reg .u32 t;\n\tshl.b32 t, %1, 28;\n\tadd.u32 t, t, %1;\n\tsub.u32 %0, 0, t;\n\t}" : "=r"(m) : "r"(a0));
+    return m;
+}
+
 __device__ __forceinline__ void red_a(uint32_t A[9], uint32_t m) {
+#if !BZK_P0_TRICK
     asm("mad.lo.cc.u32  %0, %9, %10, %0;\n\t"
         "madc.hi.cc.u32 %1, %9, %10, %1;\n\t"
         "madc.lo.cc.u32 %2, %9, %11, %2;\n\t"
@@ -261,6 +281,23 @@ __device__ __forceinline__ void red_a(uint32_t A[9], uint32_t m) {
         : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
           "+r"(A[8])
         : "r"(m), "n"(BZK_P0), "n"(BZK_P2), "n"(BZK_P4), "n"(BZK_P6));
+    return;
+#endif
+    const uint32_t h = m - (m >> 4);
+    uint32_t dummy;   // A0 + m == 0 mod 2^32; only its carry is used
+    asm("add.cc.u32     %9, %0, %10;\n\t"
+        "addc.cc.u32    %1, %1, %11;\n\t"
+        "madc.lo.cc.u32 %2, %10, %12, %2;\n\t"
+        "madc.hi.cc.u32 %3, %10, %12, %3;\n\t"
+        "madc.lo.cc.u32 %4, %10, %13, %4;\n\t"
+        "madc.hi.cc.u32 %5, %10, %13, %5;\n\t"
+        "madc.lo.cc.u32 %6, %10, %14, %6;\n\t"
+        "madc.hi.cc.u32 %7, %10, %14, %7;\n\t"
+        "addc.u32       %8, %8, 0;"
+        : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
+          "+r"(A[8]), "=r"(dummy)
+        : "r"(m), "r"(h), "n"(BZK_P2), "n"(BZK_P4), "n"(BZK_P6));
+    (void)dummy;
 }
 
 __device__ __forceinline__ void red_b(uint32_t B[9], uint32_t m) {
@@ -278,8 +315,9 @@ __device__ __forceinline__ void red_b(uint32_t B[9], uint32_t m) {
         : "r"(m), "n"(BZK_P1), "n"(BZK_P3), "n"(BZK_P5), "n"(BZK_P7));
 }
 
-// Montgomery product a*b*R^{-1} mod p; a, b canonical -> canonical.
-__device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
+// Lazy Montgomery product: returns t = a*b*R^{-1} + q*p < a*b/R + p (no final subtraction).
+// With p/R = 0.189 (BN254): a, b < 2p, or a < 4p and b < p  ->  t < 1.76p.
+__device__ __forceinline__ fe mont_mul_lz(const fe &a, const fe &b) {
     uint32_t A[9], B[9], L = 0;
     // row 0: plain products (no accumulation)
     asm("mul.lo.u32 %0, %9,  %13;\n\t"
@@ -312,7 +350,7 @@ __device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
             row_b(A, B, L, a.l, b.l[i]);
             row_a(A, a.l, b.l[i]);
         }
-        uint32_t m = A[0] * BZK_NP0;
+        uint32_t m = mont_m(A[0]);
         red_a(A, m);
         red_b(B, m);
         // divide by W: L = A1; A <- B; B <- A2..A8, 0, 0
@@ -341,13 +379,16 @@ __device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) {
           "=r"(r.l[7])
         : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
           "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
-    return fe_reduce_once(r);
+    return r;
 }
 
-// (x*y + u*v) * R^{-1} mod p with ONE Montgomery reduction (lazy sum of two products).
-// Each row adds x*y_i and u*v_i before the reduction row; with x, u < p the CIOS accumulator stays
-// below 3p + 1 (< 2^256 since 4p < 2^256), so the result needs at most two subtractions of p.
-__device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, const fe &v) {
+// Montgomery product a*b*R^{-1} mod p; a, b canonical -> canonical.
+__device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) { return fe_reduce_once(mont_mul_lz(a, b)); }
+
+// (x*y + u*v) * R^{-1} (+ q p) with ONE Montgomery reduction (lazy sum of two products).
+// Each row adds x*y_i and u*v_i before the reduction row.  Result < (x*y + u*v)/R + p: with
+// x, y, u, v < 2p it is < 2.52p (< 2^256 since 4p < 2^256); with x, u < p, y, v < 2^256 it is < 3p.
+__device__ __forceinline__ fe mont_mul2_lz(const fe &x, const fe &y, const fe &u, const fe &v) {
     uint32_t A[9], B[9], L = 0;
     asm("mul.lo.u32 %0, %9,  %13;\n\t"
         "mul.hi.u32 %1, %9,  %13;\n\t"
@@ -383,7 +424,7 @@ __device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, c
             row_b(A, B, 0u, u.l, v.l[i]);
             row_a(A, u.l, v.l[i]);
         }
-        uint32_t m = A[0] * BZK_NP0;
+        uint32_t m = mont_m(A[0]);
         red_a(A, m);
         red_b(B, m);
         L = A[1];
@@ -410,7 +451,117 @@ __device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, c
           "=r"(r.l[7])
         : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
           "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
-    return fe_reduce_once(fe_reduce_once(r));   // r <= 3p
+    return r;
+}
+
+// (x*y + u*v) * R^{-1} mod p, canonical; x, y, u, v canonical (result of the lazy form < 3p)
+__device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, const fe &v) {
+    return fe_reduce_once(fe_reduce_once(mont_mul2_lz(x, y, u, v)));
+}
+
+// ---------------------------------------------------------------- lazy ("< 2p") arithmetic
+// Hot-loop values are kept in [0, 2p) instead of [0, p); every bound below uses 4p < 2^256.
+
+// 2p (LE 32-bit limbs)
+#define BZK_2P0 0xe0000002u
+#define BZK_2P1 0x87c3eb27u
+#define BZK_2P2 0xf372e122u
+#define BZK_2P3 0x5067d090u
+#define BZK_2P4 0x0302b0bau
+#define BZK_2P5 0x70a08b6du
+#define BZK_2P6 0xc2634053u
+#define BZK_2P7 0x60c89ce5u
+
+// b + 2p - a  (a, b < 2p -> result in (0, 4p)); branch-free
+__device__ __forceinline__ fe lz_sub(const fe &b, const fe &a) {
+    fe t, r;
+    asm("sub.cc.u32  %0, %8,  %16;\n\t"
+        "subc.cc.u32 %1, %9,  %17;\n\t"
+        "subc.cc.u32 %2, %10, %18;\n\t"
+        "subc.cc.u32 %3, %11, %19;\n\t"
+        "subc.cc.u32 %4, %12, %20;\n\t"
+        "subc.cc.u32 %5, %13, %21;\n\t"
+        "subc.cc.u32 %6, %14, %22;\n\t"
+        "subc.u32    %7, %15, %23;"
+        : "=r"(t.l[0]), "=r"(t.l[1]), "=r"(t.l[2]), "=r"(t.l[3]), "=r"(t.l[4]), "=r"(t.l[5]), "=r"(t.l[6]),
+          "=r"(t.l[7])
+        : "n"(BZK_2P0), "n"(BZK_2P1), "n"(BZK_2P2), "n"(BZK_2P3), "n"(BZK_2P4), "n"(BZK_2P5), "n"(BZK_2P6),
+          "n"(BZK_2P7), "r"(a.l[0]), "r"(a.l[1]), "r"(a.l[2]), "r"(a.l[3]), "r"(a.l[4]), "r"(a.l[5]), "r"(a.l[6]),
+          "r"(a.l[7]));
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
+          "=r"(r.l[7])
+        : "r"(t.l[0]), "r"(t.l[1]), "r"(t.l[2]), "r"(t.l[3]), "r"(t.l[4]), "r"(t.l[5]), "r"(t.l[6]), "r"(t.l[7]),
+          "r"(b.l[0]), "r"(b.l[1]), "r"(b.l[2]), "r"(b.l[3]), "r"(b.l[4]), "r"(b.l[5]), "r"(b.l[6]), "r"(b.l[7]));
+    return r;
+}
+
+// x < 4p  ->  x mod 2p-range: subtract 2p when x >= 2p (result < 2p)
+__device__ __forceinline__ fe lz_red(const fe &x) {
+    fe s;
+    uint32_t borrow;
+    asm("sub.cc.u32  %0, %9,  %17;\n\t"
+        "subc.cc.u32 %1, %10, %18;\n\t"
+        "subc.cc.u32 %2, %11, %19;\n\t"
+        "subc.cc.u32 %3, %12, %20;\n\t"
+        "subc.cc.u32 %4, %13, %21;\n\t"
+        "subc.cc.u32 %5, %14, %22;\n\t"
+        "subc.cc.u32 %6, %15, %23;\n\t"
+        "subc.cc.u32 %7, %16, %24;\n\t"
+        "subc.u32    %8, 0, 0;"
+        : "=r"(s.l[0]), "=r"(s.l[1]), "=r"(s.l[2]), "=r"(s.l[3]), "=r"(s.l[4]), "=r"(s.l[5]),
+          "=r"(s.l[6]), "=r"(s.l[7]), "=r"(borrow)
+        : "r"(x.l[0]), "r"(x.l[1]), "r"(x.l[2]), "r"(x.l[3]), "r"(x.l[4]), "r"(x.l[5]), "r"(x.l[6]),
+          "r"(x.l[7]), "n"(BZK_2P0), "n"(BZK_2P1), "n"(BZK_2P2), "n"(BZK_2P3), "n"(BZK_2P4), "n"(BZK_2P5),
+          "n"(BZK_2P6), "n"(BZK_2P7));
+    fe r;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) r.l[i] = borrow ? x.l[i] : s.l[i];
+    return r;
+}
+
+// plain 256-bit add (caller guarantees no overflow, e.g. a < 2p, b < 2p)
+__device__ __forceinline__ fe lz_add(const fe &a, const fe &b) {
+    fe s;
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(s.l[0]), "=r"(s.l[1]), "=r"(s.l[2]), "=r"(s.l[3]), "=r"(s.l[4]), "=r"(s.l[5]),
+          "=r"(s.l[6]), "=r"(s.l[7])
+        : "r"(a.l[0]), "r"(a.l[1]), "r"(a.l[2]), "r"(a.l[3]), "r"(a.l[4]), "r"(a.l[5]), "r"(a.l[6]),
+          "r"(a.l[7]), "r"(b.l[0]), "r"(b.l[1]), "r"(b.l[2]), "r"(b.l[3]), "r"(b.l[4]), "r"(b.l[5]),
+          "r"(b.l[6]), "r"(b.l[7]));
+    return s;
+}
+
+// 288-bit accumulator for sums of lazy products (each < 3p): 8 limbs + a carry word
+struct acc9 { fe lo; uint32_t hi; };
+__device__ __forceinline__ acc9 acc9_zero() { acc9 a; a.lo = fe_zero(); a.hi = 0; return a; }
+__device__ __forceinline__ void acc9_add(acc9 &a, const fe &x) {
+    asm("add.cc.u32  %0, %0, %9;\n\t"
+        "addc.cc.u32 %1, %1, %10;\n\t"
+        "addc.cc.u32 %2, %2, %11;\n\t"
+        "addc.cc.u32 %3, %3, %12;\n\t"
+        "addc.cc.u32 %4, %4, %13;\n\t"
+        "addc.cc.u32 %5, %5, %14;\n\t"
+        "addc.cc.u32 %6, %6, %15;\n\t"
+        "addc.cc.u32 %7, %7, %16;\n\t"
+        "addc.u32    %8, %8, 0;"
+        : "+r"(a.lo.l[0]), "+r"(a.lo.l[1]), "+r"(a.lo.l[2]), "+r"(a.lo.l[3]), "+r"(a.lo.l[4]), "+r"(a.lo.l[5]),
+          "+r"(a.lo.l[6]), "+r"(a.lo.l[7]), "+r"(a.hi)
+        : "r"(x.l[0]), "r"(x.l[1]), "r"(x.l[2]), "r"(x.l[3]), "r"(x.l[4]), "r"(x.l[5]), "r"(x.l[6]), "r"(x.l[7]));
 }
 
 __device__ __forceinline__ fe fe_const(int which) {

@@ -6,18 +6,29 @@ namespace bzk {
 template <>
 cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
                                 const RoundParams &p) {
+    const size_t sm = first ? round_smem_bytes<BZK_D, true>(threads) : round_smem_bytes<BZK_D, false>(threads);
     if (order == 0) {
-        if (first) k_round<BZK_D, 0, true><<<grid, threads, 0, s>>>(p);
-        else       k_round<BZK_D, 0, false><<<grid, threads, 0, s>>>(p);
+        if (first) k_round<BZK_D, 0, true><<<grid, threads, sm, s>>>(p);
+        else       k_round<BZK_D, 0, false><<<grid, threads, sm, s>>>(p);
     } else {
-        if (first) k_round<BZK_D, 1, true><<<grid, threads, 0, s>>>(p);
-        else       k_round<BZK_D, 1, false><<<grid, threads, 0, s>>>(p);
+        if (first) k_round<BZK_D, 1, true><<<grid, threads, sm, s>>>(p);
+        else       k_round<BZK_D, 1, false><<<grid, threads, sm, s>>>(p);
     }
     return cudaGetLastError();
 }
 
 template <>
+size_t round_smem<BZK_D>(bool first, uint32_t threads) {
+    return first ? round_smem_bytes<BZK_D, true>(threads) : round_smem_bytes<BZK_D, false>(threads);
+}
+
+template <>
 cudaError_t set_kernel_attrs<BZK_D>() {
+    const int big = 200 * 1024;
+    cudaFuncSetAttribute(k_round<BZK_D, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
+    cudaFuncSetAttribute(k_round<BZK_D, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
+    cudaFuncSetAttribute(k_round<BZK_D, 0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
+    cudaFuncSetAttribute(k_round<BZK_D, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
     cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     return cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
 }

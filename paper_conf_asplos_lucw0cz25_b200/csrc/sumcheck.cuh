@@ -92,32 +92,78 @@ __device__ __forceinline__ void block_reduce(fe (&acc)[V], fe *smem) {
 
 // ---------------------------------------------------------------- per-pair math
 
-// number of summed evaluation points: all t = 0..D, or t in {0, 2..D} when g(1) is derived
+// Summed evaluation points of the global round kernels (the "infinity" point is the leading
+// coefficient of g_i, i.e. the sum of prod_m delta_m -- it replaces t = d and needs no additions):
+//   FIRST  (round 1)        : t = 0, 1, ..., d-1, inf          (d = 1: t = 0, 1)
+//   DERIVE (fused rounds)   : t = 0, 2, ..., d-1, inf          (d = 1: t = 0); g(1) = claim - g(0)
+// finalize_round() rebuilds g(d) = sum_{j<d} (-1)^{d-1-j} C(d,j) g(j) + d! * c_inf.
 template <int D, bool DERIVE> struct Pts { static constexpr int NV = DERIVE ? D : D + 1; };
 
-// Evaluate two pairs (a, a + delta) and (a2, a2 + delta2) at the summed points and accumulate.
-// a / a2 are overwritten (they walk through v(t) = a + t*delta).  Products of the two pairs
-// share one Montgomery reduction (mont_mul2); every sum carries R^{-(D-1)}.
 template <int D, bool DERIVE>
-__device__ __forceinline__ void eval_two(fe (&a)[D], const fe (&delta)[D], fe (&a2)[D], const fe (&delta2)[D],
-                                         fe (&acc)[Pts<D, DERIVE>::NV]) {
+__device__ __forceinline__ constexpr int point_t(int idx) {   // -1 = infinity
+    if (D == 1) return idx;
+    if (idx == Pts<D, DERIVE>::NV - 1) return -1;
+    return DERIVE ? (idx == 0 ? 0 : idx + 1) : idx;
+}
+
+// Evaluate two pairs at the summed points and accumulate (lazy arithmetic, values < 2p).
+// Inputs per table m: a[m] (= v(0)) and s[m], which is b = v(1) in round 1 and delta = b - a in
+// the fused rounds (whichever the point set needs, to keep registers down).  Products of the two
+// pairs share ONE Montgomery reduction (mont_mul2_lz); sums go to 288-bit accumulators; every sum
+// carries R^{-(D-1)}.
+template <int D, bool DERIVE>
+__device__ __forceinline__ void eval_two(const fe (&a)[D], const fe (&s)[D], const fe (&a2)[D], const fe (&s2)[D],
+                                         acc9 (&acc)[Pts<D, DERIVE>::NV]) {
+    constexpr int NV = Pts<D, DERIVE>::NV;
+    fe v[D], v2[D], dl[D], dl2[D];
 #pragma unroll
-    for (int t = 0; t <= D; ++t) {
-        if (t > 0) {
+    for (int idx = 0; idx < NV; ++idx) {
+        const int t = point_t<D, DERIVE>(idx);
+        if ((t < 0 || t == 2) && !DERIVE) {   // round 1: delta = b - a on demand
 #pragma unroll
-            for (int m = 0; m < D; ++m) { a[m] = fe_add(a[m], delta[m]); a2[m] = fe_add(a2[m], delta2[m]); }
+            for (int m = 0; m < D; ++m) {
+                dl[m] = lz_sub(s[m], a[m]);
+                dl2[m] = lz_sub(s2[m], a2[m]);
+                if (!(D == 2 && m == 0)) { dl[m] = lz_red(dl[m]); dl2[m] = lz_red(dl2[m]); }   // see load_pair
+            }
         }
-        if (DERIVE && t == 1) continue;
-        const int idx = DERIVE ? (t == 0 ? 0 : t - 1) : t;
-        if (D == 1) {
-            acc[idx] = fe_add(acc[idx], fe_add(a[0], a2[0]));
-        } else {
-            fe p = a[0], p2 = a2[0];
+        const fe *x, *x2;
+        if (t == 0) { x = a; x2 = a2; }
+        else if (t == 1) { x = s; x2 = s2; }                       // FIRST only: s = b
+        else if (t < 0) { x = DERIVE ? s : dl; x2 = DERIVE ? s2 : dl2; }
+        else {
 #pragma unroll
-            for (int m = 1; m < D - 1; ++m) { p = mont_mul(p, a[m]); p2 = mont_mul(p2, a2[m]); }
-            acc[idx] = fe_add(acc[idx], mont_mul2(p, a[D - 1], p2, a2[D - 1]));
+            for (int m = 0; m < D; ++m) {
+                const fe &d1 = DERIVE ? s[m] : dl[m];
+                const fe &d2 = DERIVE ? s2[m] : dl2[m];
+                if (t == 2) {
+                    // DERIVE: a + 2 delta;  FIRST: b + delta
+                    v[m] = lz_red(lz_add(DERIVE ? a[m] : s[m], d1));
+                    v2[m] = lz_red(lz_add(DERIVE ? a2[m] : s2[m], d2));
+                    if (DERIVE) { v[m] = lz_red(lz_add(v[m], d1)); v2[m] = lz_red(lz_add(v2[m], d2)); }
+                } else {
+                    v[m] = lz_red(lz_add(v[m], d1));
+                    v2[m] = lz_red(lz_add(v2[m], d2));
+                }
+            }
+            x = v; x2 = v2;
+        }
+        if (D == 1) {
+            acc9_add(acc[idx], lz_add(x[0], x2[0]));
+        } else {
+            fe p = x[0], p2 = x2[0];
+#pragma unroll
+            for (int m = 1; m < D - 1; ++m) { p = mont_mul_lz(p, x[m]); p2 = mont_mul_lz(p2, x2[m]); }
+            acc9_add(acc[idx], mont_mul2_lz(p, x[D - 1], p2, x2[D - 1]));
         }
     }
+}
+
+// 288-bit accumulator -> canonical field element: hi * 2^256 + lo = hi * (R mod p) + lo (mod p)
+__device__ __forceinline__ fe acc9_to_fe(const acc9 &a) {
+    fe h = fe_zero();
+    h.l[0] = a.hi;
+    return fe_add(fe_reduce_256(a.lo), mont_mul(h, fe_const(2)));   // hi * R^2 * R^-1 = hi * R
 }
 
 // single pair, every point t = 0..D (used by the on-chip tail)
@@ -146,6 +192,11 @@ __device__ __forceinline__ fe fold1(const fe &a, const fe &b, const fe &rmont) {
     return fe_add(a, mont_mul(rmont, fe_sub(b, a)));
 }
 
+// lazy fold for the hot loop: a, b < 2p, rmont < p  ->  a + r (b - a) (mod p), result < 2p
+__device__ __forceinline__ fe fold_lz(const fe &a, const fe &b, const fe &rmont) {
+    return lz_red(lz_add(a, mont_mul_lz(rmont, lz_sub(b, a))));
+}
+
 // ---------------------------------------------------------------- per-round finalisation
 
 // g(r) from g(0..D) by Lagrange interpolation on the nodes 0..D (all standard form; rm = r R).
@@ -163,22 +214,56 @@ __device__ __forceinline__ fe lagrange_at(const fe (&g)[D + 1], const fe &rm, co
     return acc;
 }
 
-// Fix the R^{-(D-1)} scale of the round sums, complete g(1) when derived, absorb g into the
-// transcript, derive r_i, write the round's outputs and the next claim.  ONE thread per proof.
-template <int D, bool DERIVE>
-__device__ __forceinline__ void finalize_round(fe (&S)[Pts<D, DERIVE>::NV], uint32_t round, ProofState &ps,
+// x * c for a small non-negative integer c (finalisation only)
+__device__ __forceinline__ fe fe_mul_small(const fe &x, int c) {
+    fe r = fe_zero(), y = x;
+    for (; c; c >>= 1) {
+        if (c & 1) r = fe_add(r, y);
+        y = fe_add(y, y);
+    }
+    return r;
+}
+
+// g(D) from g(0..D-1) and the leading coefficient c_inf:  sum_j (-1)^{D-1-j} C(D,j) g(j) + D! c_inf
+template <int D>
+__device__ __forceinline__ fe extrapolate_top(const fe (&g)[D + 1], const fe &cinf) {
+    int binom = 1, fact = 1;
+    fe pos = fe_zero(), neg = fe_zero();
+    for (int j = 0; j < D; ++j) {
+        const fe term = fe_mul_small(g[j], binom);
+        if (((D - 1 - j) & 1) == 0) pos = fe_add(pos, term); else neg = fe_add(neg, term);
+        binom = binom * (D - j) / (j + 1);
+    }
+    for (int j = 2; j <= D; ++j) fact *= j;
+    return fe_add(fe_sub(pos, neg), fe_mul_small(cinf, fact));
+}
+
+// Fix the R^{-(D-1)} scale of the round sums, rebuild g(0..D), absorb g into the transcript,
+// derive r_i, write the round's outputs and the next claim.  ONE thread per proof.
+//   MODE 0: S holds g(0..D) directly (on-chip tail)
+//   MODE 1: S holds the FIRST point set, MODE 2 the DERIVE point set (see Pts / point_t)
+template <int D, int MODE>
+__device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], uint32_t round, ProofState &ps,
                                                fe *round_evals, fe *challenges, fe *claims, const fe *consts,
                                                fe *rmont_out) {
+    constexpr int NS = MODE == 2 ? D : D + 1;
     fe g[D + 1];
     const fe RD = fe_R_pow(D);
-    if (DERIVE) {
-        g[0] = mont_mul(S[0], RD);
-        g[1] = fe_sub(ps.claim, g[0]);
+    fe fixd[NS];
 #pragma unroll
-        for (int t = 2; t <= D; ++t) g[t] = mont_mul(S[t - 1], RD);
+    for (int i = 0; i < NS; ++i) fixd[i] = mont_mul(S[i], RD);
+    if (MODE == 0) {
+#pragma unroll
+        for (int t = 0; t <= D; ++t) g[t] = fixd[t];
     } else {
+        constexpr bool DERIVE = MODE == 2;
 #pragma unroll
-        for (int t = 0; t <= D; ++t) g[t] = mont_mul(S[t], RD);
+        for (int idx = 0; idx < NS; ++idx) {
+            const int t = point_t<D, DERIVE>(idx);
+            if (t >= 0) g[t] = fixd[idx];
+        }
+        if (DERIVE) g[1] = fe_sub(ps.claim, g[0]);
+        if (D >= 2) g[D] = extrapolate_top<D>(g, fixd[NS - 1]);
     }
     uint32_t st[8];
 #pragma unroll
@@ -250,7 +335,7 @@ static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed3
 
 template <int D, int ORDER, bool FIRST>
 __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, uint64_t j, const fe &rm,
-                                          fe (&a)[D], fe (&delta)[D]) {
+                                          fe (&a)[D], fe (&sv)[D]) {
 #pragma unroll
     for (int m = 0; m < D; ++m) {
         fe lo, hi;
@@ -264,22 +349,24 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
             if (ORDER == 0) {
                 fe x0 = ld_fe_stream(T + 4 * j), x1 = ld_fe_stream(T + 4 * j + 1);
                 fe x2 = ld_fe_stream(T + 4 * j + 2), x3 = ld_fe_stream(T + 4 * j + 3);
-                lo = fold1(x0, x1, rm);
-                hi = fold1(x2, x3, rm);
+                lo = fold_lz(x0, x1, rm);
+                hi = fold_lz(x2, x3, rm);
                 st_fe(U + 2 * j, lo);
                 st_fe(U + 2 * j + 1, hi);
             } else {
                 // previous round paired (x, x + 2h); this round pairs (j, j + h)
                 fe x0 = ld_fe_stream(T + j), x1 = ld_fe_stream(T + j + 2 * h);
                 fe x2 = ld_fe_stream(T + j + h), x3 = ld_fe_stream(T + j + 3 * h);
-                lo = fold1(x0, x1, rm);
-                hi = fold1(x2, x3, rm);
+                lo = fold_lz(x0, x1, rm);
+                hi = fold_lz(x2, x3, rm);
                 st_fe(U + j, lo);
                 st_fe(U + j + h, hi);
             }
         }
         a[m] = lo;
-        delta[m] = fe_sub(hi, lo);
+        // round 1: b; fused rounds: delta (for d = 2 the table-0 delta may stay < 4p: it only
+        // meets mont_mul2_lz(<4p, <2p, <4p, <2p) < 4.02p)
+        sv[m] = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
     }
 }
 
@@ -314,6 +401,97 @@ __device__ __forceinline__ void prefetch_pairs(const fe *src, uint64_t h, uint64
     }
 }
 
+// ---------------------------------------------------------------- cp.async staging of fold groups
+//
+// A "group" is what one fold step of one thread consumes: the E entries (E = 2 in round 1, 4 in a
+// fused round) of ONE table for ONE pair.  Groups stream through a per-thread ring of kStageSlots
+// shared-memory slots filled by cp.async (LDGSTS, no registers held while in flight) kStageDist
+// groups ahead of use, so the IMAD chains of the current group overlap the DRAM latency of the
+// next ones.  Slot layout is transposed (chunk-major across the CTA's threads): the 16-byte chunk c
+// of thread t sits at ((slot * 2E + c) * blockDim + t) * 16, so both the cp.async writes and the
+// LDS.128 reads of a warp are bank-conflict free.
+#ifndef BZK_STAGE
+#define BZK_STAGE 0   // measured slower on B200; kept as an option
+#endif
+constexpr int kStageDist = 2;
+constexpr int kStageSlots = kStageDist + 1;
+
+template <bool FIRST> struct GroupE { static constexpr int E = FIRST ? 2 : 4; };
+
+template <int D, int ORDER, bool FIRST>
+__device__ __forceinline__ const fe *group_entry(const fe *src, uint64_t h, uint64_t jj, int m, int e) {
+    if (FIRST) {
+        const fe *T = src + (size_t)m * (2 * h);
+        return ORDER == 0 ? T + 2 * jj + e : T + jj + (e ? h : 0);
+    }
+    const fe *T = src + (size_t)m * (4 * h);
+    if (ORDER == 0) return T + 4 * jj + e;
+    // MSB fused: the fold pairs are (x, x + 2h); this round pairs (jj, jj + h)
+    const uint64_t off[4] = {0, 2 * h, h, 3 * h};
+    return T + jj + off[e];
+}
+
+__device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc) {
+    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int D, int ORDER, bool FIRST>
+__device__ __forceinline__ void issue_group(uint4 *ring, uint32_t slot, const fe *src, uint64_t h, uint64_t jj,
+                                            int m) {
+    constexpr int E = GroupE<FIRST>::E;
+    if (jj < h) {
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+            const uint4 *g = reinterpret_cast<const uint4 *>(group_entry<D, ORDER, FIRST>(src, h, jj, m, e));
+#pragma unroll
+            for (int c = 0; c < 2; ++c)
+                cp_async16(&ring[((size_t)(slot * 2 * E + 2 * e + c)) * blockDim.x + threadIdx.x], g + c);
+        }
+    }
+    cp_async_commit();   // always commit (possibly empty) so group counting stays uniform
+}
+
+__device__ __forceinline__ fe lds_entry(const uint4 *ring, uint32_t chunk0) {
+    const uint4 x = ring[(size_t)chunk0 * blockDim.x + threadIdx.x];
+    const uint4 y = ring[(size_t)(chunk0 + 1) * blockDim.x + threadIdx.x];
+    fe r;
+    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
+    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+    return r;
+}
+
+// consume group (q, m) of the current iteration from its ring slot: fold (fused rounds) or pass
+// through (round 1); write the folded entries to dst; return (a, b - a)
+template <int D, int ORDER, bool FIRST>
+__device__ __forceinline__ void consume_group(const uint4 *ring, uint32_t slot, fe *dst, uint64_t h, uint64_t jj,
+                                              int m, const fe &rm, fe &a, fe &sv) {
+    constexpr int E = GroupE<FIRST>::E;
+    const uint32_t c0 = slot * 2 * E;
+    fe lo, hi;
+    if (FIRST) {
+        lo = lds_entry(ring, c0);
+        hi = lds_entry(ring, c0 + 2);
+    } else {
+        lo = fold_lz(lds_entry(ring, c0), lds_entry(ring, c0 + 2), rm);
+        hi = fold_lz(lds_entry(ring, c0 + 4), lds_entry(ring, c0 + 6), rm);
+        fe *U = dst + (size_t)m * (2 * h);
+        if (ORDER == 0) { st_fe(U + 2 * jj, lo); st_fe(U + 2 * jj + 1, hi); }
+        else            { st_fe(U + jj, lo);     st_fe(U + jj + h, hi); }
+    }
+    a = lo;
+    sv = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));   // see load_pair
+}
+
+// dynamic shared memory of k_round (bytes) for a CTA of `threads`
+template <int D, bool FIRST>
+constexpr size_t round_smem_bytes(uint32_t threads) {
+    return BZK_STAGE ? (size_t)kStageSlots * 2 * GroupE<FIRST>::E * 16 * threads : 0;
+}
+
 template <int D, int ORDER, bool FIRST>
 __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
     constexpr bool DERIVE = !FIRST;
@@ -322,39 +500,81 @@ __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(Rou
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
     const uint64_t h = 1ull << P.log_h;
-    fe acc[NV];
+    acc9 wacc[NV];
 #pragma unroll
-    for (int t = 0; t < NV; ++t) acc[t] = fe_zero();
+    for (int t = 0; t < NV; ++t) wacc[t] = acc9_zero();
 
     const fe *src = P.src + (size_t)b * D * (FIRST ? 2 * h : 4 * h);
     fe *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const fe rm = FIRST ? fe_zero() : P.ps[b].rmont;
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     const uint32_t lane = threadIdx.x & 31;
+#ifdef BZK_STAGGER_NS
+    // experiment: de-phase the warps of a CTA so their IMAD-heavy and ALU-heavy stretches interleave
+    if (BZK_STAGGER_NS > 0) __nanosleep((threadIdx.x >> 5) % 4 * BZK_STAGGER_NS);
+#endif
+#if BZK_STAGE
+    extern __shared__ __align__(16) uint4 ring[];
+    {
+        const uint64_t j0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+        // group g -> iteration g / (2D), pair slot q = (g % 2D) / D, table m = g % D
+        auto g_jj = [&](uint64_t g) { return j0 + (g / (2 * D)) * 2 * stride + ((g % (2 * D)) / D) * stride; };
+#pragma unroll
+        for (int g = 0; g < kStageDist; ++g)
+            issue_group<D, ORDER, FIRST>(ring, g % kStageSlots, src, h, g_jj(g), g % D);
+        uint64_t g = 0;
+        for (uint64_t j = j0; j < h; j += 2 * stride) {
+            fe a[2][D], sv[2][D];
+#pragma unroll
+            for (int q = 0; q < 2; ++q)
+#pragma unroll
+                for (int m = 0; m < D; ++m, ++g) {
+                    const uint64_t gn = g + kStageDist;
+                    issue_group<D, ORDER, FIRST>(ring, (uint32_t)(gn % kStageSlots), src, h, g_jj(gn), (int)(gn % D));
+                    cp_async_wait<kStageDist>();
+                    const uint64_t jj = j + q * stride;
+                    if (jj < h) {
+                        consume_group<D, ORDER, FIRST>(ring, (uint32_t)(g % kStageSlots), dst, h, jj, m, rm, a[q][m],
+                                                       sv[q][m]);
+                    } else {
+                        a[q][m] = fe_zero();
+                        sv[q][m] = fe_zero();
+                    }
+                }
+            eval_two<D, DERIVE>(a[0], sv[0], a[1], sv[1], wacc);
+        }
+        cp_async_wait<0>();
+    }
+#else
     for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += 2 * stride) {
         if (P.prefetch && lane == 0) {
             prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
             prefetch_pairs<D, ORDER, FIRST>(src, h, j + 3 * stride);
         }
-        fe a[D], da[D], a2[D], da2[D];
-        load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, da);
+        fe a[D], sv[D], a2[D], sv2[D];
+        load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, sv);
         const uint64_t j2 = j + stride;
         if (j2 < h) {
-            load_pair<D, ORDER, FIRST>(src, dst, h, j2, rm, a2, da2);
+            load_pair<D, ORDER, FIRST>(src, dst, h, j2, rm, a2, sv2);
         } else {
 #pragma unroll
-            for (int m = 0; m < D; ++m) { a2[m] = fe_zero(); da2[m] = fe_zero(); }
+            for (int m = 0; m < D; ++m) { a2[m] = fe_zero(); sv2[m] = fe_zero(); }
         }
-        eval_two<D, DERIVE>(a, da, a2, da2, acc);
+        eval_two<D, DERIVE>(a, sv, a2, sv2, wacc);
     }
 
+#endif
+
+    fe acc[NV];
+#pragma unroll
+    for (int t = 0; t < NV; ++t) acc[t] = acc9_to_fe(wacc[t]);
     block_reduce<NV>(acc, s_red);
     fe *evals = P.round_evals + (size_t)b * P.k * (D + 1);
     fe *chals = P.challenges + (size_t)b * P.k;
     fe *claim = P.claims ? P.claims + b : nullptr;
     if (P.ctas == 1) {
         if (threadIdx.x == 0)
-            finalize_round<D, DERIVE>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
+            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
         return;
     }
     fe *part = P.partials + (size_t)b * P.ctas * NV;
@@ -377,7 +597,7 @@ __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(Rou
     block_reduce<NV>(acc, s_red);
     if (threadIdx.x == 0) {
         P.tickets[b] = 0;
-        finalize_round<D, DERIVE>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
+        finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
     }
 }
 
@@ -434,7 +654,8 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
             fe lo, hi;
             if (ORDER == 0) { lo = ld_fe(T + 2 * y); hi = ld_fe(T + 2 * y + 1); }
             else            { lo = ld_fe(T + y);     hi = ld_fe(T + y + 2 * h0); }
-            A[x] = fold1(lo, hi, rm);
+            // entries written by a fused round are lazily reduced (< 2p): canonicalise first
+            A[x] = fold1(fe_reduce_once(lo), fe_reduce_once(hi), rm);
         }
     }
     __syncthreads();
@@ -458,7 +679,7 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
         block_reduce<D + 1>(acc, s_red);
         if (threadIdx.x == 0) {
             fe rm;
-            finalize_round<D, false>(acc, i, P.ps[b], evals, chals, claim, P.consts, &rm);
+            finalize_round<D, 0>(acc, i, P.ps[b], evals, chals, claim, P.consts, &rm);
             s_r = rm;
         }
         __syncthreads();
@@ -489,5 +710,7 @@ cudaError_t launch_tail(uint32_t order, uint32_t grid, uint32_t threads, size_t 
                         const TailParams &p);
 template <int D>
 cudaError_t set_kernel_attrs();   // once per process, before any launch or graph capture
+template <int D>
+size_t round_smem(bool first, uint32_t threads);
 
 }  // namespace bzk
