@@ -546,23 +546,31 @@ __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(Rou
         cp_async_wait<0>();
     }
 #else
-    for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += 2 * stride) {
-        if (P.prefetch && lane == 0) {
-            prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
-            prefetch_pairs<D, ORDER, FIRST>(src, h, j + 3 * stride);
-        }
-        fe a[D], sv[D], a2[D], sv2[D];
-        load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, sv);
-        const uint64_t j2 = j + stride;
-        if (j2 < h) {
-            load_pair<D, ORDER, FIRST>(src, dst, h, j2, rm, a2, sv2);
-        } else {
+    // One pair per loop iteration (keeps the loop body -- 2d folds + one two-pair evaluation -- small
+    // enough for the instruction cache); every second pair is held in registers and evaluated
+    // together with the next one, so the two pairs' products share one Montgomery reduction.
+    {
+        fe ha[D], hs[D];
+        bool held = false;
+        for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
+            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
+            fe a[D], sv[D];
+            load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, sv);
+            if (held) {
+                eval_two<D, DERIVE>(ha, hs, a, sv, wacc);
+            } else {
 #pragma unroll
-            for (int m = 0; m < D; ++m) { a2[m] = fe_zero(); sv2[m] = fe_zero(); }
+                for (int m = 0; m < D; ++m) { ha[m] = a[m]; hs[m] = sv[m]; }
+            }
+            held = !held;
         }
-        eval_two<D, DERIVE>(a, sv, a2, sv2, wacc);
+        if (held) {
+            fe z[D];
+#pragma unroll
+            for (int m = 0; m < D; ++m) z[m] = fe_zero();
+            eval_two<D, DERIVE>(ha, hs, z, z, wacc);
+        }
     }
-
 #endif
 
     fe acc[NV];
