@@ -43,6 +43,7 @@ def lib():
         L.orc_prove_batch.argtypes = [u32, u32, u32, u8p, u64, u64, u64p, u64p, u64p, u64p, u64p,
                                       ctypes.c_int]
         L.orc_alg1.argtypes = [u32, u64p, u64p, u64p]
+        L.orc_prove_given.argtypes = [u32, u32, u32, u64p, u64p, u64p, u64p, u64p, u64p]
         L.orc_verify.argtypes = [u32, u32, u32, u8p, u64, u64p, u64p, u64p, u64p]
         L.orc_mle.argtypes = [u32, u64p, u64p, u64p]
         L.orc_hsum.argtypes = [u32, u32, u64p, u64p]
@@ -90,6 +91,21 @@ def prove(tables: np.ndarray, k: int, d: int, order: int, seed: bytes, index: in
     s = lib().orc_prove(k, d, order, seed, index, _p(tables), _p(ev), _p(ch), _p(fi), _p(cl))
     if s:
         raise ValueError(f"orc_prove failed: {s}")
+    return {"round_evals": ev, "challenges": ch, "final_evals": fi, "claims": cl}
+
+
+def prove_given(tables: np.ndarray, k: int, d: int, order: int, challenges: np.ndarray):
+    """Paper-literal mode (Alg. 1): challenges [k][4] are inputs."""
+    tables = np.ascontiguousarray(tables, dtype=np.uint64)
+    challenges = np.ascontiguousarray(challenges, dtype=np.uint64)
+    assert tables.shape == (d, 1 << k, 4) and challenges.shape == (k, 4)
+    ev = np.zeros((k, d + 1, 4), np.uint64)
+    ch = np.zeros((k, 4), np.uint64)
+    fi = np.zeros((d, 4), np.uint64)
+    cl = np.zeros((4,), np.uint64)
+    s = lib().orc_prove_given(k, d, order, _p(tables), _p(challenges), _p(ev), _p(ch), _p(fi), _p(cl))
+    if s:
+        raise ValueError(f"orc_prove_given failed: {s}")
     return {"round_evals": ev, "challenges": ch, "final_evals": fi, "claims": cl}
 
 

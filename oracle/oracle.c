@@ -316,9 +316,9 @@ enum { ORC_OK = 0, ORC_EINVAL = 1, ORC_ENONCANON = 4, ORC_ENOMEM = 2 };
  * round_evals: [k][d+1][4]; challenges: [k][4]; final_evals: [d][4]; claim: [4] (may be NULL).
  * order 0 = LSB (pairs (2j, 2j+1), binds x_1 first); 1 = MSB (pairs (j, j+h), Alg. 1).
  */
-int orc_prove(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], uint64_t I,
-              const uint64_t *tables, uint64_t *round_evals, uint64_t *challenges,
-              uint64_t *final_evals, uint64_t *claim) {
+static int prove_impl(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], uint64_t I,
+                      const uint64_t *tables, uint64_t *round_evals, uint64_t *challenges,
+                      uint64_t *final_evals, uint64_t *claim, const uint64_t *given_r) {
     if (k > 30 || d < 1 || d > 4 || order > 1) return ORC_EINVAL;
     ensure_mu();
     const uint64_t N = (uint64_t)1 << k;
@@ -361,8 +361,14 @@ int orc_prove(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], ui
             }
             g[t] = acc;
         }
-        /* (b), (c) transcript -> r_i */
-        fr r = transcript_round(state, g, d);
+        /* (b), (c) transcript -> r_i; or, paper-literal mode (Alg. 1), r_i given */
+        fr r;
+        if (given_r) {
+            memcpy(r.v, given_r + 4 * (uint64_t)(i - 1), 32);
+            if (!fr_is_canon(&r)) { free(T); return ORC_ENONCANON; }
+        } else {
+            r = transcript_round(state, g, d);
+        }
         for (uint32_t t = 0; t <= d; ++t)
             memcpy(round_evals + 4 * ((uint64_t)(i - 1) * (d + 1) + t), g[t].v, 32);
         memcpy(challenges + 4 * (uint64_t)(i - 1), r.v, 32);
@@ -382,6 +388,20 @@ int orc_prove(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], ui
     if (claim) memcpy(claim, H.v, 32);
     free(T);
     return ORC_OK;
+}
+
+int orc_prove(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], uint64_t I,
+              const uint64_t *tables, uint64_t *round_evals, uint64_t *challenges,
+              uint64_t *final_evals, uint64_t *claim) {
+    return prove_impl(k, d, order, seed, I, tables, round_evals, challenges, final_evals, claim, NULL);
+}
+
+/* Paper-literal mode: challenges r_1..r_k are inputs (Alg. 1), no transcript.  The same
+ * fold algorithm; `challenges` is read and copied through unchanged. */
+int orc_prove_given(uint32_t k, uint32_t d, uint32_t order, const uint64_t *tables, const uint64_t *given_r,
+                    uint64_t *round_evals, uint64_t *challenges_out, uint64_t *final_evals, uint64_t *claim) {
+    uint8_t seed[32] = {0};
+    return prove_impl(k, d, order, seed, 0, tables, round_evals, challenges_out, final_evals, claim, given_r);
 }
 
 /* batch of proofs over pthreads (one proof per task) */

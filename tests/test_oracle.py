@@ -345,3 +345,34 @@ def test_golden_proof_regression(orc):
         else:
             key, vals = r[0], [int(v, 16) for v in r[1:]]
             assert ints(out[key]) == vals, (cur, key)
+
+
+@pytest.mark.parametrize("order", [0, 1])
+@pytest.mark.parametrize("d", [1, 2, 3])
+def test_given_challenge_mode(orc, d, order):
+    """Paper-literal mode (Alg. 1, r_i given): fed the Fiat-Shamir challenges it reproduces the FS
+    proof; for d = 1, MSB it equals Alg. 1 line by line; with other challenges the round invariant
+    and final check still hold."""
+    k = 7
+    t = inputs.gen_tables(1, d, k, first_index=12)[0]
+    fs = orc.prove(t, k, d, order, SEED, 12)
+    given = orc.prove_given(t, k, d, order, fs["challenges"])
+    for key in fs:
+        assert np.array_equal(given[key], fs[key]), key
+    rng = np.random.default_rng(d)
+    r = orc.to_limbs([int(x) * 0x9E3779B97F4A7C15 % P for x in rng.integers(1, 2**62, size=k)])
+    out = orc.prove_given(t, k, d, order, r)
+    assert np.array_equal(out["challenges"], r)
+    if d == 1 and order == 1:
+        assert np.array_equal(orc.alg1(t[0], r), out["round_evals"])
+    ev = [ints(out["round_evals"][i]) for i in range(k)]
+    claim = ints(out["claims"])[0]
+    for i in range(k):
+        assert (ev[i][0] + ev[i][1]) % P == claim
+        claim = py.lagrange_eval(ev[i], ints(r)[i])
+    prod = 1
+    for f in ints(out["final_evals"]):
+        prod = prod * f % P
+    assert prod == claim
+    rho = py.rho_point(ints(r), k, order)
+    assert ints(out["final_evals"])[0] == py.mle(ints(t[0]), rho)
