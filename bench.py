@@ -41,6 +41,8 @@ CONFIGS = {
                                      "consume mode"),
     "m0": (1024, 1, 20, 1, "uniform", "paper shape (Table 4 analogue): 1024 proofs x single multilinear (d=1), "
                                       "k=20, MSB order = Alg. 1 pairing"),
+    "m0lit": (1024, 1, 20, 1, "uniform", "paper-literal Table 4 analogue: 1024 proofs x single multilinear (d=1), "
+                                         "k=20, MSB = Alg. 1 pairing, challenges given (no Fiat-Shamir, P:111)"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -317,11 +319,19 @@ def main():
     first, _ = shard.weak_range(B, rank)
     consume = args.config == "c3"
     flags = 0 if consume else bzk.BZK_F_PRESERVE_INPUT
+    if args.config == "m0lit":
+        flags |= bzk.BZK_F_GIVEN_CHALLENGES
     stream = torch.cuda.Stream()
     tables = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
     bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
     prover = bzk.Prover(local)
     out = bzk.Prover.alloc_outputs(B, k, d)
+    if flags & bzk.BZK_F_GIVEN_CHALLENGES:
+        # pre-seeded challenges (the paper's PRG output): any canonical values < 2^253
+        g = torch.empty((B, 1, k, 4), dtype=torch.int64, device="cuda")
+        bzk.bzk_generate(g, B, 1, k, first, "uniform", data_seed=0x5052470000000000, stream=stream)
+        out["challenges"].copy_(g.view(B, k, 4))
+        stream.synchronize()
     batch = prover.batch(tables, k, d, order, None, first, flags, out)
 
     batch_g = prover.batch(tables, k, d, order, None, first, flags | bzk.BZK_F_GRAPH, out)

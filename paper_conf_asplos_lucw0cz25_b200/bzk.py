@@ -23,7 +23,7 @@ LIB_PATH = os.environ.get("BZK_LIB", os.path.join(HERE, "libbzk.so"))
 BZK_OK, BZK_EINVAL, BZK_ENOMEM, BZK_ECUDA, BZK_ENONCANON, BZK_EUNSUPPORTED = range(6)
 BZK_ORDER_LSB, BZK_ORDER_MSB = 0, 1
 BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
-BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH = 1, 2, 4, 8
+BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
 BZK_PROF_KINDS = 6
 PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy"]
 

@@ -115,6 +115,7 @@ struct Plan {
     size_t stage_bytes;  // bytes of one staging slot (host tables), 0 otherwise
     uint32_t cmax;
     bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
+    uint32_t given;       // BZK_F_GIVEN_CHALLENGES
     size_t out_bytes_per_proof;
 };
 
@@ -164,6 +165,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.elem_table = (size_t)P.D * P.N * 32;
     P.host_tables = b->tables_mem == BZK_MEM_HOST;
     P.host_outputs = b->outputs_mem == BZK_MEM_HOST;
+    P.given = (b->flags & BZK_F_GIVEN_CHALLENGES) ? 1u : 0u;
     if (P.k == 0) { P.i0 = 1; P.log_h0 = 0; }
     else if (P.k - 1 <= kTailLog) { P.i0 = 1; P.log_h0 = P.k - 1; }
     else { P.i0 = P.k - kTailLog; P.log_h0 = kTailLog; }
@@ -324,6 +326,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.round_evals = io.round_evals; rp.challenges = io.challenges; rp.claims = io.claims;
         rp.consts = ctx->consts;
         rp.prefetch = knobs().prefetch;
+        rp.given = P.given;
         if (i == 1) { rp.src = io.tables; rp.dst = nullptr; }
         else {
             rp.src = (i == 2) ? io.tables : ((i - 1) % 2 == 0 ? bufX : bufY);
@@ -342,6 +345,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         tp.round_evals = io.round_evals; tp.challenges = io.challenges;
         tp.final_evals = io.final_evals; tp.claims = io.claims;
         tp.consts = ctx->consts;
+        tp.given = P.given;
         if (P.i0 <= 2) tp.src = io.tables;
         else tp.src = ((P.i0 - 1) % 2 == 0) ? bufX : bufY;
         size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 32;
@@ -369,6 +373,8 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     if (P.host_outputs) {
         fe *base = (fe *)(ws + P.off_out);
         o_ev = base; o_ch = o_ev + P.B * ev_pp; o_fi = o_ch + P.B * ch_pp; o_cl = o_fi + P.B * fi_pp;
+        if (P.given && P.k)
+            CK(cudaMemcpyAsync(o_ch, b->challenges, P.B * ch_pp * 32, cudaMemcpyHostToDevice, s));
     } else {
         o_ev = (fe *)b->round_evals; o_ch = (fe *)b->challenges; o_fi = (fe *)b->final_evals;
         o_cl = (fe *)b->claims;
@@ -415,7 +421,7 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     if (P.host_outputs) {
         if (P.k) {
             CK(cudaMemcpyAsync(b->round_evals, o_ev, P.B * ev_pp * 32, cudaMemcpyDeviceToHost, s));
-            CK(cudaMemcpyAsync(b->challenges, o_ch, P.B * ch_pp * 32, cudaMemcpyDeviceToHost, s));
+            if (!P.given) CK(cudaMemcpyAsync(b->challenges, o_ch, P.B * ch_pp * 32, cudaMemcpyDeviceToHost, s));
         }
         CK(cudaMemcpyAsync(b->final_evals, o_fi, P.B * fi_pp * 32, cudaMemcpyDeviceToHost, s));
         if (b->claims) CK(cudaMemcpyAsync(b->claims, o_cl, P.B * 32, cudaMemcpyDeviceToHost, s));

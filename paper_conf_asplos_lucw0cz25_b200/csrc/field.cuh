@@ -231,6 +231,40 @@ __device__ __forceinline__ void row_b(uint32_t A[9], uint32_t B[9], uint32_t L, 
         : "r"(L), "r"(a[1]), "r"(a[3]), "r"(a[5]), "r"(a[7]), "r"(bi));
 }
 
+// Same as row_b when B7 == B8 == 0 on entry (the first B chain of a row after the shift): the top
+// product is written, not accumulated, and no zero needs to be materialised (no IMAD.MOV).
+__device__ __forceinline__ void row_b_z(uint32_t A[9], uint32_t B[9], uint32_t L, const uint32_t a[8], uint32_t bi) {
+    asm("add.cc.u32     %0, %0, %10;\n\t"
+        "madc.lo.cc.u32 %1, %11, %15, %1;\n\t"
+        "madc.hi.cc.u32 %2, %11, %15, %2;\n\t"
+        "madc.lo.cc.u32 %3, %12, %15, %3;\n\t"
+        "madc.hi.cc.u32 %4, %12, %15, %4;\n\t"
+        "madc.lo.cc.u32 %5, %13, %15, %5;\n\t"
+        "madc.hi.cc.u32 %6, %13, %15, %6;\n\t"
+        "madc.lo.cc.u32 %7, %14, %15, %7;\n\t"
+        "madc.hi.cc.u32 %8, %14, %15, 0;\n\t"
+        "addc.u32       %9, 0, 0;"
+        : "+r"(A[0]), "+r"(B[0]), "+r"(B[1]), "+r"(B[2]), "+r"(B[3]), "+r"(B[4]), "+r"(B[5]), "+r"(B[6]),
+          "=r"(B[7]), "=r"(B[8])
+        : "r"(L), "r"(a[1]), "r"(a[3]), "r"(a[5]), "r"(a[7]), "r"(bi));
+}
+
+// B chain without a pending word: B[0..7] += a_odd * bi, carry into B8 (second product of a row)
+__device__ __forceinline__ void row_b_nl(uint32_t B[9], const uint32_t a[8], uint32_t bi) {
+    asm("mad.lo.cc.u32  %0, %9,  %13, %0;\n\t"
+        "madc.hi.cc.u32 %1, %9,  %13, %1;\n\t"
+        "madc.lo.cc.u32 %2, %10, %13, %2;\n\t"
+        "madc.hi.cc.u32 %3, %10, %13, %3;\n\t"
+        "madc.lo.cc.u32 %4, %11, %13, %4;\n\t"
+        "madc.hi.cc.u32 %5, %11, %13, %5;\n\t"
+        "madc.lo.cc.u32 %6, %12, %13, %6;\n\t"
+        "madc.hi.cc.u32 %7, %12, %13, %7;\n\t"
+        "addc.u32       %8, %8, 0;"
+        : "+r"(B[0]), "+r"(B[1]), "+r"(B[2]), "+r"(B[3]), "+r"(B[4]), "+r"(B[5]), "+r"(B[6]), "+r"(B[7]),
+          "+r"(B[8])
+        : "r"(a[1]), "r"(a[3]), "r"(a[5]), "r"(a[7]), "r"(bi));
+}
+
 // A chain of a row: A[0..7] += a_even * bi, carry into A8
 __device__ __forceinline__ void row_a(uint32_t A[9], const uint32_t a[8], uint32_t bi) {
     asm("mad.lo.cc.u32  %0, %9,  %13, %0;\n\t"
@@ -347,7 +381,7 @@ __device__ __forceinline__ fe mont_mul_lz(const fe &a, const fe &b) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
         if (i > 0) {
-            row_b(A, B, L, a.l, b.l[i]);
+            row_b_z(A, B, L, a.l, b.l[i]);
             row_a(A, a.l, b.l[i]);
         }
         uint32_t m = mont_m(A[0]);
@@ -415,13 +449,13 @@ __device__ __forceinline__ fe mont_mul2_lz(const fe &x, const fe &y, const fe &u
           "=r"(B[8])
         : "r"(x.l[1]), "r"(x.l[3]), "r"(x.l[5]), "r"(x.l[7]), "r"(y.l[0]));
     row_a(A, u.l, v.l[0]);
-    row_b(A, B, 0u, u.l, v.l[0]);
+    row_b_nl(B, u.l, v.l[0]);
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
         if (i > 0) {
-            row_b(A, B, L, x.l, y.l[i]);
+            row_b_z(A, B, L, x.l, y.l[i]);
             row_a(A, x.l, y.l[i]);
-            row_b(A, B, 0u, u.l, v.l[i]);
+            row_b_nl(B, u.l, v.l[i]);
             row_a(A, u.l, v.l[i]);
         }
         uint32_t m = mont_m(A[0]);

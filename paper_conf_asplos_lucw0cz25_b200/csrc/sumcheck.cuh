@@ -61,6 +61,7 @@ struct RoundParams {
     fe *claims;           // [Bw] (may be null)
     const fe *consts;     // kNumConsts
     uint32_t prefetch;    // 1: bulk-prefetch the next iteration's tiles into L2
+    uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
 };
 
 // ---------------------------------------------------------------- reductions
@@ -245,7 +246,7 @@ __device__ __forceinline__ fe extrapolate_top(const fe (&g)[D + 1], const fe &ci
 template <int D, int MODE>
 __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], uint32_t round, ProofState &ps,
                                                fe *round_evals, fe *challenges, fe *claims, const fe *consts,
-                                               fe *rmont_out) {
+                                               fe *rmont_out, bool given) {
     constexpr int NS = MODE == 2 ? D : D + 1;
     fe g[D + 1];
     const fe RD = fe_R_pow(D);
@@ -265,15 +266,21 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
         if (DERIVE) g[1] = fe_sub(ps.claim, g[0]);
         if (D >= 2) g[D] = extrapolate_top<D>(g, fixd[NS - 1]);
     }
-    uint32_t st[8];
+    fe r;
+    if (given) {
+        // paper-literal mode (Alg. 1: r_1..r_n are inputs): the challenge is read, not hashed
+        r = ld_fe(&challenges[round - 1]);
+    } else {
+        uint32_t st[8];
 #pragma unroll
-    for (int i = 0; i < 8; ++i) st[i] = ps.st[i];
-    fe r = transcript_round(st, g, D);
+        for (int i = 0; i < 8; ++i) st[i] = ps.st[i];
+        r = transcript_round(st, g, D);
 #pragma unroll
-    for (int i = 0; i < 8; ++i) ps.st[i] = st[i];
+        for (int i = 0; i < 8; ++i) ps.st[i] = st[i];
+        st_fe(&challenges[round - 1], r);
+    }
 #pragma unroll
     for (int t = 0; t <= D; ++t) st_fe(&round_evals[(size_t)(round - 1) * (D + 1) + t], g[t]);
-    st_fe(&challenges[round - 1], r);
     if (round == 1 && claims) st_fe(claims, fe_add(g[0], g[1]));
     fe rm = mont_mul(r, fe_const(2));
     ps.rmont = rm;
@@ -582,7 +589,7 @@ __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(Rou
     fe *claim = P.claims ? P.claims + b : nullptr;
     if (P.ctas == 1) {
         if (threadIdx.x == 0)
-            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
+            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr, P.given);
         return;
     }
     fe *part = P.partials + (size_t)b * P.ctas * NV;
@@ -605,7 +612,7 @@ __global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(Rou
     block_reduce<NV>(acc, s_red);
     if (threadIdx.x == 0) {
         P.tickets[b] = 0;
-        finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr);
+        finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr, P.given);
     }
 }
 
@@ -619,6 +626,7 @@ struct TailParams {
     ProofState *ps;
     fe *round_evals, *challenges, *final_evals, *claims;
     const fe *consts;
+    uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
 };
 
 template <int D, int ORDER>
@@ -687,7 +695,7 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
         block_reduce<D + 1>(acc, s_red);
         if (threadIdx.x == 0) {
             fe rm;
-            finalize_round<D, 0>(acc, i, P.ps[b], evals, chals, claim, P.consts, &rm);
+            finalize_round<D, 0>(acc, i, P.ps[b], evals, chals, claim, P.consts, &rm, P.given);
             s_r = rm;
         }
         __syncthreads();

@@ -280,3 +280,28 @@ def test_cuda_graph_replay_and_recapture(prover):
     for key in ref2:
         assert torch.equal(out[key], ref2[key]), key
     assert not torch.equal(ref2["challenges"], ref["challenges"])
+
+
+@pytest.mark.parametrize("order", [0, 1])
+@pytest.mark.parametrize("d,k", [(1, 12), (2, 13), (3, 10), (1, 16), (2, 4)])
+def test_given_challenges_paper_literal(prover, orc, d, k, order):
+    """BZK_F_GIVEN_CHALLENGES (Alg. 1, P:111: r_i are inputs) vs the oracle's given-challenge mode;
+    d = 1, MSB is Algorithm 1 literally."""
+    B = 3
+    t = dev_tables(B, d, k, 30)
+    rng = np.random.default_rng(k)
+    P = orc.P
+    r_int = [[int(x) * 0x9E3779B97F4A7C15 % P for x in rng.integers(1, 2**62, size=k)] for _ in range(B)]
+    r = np.stack([orc.to_limbs(rr) for rr in r_int])
+    out = bzk.Prover.alloc_outputs(B, k, d)
+    out["challenges"].copy_(torch.from_numpy(r.view(np.int64)))
+    b = prover.batch(t, k, d, order, None, 30, bzk.BZK_F_PRESERVE_INPUT | bzk.BZK_F_GIVEN_CHALLENGES, out)
+    bzk.bzk_prove(prover.ctx, b)
+    torch.cuda.synchronize()
+    host = np64(t)
+    for i in range(B):
+        ref = orc.prove_given(host[i], k, d, order, r[i])
+        for key in KEYS:
+            assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), (key, i)
+        if d == 1 and order == 1:
+            assert np.array_equal(orc.alg1(host[i][0], r[i]), np64(out["round_evals"][i]).reshape(k, 2, 4))
