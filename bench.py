@@ -85,6 +85,16 @@ def alg_mulmods(d: int, k: int, kind: str) -> int:
     raise ValueError(kind)
 
 
+def alg_bytes_kind(d: int, k: int, kind: str) -> int:
+    """Algorithmic HBM bytes per proof of a kernel kind: round 1 reads d 2^k x 32 B; a fused round
+    i reads 4 d h_i x 32 B and writes 2 d h_i x 32 B (ping-pong)."""
+    tail_log = 8
+    i0 = 1 if k - 1 <= tail_log else k - tail_log
+    if kind == "round1":
+        return d * (1 << k) * 32
+    return sum(6 * d * (1 << (k - i)) * 32 for i in range(2, i0))
+
+
 class ClockSampler:
     """nvidia-smi clocks + throttle reasons during the timed region (B200_PROFILING.md recipe)."""
 
@@ -295,6 +305,10 @@ def main():
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    # BZK_BENCH_DEVICE pins every rank to one GPU and BZK_DIST_BACKEND=gloo swaps the collective
+    # backend: together they smoke-test the multi-rank path on a single-GPU box
+    if os.environ.get("BZK_BENCH_DEVICE") is not None:
+        local = int(os.environ["BZK_BENCH_DEVICE"])
 
     if args.impl == "reference":
         run_reference(args, rank, world)
@@ -311,7 +325,11 @@ def main():
     dist = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
 
     B, d, k, order, gen_dist, desc = CONFIGS[args.config]
     if args.batch:
@@ -328,9 +346,10 @@ def main():
     out = bzk.Prover.alloc_outputs(B, k, d)
     if flags & bzk.BZK_F_GIVEN_CHALLENGES:
         # pre-seeded challenges (the paper's PRG output): any canonical values < 2^253
-        g = torch.empty((B, 1, k, 4), dtype=torch.int64, device="cuda")
-        bzk.bzk_generate(g, B, 1, k, first, "uniform", data_seed=0x5052470000000000, stream=stream)
-        out["challenges"].copy_(g.view(B, k, 4))
+        kk = max(1, (k - 1).bit_length())          # generator tables have 2^kk >= k entries
+        g = torch.empty((B, 1, 1 << kk, 4), dtype=torch.int64, device="cuda")
+        bzk.bzk_generate(g, B, 1, kk, first, "uniform", data_seed=0x5052470000000000, stream=stream)
+        out["challenges"].copy_(g[:, 0, :k, :])
         stream.synchronize()
     batch = prover.batch(tables, k, d, order, None, first, flags, out)
 
@@ -401,8 +420,18 @@ def main():
     step_gmulmod = total_alg / (ms_per_step / 1000.0) / 1e9
     # HBM: algorithmic bytes (read each input once) and the streaming schedule's bytes
     alg_bytes = d * (1 << k) * 32 * B
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        # DRAM bytes per launch of the dominant kernel from one `ncu --set full` capture of the same
+        # command (scripts/ncu_traffic.sh), if it was taken on this workload
+        with open(tpath) as f:
+            tj = json.load(f)
+        if tj.get("config") == args.config and tj.get("kernel_kind") == dom and tj.get("batch") == B:
+            traffic = tj["dram_bytes_per_launch"]
     roofline = {"bound": "alu", "kernel": dom, "achieved": round(achieved, 2), "peak": round(int_peak, 2),
-                "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": None,
+                "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": traffic,
+                "alg_bytes_per_launch": alg_bytes_kind(d, k, kinds[dom]) * B / max(1, dom_cnt / args.steps),
                 "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} MHz "
                                f"({peak_src} max clock) / {IMAD_PER_MULMOD} IMAD per mulmod",
                 "step_frac": round(step_gmulmod / int_peak, 4),
@@ -436,7 +465,9 @@ def main():
         del tmp
         torch.cuda.empty_cache()
         out_h = bzk.Prover.alloc_outputs(B, k, d, device="cpu", pin=True)
-        hb = prover.batch(host_t, k, d, order, None, first, 0, out_h)
+        if flags & bzk.BZK_F_GIVEN_CHALLENGES:
+            out_h["challenges"].copy_(out["challenges"])
+        hb = prover.batch(host_t, k, d, order, None, first, flags & bzk.BZK_F_GIVEN_CHALLENGES, out_h)
         bzk.bzk_prove(prover.ctx, hb, stream)   # warm-up (allocates staging)
         barrier()
         t0 = time.perf_counter()

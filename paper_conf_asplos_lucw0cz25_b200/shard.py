@@ -31,12 +31,17 @@ def output_digest(arrays) -> str:
     return h.hexdigest()
 
 
+def _dev(dist, device):
+    """NCCL needs CUDA tensors; gloo (CPU tests, single-GPU smoke runs) takes CPU tensors."""
+    return device if dist.get_backend() == "nccl" else None
+
+
 def max_over_ranks(value: float, dist, device=None) -> float:
     """Max of a per-rank scalar (the device time of the timed region)."""
     import torch
     if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
         return float(value)
-    t = torch.tensor([float(value)], dtype=torch.float64, device=device)
+    t = torch.tensor([float(value)], dtype=torch.float64, device=_dev(dist, device))
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -46,7 +51,7 @@ def gather_bytes(blob: bytes, dist, device=None) -> list[bytes]:
     import torch
     if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
         return [blob]
-    t = torch.tensor(list(blob), dtype=torch.uint8, device=device)
+    t = torch.tensor(list(blob), dtype=torch.uint8, device=_dev(dist, device))
     out = [torch.zeros_like(t) for _ in range(dist.get_world_size())]
     dist.all_gather(out, t)
     return [bytes(x.cpu().tolist()) for x in out]
