@@ -14,6 +14,7 @@
 
 #include "bzk.h"
 #include "field.cuh"
+#include "field_f64.cuh"
 #include "gen.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
@@ -512,6 +513,8 @@ __global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *
             case 1: r = fe_sub(x, ld_fe(b + i)); break;
             case 2: r = mont_mul(x, ld_fe(b + i)); break;
             case 3: r = mont_mul(mont_mul(x, ld_fe(b + i)), fe_const(2)); break;
+            case 5: { f6 fx = to_f6(x), fy = to_f6(ld_fe(b + i)); r = fmont<1>(fx, fy, fx, fy); break; }
+            case 6: { f6 fx = to_f6(x), fy = to_f6(ld_fe(b + i)); r = fmont<2>(fx, fy, fy, fx); break; }
             default: r = fe_reduce_256(x); break;
         }
         st_fe(out + i, r);
@@ -541,7 +544,7 @@ __global__ void k_debug_sha256(const uint8_t *msgs, uint32_t len, uint64_t n, ui
 //   kind 0: mad.lo.u32 (IMAD)      kind 1: mul.wide.u32 (IMAD.WIDE.U32)
 //   kind 2: mont_mul_v1            kind 3: mont_mul (hot path)
 template <int KIND>
-__global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, uint32_t *sink) {
+__global__ void __launch_bounds__(256, 2) k_bench(uint32_t iters, uint32_t seed, uint32_t *sink) {
     const uint32_t tid = blockIdx.x * blockDim.x + threadIdx.x;
     if (KIND == 4) {   // DFMA throughput (FP64 pipe)
         double a[8];
@@ -580,7 +583,7 @@ __global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, ui
         for (int i = 0; i < 8; ++i) acc ^= a[i] ^ (uint32_t)w[i] ^ (uint32_t)(w[i] >> 32);
         sink[tid] = acc;
     } else {
-        constexpr int CH = KIND == 5 ? 1 : (KIND == 6 ? 2 : 4);
+        constexpr int CH = KIND == 5 ? 1 : (KIND == 6 ? 2 : (KIND >= 9 ? 2 : 4));
         fe x[4], y;
 #pragma unroll
         for (int c = 0; c < 4; ++c)
@@ -591,7 +594,13 @@ __global__ void __launch_bounds__(256) k_bench(uint32_t iters, uint32_t seed, ui
         for (uint32_t it = 0; it < iters; ++it)
 #pragma unroll
             for (int c = 0; c < CH; ++c) {
-                if (KIND == 2) x[c] = mont_mul_v1(x[c], y);
+                // 9: FP64 only; 10: odd warps FP64, even warps IMAD; 11: each thread alternates
+                const bool fp = KIND == 9 || (KIND == 10 && ((threadIdx.x >> 5) & 1)) || (KIND == 11 && (c & 1));
+                if (KIND >= 9 && fp) {
+                    const f6 a = to_f6(x[c]), b = to_f6(y), u = to_f6(x[(c + 1) & 3]);
+                    x[c] = fmont<2>(a, b, u, b);
+                } else if (KIND >= 9) x[c] = mont_mul2(x[c], y, x[(c + 1) & 3], y);
+                else if (KIND == 2) x[c] = mont_mul_v1(x[c], y);
                 else if (KIND == 8) x[c] = mont_mul2(x[c], y, x[(c + 1) & 3], y);
                 else x[c] = mont_mul(x[c], y);
             }
@@ -631,7 +640,7 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
     cudaFree(sink);
-    const double per = (KIND <= 1 || KIND == 4) ? 32.0 : (KIND == 5 ? 1.0 : (KIND == 6 ? 2.0 : 4.0));
+    const double per = (KIND <= 1 || KIND == 4) ? 32.0 : (KIND == 5 ? 1.0 : ((KIND == 6 || KIND >= 9) ? 2.0 : 4.0));
     const double ops = (double)blocks * threads * iters * per;   // kind 8 counts mont_mul2 calls
     *rate = ops / (ms * 1e-3) / ((double)clk_khz * 1e3) / nsm;   // per SM per clock (at the max clock)
     return e;
@@ -788,7 +797,7 @@ uint64_t bzk_launch_count(bzk_ctx *ctx, int reset) {
 
 bzk_status bzk_debug_field(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out,
                            void *cuda_stream) {
-    if (op < 0 || op > 4 || !a || !out || (op < 4 && !b)) return BZK_EINVAL;
+    if (op < 0 || op > 6 || !a || !out || (op != 4 && !b)) return BZK_EINVAL;
     if (n == 0) return BZK_OK;
     k_debug_field<<<kSMs * 8, 256, 0, (cudaStream_t)cuda_stream>>>(op, n, (const fe *)a, (const fe *)b, (fe *)out);
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
@@ -802,7 +811,7 @@ bzk_status bzk_debug_sha256(const uint8_t *msgs, uint32_t msg_len, uint64_t n, u
 }
 
 bzk_status bzk_debug_bench(int kind, uint32_t iters, double *rate, void *cuda_stream) {
-    if (!rate || iters == 0 || kind < 0 || kind > 8) return BZK_EINVAL;
+    if (!rate || iters == 0 || kind < 0 || kind > 11) return BZK_EINVAL;
     cudaStream_t s = (cudaStream_t)cuda_stream;
     cudaError_t e = cudaErrorInvalidValue;
     switch (kind) {
@@ -815,6 +824,9 @@ bzk_status bzk_debug_bench(int kind, uint32_t iters, double *rate, void *cuda_st
         case 6: e = run_bench<6>(iters, rate, s); break;
         case 7: e = run_bench<7>(iters, rate, s); break;
         case 8: e = run_bench<8>(iters, rate, s); break;
+        case 9: e = run_bench<9>(iters, rate, s); break;
+        case 10: e = run_bench<10>(iters, rate, s); break;
+        case 11: e = run_bench<11>(iters, rate, s); break;
     }
     return e == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }

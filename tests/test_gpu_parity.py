@@ -305,3 +305,22 @@ def test_given_challenges_paper_literal(prover, orc, d, k, order):
             assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), (key, i)
         if d == 1 and order == 1:
             assert np.array_equal(orc.alg1(host[i][0], r[i]), np64(out["round_evals"][i]).reshape(k, 2, 4))
+
+
+def test_fp64_pipe_montgomery_vs_oracle(orc):
+    """field_f64.cuh: radix-2^48 FP64 Montgomery products (R' = 2^288) on random and edge inputs up
+    to 2^256 - 1 (the lazy representation)."""
+    rng = np.random.default_rng(17)
+    P = orc.P
+    n = 1 << 15
+    edge = [0, 1, P - 1, P, 2 * P - 1, 2**256 - 1, 2**255, 2**48 - 1, 2**48, 2**253]
+    av = [int.from_bytes(rng.bytes(32), "little") for _ in range(n)] + [e for e in edge for _ in edge]
+    bv = [int.from_bytes(rng.bytes(32), "little") for _ in range(n)] + edge * len(edge)
+    A = torch.from_numpy(orc.to_limbs(av).view(np.int64)).cuda()
+    Bt = torch.from_numpy(orc.to_limbs(bv).view(np.int64)).cuda()
+    out = torch.empty_like(A)
+    inv = pow(2**288, P - 2, P)
+    for op, f in [(5, 1), (6, 2)]:
+        bzk.bzk_debug_field(op, A.shape[0], A, Bt, out)
+        torch.cuda.synchronize()
+        assert orc.from_limbs(np64(out)) == [f * x * y * inv % P for x, y in zip(av, bv)], op
