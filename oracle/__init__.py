@@ -50,6 +50,8 @@ def lib():
         L.orc_fr_op.argtypes = [ctypes.c_int, u64, u64p, u64p, u64p]
         L.orc_sha256.argtypes = [u8p, u64, ctypes.c_char_p]
         L.orc_mu.argtypes = [u64p]
+        L.orc_gl_prove.argtypes = [u32, u32, u32, u8p, u64, u64p, u64p, u64p, u64p, u64p, u64p]
+        L.orc_gl_op.argtypes = [ctypes.c_int, u64, u64p, u64p, u64p]
         _lib = L
     return _lib
 
@@ -179,3 +181,32 @@ def mu() -> int:
     out = np.zeros(5, np.uint64)
     lib().orc_mu(_p(out))
     return sum(int(out[i]) << (64 * i) for i in range(5))
+
+
+# ---------------------------------------------------------------- Goldilocks (NEXT-2, reading R15)
+
+PGL = 0xFFFFFFFF00000001
+
+
+def gl_prove(tables: np.ndarray, k: int, d: int, order: int, seed: bytes, index: int, given=None):
+    """One Goldilocks proof.  tables: uint64 [d][2^k].  given: optional challenges [k] (Alg. 1 mode)."""
+    tables = np.ascontiguousarray(tables, dtype=np.uint64)
+    assert tables.shape == (d, 1 << k)
+    ev = np.zeros((k, d + 1), np.uint64)
+    ch = np.zeros((k,), np.uint64)
+    fi = np.zeros((d,), np.uint64)
+    cl = np.zeros((1,), np.uint64)
+    g = None if given is None else np.ascontiguousarray(given, dtype=np.uint64)
+    s = lib().orc_gl_prove(k, d, order, seed, index, _p(tables), _p(g), _p(ev), _p(ch), _p(fi), _p(cl))
+    if s:
+        raise ValueError(f"orc_gl_prove failed: {s}")
+    return {"round_evals": ev, "challenges": ch, "final_evals": fi, "claims": cl}
+
+
+def gl_op(op: str, a: np.ndarray, b: np.ndarray) -> np.ndarray:
+    code = {"add": 0, "sub": 1, "mul": 2}[op]
+    a = np.ascontiguousarray(a, dtype=np.uint64)
+    b = np.ascontiguousarray(b, dtype=np.uint64)
+    out = np.zeros_like(a)
+    lib().orc_gl_op(code, a.shape[0], _p(a), _p(b), _p(out))
+    return out

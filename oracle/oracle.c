@@ -596,3 +596,120 @@ int orc_fr_op(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t
 
 /* expose mu for the pin test (mu = floor(2^512/p)) */
 void orc_mu(uint64_t out[5]) { ensure_mu(); memcpy(out, MU, sizeof MU); }
+
+/* ================================================================== */
+/* Second field instance (reading R15): Goldilocks  */
+/* p_gl = 2^64 - 2^32 + 1, elements one u64, canonical.  Same prover,   */
+/* transcript framed with field id 1 (the reserved LE16 of state_0) and */
+/* LE64-encoded evaluations; r_i = LE64(state_i[0..8]) mod p_gl.        */
+/* Arithmetic is the plain definition: unsigned __int128 then % p.      */
+/* ================================================================== */
+
+static const uint64_t PGL = 0xffffffff00000001ULL;
+
+static uint64_t gl_add(uint64_t a, uint64_t b) { return (uint64_t)(((u128)a + b) % PGL); }
+static uint64_t gl_sub(uint64_t a, uint64_t b) { return (uint64_t)(((u128)a + PGL - b) % PGL); }
+static uint64_t gl_mul(uint64_t a, uint64_t b) { return (uint64_t)(((u128)a * b) % PGL); }
+
+static void gl_transcript_init(uint8_t state[32], const uint8_t seed[32], uint64_t I, uint32_t k, uint32_t d,
+                               uint32_t order) {
+    uint8_t m[64];
+    memcpy(m, "BZK-SUMCHECK-V1", 15); m[15] = 0;
+    memcpy(m + 16, seed, 32);
+    for (int i = 0; i < 8; ++i) m[48 + i] = (uint8_t)(I >> (8 * i));
+    m[56] = (uint8_t)k; m[57] = (uint8_t)(k >> 8);
+    m[58] = (uint8_t)d; m[59] = (uint8_t)(d >> 8);
+    m[60] = (uint8_t)order; m[61] = (uint8_t)(order >> 8);
+    m[62] = 1; m[63] = 0;                                  /* field id 1 = Goldilocks */
+    orc_sha256(m, 64, state);
+}
+
+static uint64_t gl_transcript_round(uint8_t state[32], const uint64_t *g, uint32_t d) {
+    sha256_ctx c; sha256_init(&c);
+    sha256_update(&c, state, 32);
+    for (uint32_t t = 0; t <= d; ++t) {
+        uint8_t b[8];
+        for (int j = 0; j < 8; ++j) b[j] = (uint8_t)(g[t] >> (8 * j));
+        sha256_update(&c, b, 8);
+    }
+    sha256_final(&c, state);
+    uint64_t v = 0;
+    for (int j = 0; j < 8; ++j) v |= (uint64_t)state[j] << (8 * j);
+    return v % PGL;
+}
+
+/* One Goldilocks proof: tables [d][2^k] u64; round_evals [k][d+1]; challenges [k]; final [d];
+ * claim [1].  given_r (may be NULL): paper-literal mode, challenges are inputs. */
+int orc_gl_prove(uint32_t k, uint32_t d, uint32_t order, const uint8_t seed[32], uint64_t I,
+                 const uint64_t *tables, const uint64_t *given_r, uint64_t *round_evals, uint64_t *challenges,
+                 uint64_t *final_evals, uint64_t *claim) {
+    if (k > 30 || d < 1 || d > 4 || order > 1) return ORC_EINVAL;
+    const uint64_t N = (uint64_t)1 << k;
+    uint64_t *T = (uint64_t *)malloc(sizeof(uint64_t) * N * d);
+    if (!T) return ORC_ENOMEM;
+    for (uint64_t x = 0; x < N * d; ++x) {
+        if (tables[x] >= PGL) { free(T); return ORC_ENONCANON; }
+        T[x] = tables[x];
+    }
+    uint64_t H = 0;
+    for (uint64_t x = 0; x < N; ++x) {
+        uint64_t prod = T[x];
+        for (uint32_t m = 1; m < d; ++m) prod = gl_mul(prod, T[m * N + x]);
+        H = gl_add(H, prod);
+    }
+    uint8_t state[32];
+    gl_transcript_init(state, seed, I, k, d, order);
+    uint64_t size = N, g[5];
+    for (uint32_t i = 1; i <= k; ++i) {
+        uint64_t h = size / 2;
+        for (uint32_t t = 0; t <= d; ++t) {
+            uint64_t acc = 0;
+            for (uint64_t j = 0; j < h; ++j) {
+                uint64_t prod = 1;
+                for (uint32_t m = 0; m < d; ++m) {
+                    const uint64_t *Tm = T + (uint64_t)m * N;
+                    uint64_t a = order == 0 ? Tm[2 * j] : Tm[j];
+                    uint64_t b = order == 0 ? Tm[2 * j + 1] : Tm[j + h];
+                    prod = gl_mul(prod, gl_add(a, gl_mul(t, gl_sub(b, a))));
+                }
+                acc = gl_add(acc, prod);
+            }
+            g[t] = acc;
+        }
+        uint64_t r;
+        if (given_r) {
+            r = given_r[i - 1];
+            if (r >= PGL) { free(T); return ORC_ENONCANON; }
+        } else {
+            r = gl_transcript_round(state, g, d);
+        }
+        for (uint32_t t = 0; t <= d; ++t) round_evals[(uint64_t)(i - 1) * (d + 1) + t] = g[t];
+        challenges[i - 1] = r;
+        for (uint32_t m = 0; m < d; ++m) {
+            uint64_t *Tm = T + (uint64_t)m * N;
+            for (uint64_t j = 0; j < h; ++j) {
+                uint64_t a = order == 0 ? Tm[2 * j] : Tm[j];
+                uint64_t b = order == 0 ? Tm[2 * j + 1] : Tm[j + h];
+                Tm[j] = gl_add(a, gl_mul(r, gl_sub(b, a)));
+            }
+        }
+        size = h;
+    }
+    for (uint32_t m = 0; m < d; ++m) final_evals[m] = T[(uint64_t)m * N];
+    if (claim) claim[0] = H;
+    free(T);
+    return ORC_OK;
+}
+
+/* element-wise Goldilocks ops for pins: op 0 add, 1 sub, 2 mul */
+int orc_gl_op(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out) {
+    for (uint64_t i = 0; i < n; ++i) {
+        switch (op) {
+            case 0: out[i] = gl_add(a[i] % PGL, b[i] % PGL); break;
+            case 1: out[i] = gl_sub(a[i] % PGL, b[i] % PGL); break;
+            case 2: out[i] = gl_mul(a[i] % PGL, b[i] % PGL); break;
+            default: return ORC_EINVAL;
+        }
+    }
+    return ORC_OK;
+}

@@ -29,7 +29,9 @@ MASK61 = np.uint64((1 << 61) - 1)
 DIST_UNIFORM = 0
 DIST_SMALLINT = 1
 DIST_VML = 2
-DISTS = {"uniform": DIST_UNIFORM, "smallint": DIST_SMALLINT, "vml": DIST_VML}
+DIST_GL = 3          # Goldilocks (NEXT-2): ONE word per element, masked to 63 bits -> < 2^63 < p_gl
+DISTS = {"uniform": DIST_UNIFORM, "smallint": DIST_SMALLINT, "vml": DIST_VML, "gl": DIST_GL}
+MASK63 = np.uint64((1 << 63) - 1)
 
 
 def splitmix64(ctr: np.ndarray, data_seed: int = DATA_SEED) -> np.ndarray:
@@ -38,6 +40,19 @@ def splitmix64(ctr: np.ndarray, data_seed: int = DATA_SEED) -> np.ndarray:
         z = (z ^ (z >> np.uint64(30))) * M1
         z = (z ^ (z >> np.uint64(27))) * M2
         return z ^ (z >> np.uint64(31))
+
+
+def gen_tables_gl(batch: int, d: int, k: int, first_index: int = 0, data_seed: int = DATA_SEED) -> np.ndarray:
+    """Goldilocks tables, uint64 [B][d][2^k]: word(I, m, x, w=0) & (2^63 - 1)."""
+    N = 1 << k
+    out = np.empty((batch, d, N), dtype=np.uint64)
+    x = np.arange(N, dtype=np.uint64)
+    for bi in range(batch):
+        I = np.uint64(first_index + bi)
+        for m in range(d):
+            ctr = (I << np.uint64(36)) | (np.uint64(m) << np.uint64(32)) | (x << np.uint64(2))
+            out[bi, m] = splitmix64(ctr, data_seed) & MASK63
+    return out
 
 
 def gen_tables(batch: int, d: int, k: int, first_index: int = 0, dist: str | int = "uniform",

@@ -376,3 +376,69 @@ def test_given_challenge_mode(orc, d, order):
     assert prod == claim
     rho = py.rho_point(ints(r), k, order)
     assert ints(out["final_evals"])[0] == py.mle(ints(t[0]), rho)
+
+
+# ---------------------------------------------------------------- Goldilocks instance (NEXT-2)
+
+from oracle.py import goldilocks as pgl  # noqa: E402
+
+PGL = pgl.P
+
+
+def test_goldilocks_modulus():
+    assert PGL == 2**64 - 2**32 + 1
+    assert is_probable_prime(PGL)
+    assert (PGL - 1) % 2**32 == 0 and (PGL - 1) % 2**33 != 0     # 2-adicity 32
+    assert pow(7, (PGL - 1) // 2, PGL) == PGL - 1                 # 7 is a non-residue (generator family)
+
+
+def test_goldilocks_field_ops(orc):
+    rng = np.random.default_rng(3)
+    a = rng.integers(0, 2**63, size=5000, dtype=np.uint64) * np.uint64(2) + np.uint64(1)
+    b = rng.integers(0, 2**63, size=5000, dtype=np.uint64)
+    edge = np.array([0, 1, PGL - 1, 2**32, 2**32 - 1, 2**63, PGL - 2**32], dtype=np.uint64)
+    a = np.concatenate([a, np.repeat(edge, len(edge))])
+    b = np.concatenate([b, np.tile(edge, len(edge))])
+    A, B = [int(x) % PGL for x in a], [int(x) % PGL for x in b]
+    assert [int(x) for x in orc.gl_op("add", a, b)] == [(x + y) % PGL for x, y in zip(A, B)]
+    assert [int(x) for x in orc.gl_op("sub", a, b)] == [(x - y) % PGL for x, y in zip(A, B)]
+    assert [int(x) for x in orc.gl_op("mul", a, b)] == [(x * y) % PGL for x, y in zip(A, B)]
+
+
+@pytest.mark.parametrize("order", [0, 1])
+@pytest.mark.parametrize("d", [1, 2, 3])
+def test_goldilocks_oracle_pins(orc, d, order):
+    k = 5
+    t = inputs.gen_tables_gl(1, d, k, first_index=3)[0]
+    tabs = [[int(x) for x in t[m]] for m in range(d)]
+    out = orc.gl_prove(t, k, d, order, SEED, 3)
+    ev, ch, fi, H = pgl.prove(tabs, k, SEED, 3, order)
+    assert [[int(x) for x in row] for row in out["round_evals"]] == ev            # C == Python
+    assert [int(x) for x in out["challenges"]] == ch
+    assert [int(x) for x in out["final_evals"]] == fi and int(out["claims"][0]) == H
+    brute = 0
+    for x in range(1 << k):
+        prod = 1
+        for m in range(d):
+            prod = prod * tabs[m][x] % PGL
+        brute = (brute + prod) % PGL
+    assert H == brute and (ev[0][0] + ev[0][1]) % PGL == H
+    claim = H
+    for i in range(k):
+        assert (ev[i][0] + ev[i][1]) % PGL == claim
+        for X in (0, d + 1) if i < 3 else (0,):
+            direct = pgl.round_poly_direct(tabs, k, ch[:i], X, order)
+            assert direct == (ev[i][X] if X <= d else pgl.lagrange_eval(ev[i], X))
+        claim = pgl.lagrange_eval(ev[i], ch[i])
+    prod = 1
+    for f in fi:
+        prod = prod * f % PGL
+    assert prod == claim
+    z = [0] * k
+    for i, r in enumerate(ch, start=1):
+        z[i - 1 if order == 0 else k - i] = r
+    assert fi[0] == pgl.mle(tabs[0], z)
+    # paper-literal mode: fed the FS challenges it reproduces the proof
+    giv = orc.gl_prove(t, k, d, order, SEED, 3, given=out["challenges"])
+    for key in out:
+        assert np.array_equal(giv[key], out[key])
