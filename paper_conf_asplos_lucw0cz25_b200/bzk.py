@@ -24,6 +24,7 @@ BZK_OK, BZK_EINVAL, BZK_ENOMEM, BZK_ECUDA, BZK_ENONCANON, BZK_EUNSUPPORTED = ran
 BZK_ORDER_LSB, BZK_ORDER_MSB = 0, 1
 BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
 BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
+BZK_F_FIELD_GOLDILOCKS = 32
 BZK_PROF_KINDS = 6
 PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy"]
 
@@ -237,6 +238,16 @@ class Prover:
                 "final_evals": torch.empty((B, d, 4), **kw),
                 "claims": torch.empty((B, 4), **kw)}
 
+    @staticmethod
+    def alloc_outputs_gl(B, k, d, device="cuda", pin=False):
+        """Output tensors for BZK_F_FIELD_GOLDILOCKS (one 64-bit word per element)."""
+        import torch
+        kw = dict(dtype=torch.int64, device=device)
+        if device == "cpu" and pin:
+            kw["pin_memory"] = True
+        return {"round_evals": torch.empty((B, k, d + 1), **kw), "challenges": torch.empty((B, k), **kw),
+                "final_evals": torch.empty((B, d), **kw), "claims": torch.empty((B,), **kw)}
+
     def batch(self, tables, k, d, order=0, seed=None, first_index=0, flags=0, out=None, batch=None):
         from .inputs import DEFAULT_SEED
         seed = DEFAULT_SEED if seed is None else seed
@@ -255,8 +266,8 @@ class Prover:
         """tables: int64 tensor [B][d][2^k][4]. Returns the output dict (torch tensors)."""
         B = tables.shape[0]
         if out is None:
-            out = self.alloc_outputs(B, k, d, device="cuda" if tables.is_cuda else "cpu",
-                                     pin=not tables.is_cuda)
+            alloc = self.alloc_outputs_gl if flags & BZK_F_FIELD_GOLDILOCKS else self.alloc_outputs
+            out = alloc(B, k, d, device="cuda" if tables.is_cuda else "cpu", pin=not tables.is_cuda)
         b = self.batch(tables, k, d, order, seed, first_index, flags, out)
         bzk_prove(self.ctx, b, stream)
         return out

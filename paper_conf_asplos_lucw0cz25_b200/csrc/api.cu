@@ -15,6 +15,7 @@
 #include "bzk.h"
 #include "field.cuh"
 #include "field_f64.cuh"
+#include "gl.cuh"
 #include "gen.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
@@ -117,6 +118,8 @@ struct Plan {
     uint32_t cmax;
     bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
     uint32_t given;       // BZK_F_GIVEN_CHALLENGES
+    bool gl;              // BZK_F_FIELD_GOLDILOCKS (NEXT-2)
+    size_t esz;           // bytes per element: 32 (BN254) or 8 (Goldilocks)
     size_t out_bytes_per_proof;
 };
 
@@ -163,7 +166,9 @@ bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
 bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.k = b->num_vars; P.D = b->degree; P.order = b->order; P.B = b->batch;
     P.N = 1ull << P.k;
-    P.elem_table = (size_t)P.D * P.N * 32;
+    P.gl = (b->flags & BZK_F_FIELD_GOLDILOCKS) != 0;
+    P.esz = P.gl ? 8 : 32;
+    P.elem_table = (size_t)P.D * P.N * P.esz;
     P.host_tables = b->tables_mem == BZK_MEM_HOST;
     P.host_outputs = b->outputs_mem == BZK_MEM_HOST;
     P.given = (b->flags & BZK_F_GIVEN_CHALLENGES) ? 1u : 0u;
@@ -175,7 +180,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.need_bufY = P.i0 > 3;
     // consume mode (or host tables staged into our own buffers): round 3+ may overwrite the input
     P.bufY_alias_input = P.need_bufY && (P.host_tables || !preserve);
-    P.out_bytes_per_proof = (size_t)32 * ((size_t)P.k * (P.D + 1) + P.k + P.D + 1);
+    P.out_bytes_per_proof = P.esz * ((size_t)P.k * (P.D + 1) + P.k + P.D + 1);
 
     size_t limit = ctx->workspace_limit;
     if (limit == 0) {
@@ -190,11 +195,11 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     }
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
-        size_t s = sizeof(ProofState) + 4;
+        size_t s = std::max(sizeof(ProofState), sizeof(gl::State)) + 4;
         uint32_t c = P.k ? ctas_for(1ull << (P.k - 1), bw) : 1;
-        s += (size_t)c * (P.D + 1) * 32;
-        if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * 32;
-        if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * 32;
+        s += (size_t)c * (P.D + 1) * P.esz;
+        if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * P.esz;
+        if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * P.esz;
         if (P.host_tables) s += 2 * P.elem_table;
         return s;
     };
@@ -215,11 +220,11 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
 
     size_t off = 0;
     P.off_seed = off; off += 256;
-    P.off_ps = off; off = align_up(off + bw * sizeof(ProofState));
+    P.off_ps = off; off = align_up(off + bw * std::max(sizeof(ProofState), sizeof(gl::State)));
     P.off_tick = off; off = align_up(off + bw * 4);
-    P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * (P.D + 1) * 32);
-    P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * 32);
-    P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * 32);
+    P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * (P.D + 1) * P.esz);
+    P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * P.esz);
+    P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * P.esz);
     P.off_out = off; if (P.host_outputs) off = align_up(off + P.B * P.out_bytes_per_proof);
     P.total = off;
     P.stage_bytes = P.host_tables ? align_up(bw * P.elem_table) : 0;
@@ -284,6 +289,11 @@ cudaError_t dispatch_tail(uint32_t D, uint32_t order, uint32_t grid, size_t smem
     return cudaErrorInvalidValue;
 }
 
+__global__ void k_validate_gl(const uint64_t *t, uint64_t n, uint32_t *flag) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        if (t[i] >= gl::P) atomicOr(flag, 1u);
+}
+
 __global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
     for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
          i += (uint64_t)gridDim.x * blockDim.x) {
@@ -296,10 +306,61 @@ __global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
 
 struct WaveIO {
     Seed32 seed;       // transcript seed, passed to the kernel by value
-    fe *tables;        // device tables of this wave [nb][D][N]
-    fe *round_evals, *challenges, *final_evals, *claims;   // device outputs of this wave
+    char *tables;      // device tables of this wave [nb][D][N] x esz
+    char *round_evals, *challenges, *final_evals, *claims;   // device outputs of this wave
     uint64_t nb, first_index;
 };
+
+// Goldilocks wave (gl.cuh): same schedule as run_wave, 8-byte elements
+bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
+    char *ws = (char *)ctx->ws;
+    gl::State *ps = (gl::State *)(ws + P.off_ps);
+    uint32_t *tick = (uint32_t *)(ws + P.off_tick);
+    uint64_t *part = (uint64_t *)(ws + P.off_part);
+    uint64_t *tab = (uint64_t *)io.tables;
+    uint64_t *bufX = (uint64_t *)(ws + P.off_bufX);
+    uint64_t *bufY = P.bufY_alias_input ? tab : (uint64_t *)(ws + P.off_bufY);
+    const uint32_t D = P.D, k = P.k;
+    {
+        ProfScope ps_(ctx, s, 3);
+        cudaError_t e = gl_launch_init(ps, (uint32_t)io.nb, io.seed.b, io.first_index, k, D, P.order, s);
+        ++ctx->launches;
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "gl init launch");
+    }
+    for (uint32_t i = 1; i < P.i0; ++i) {
+        gl::RoundParams rp;
+        memset(&rp, 0, sizeof rp);
+        rp.log_h = k - i; rp.round = i; rp.k = k; rp.order = P.order; rp.given = P.given;
+        rp.ctas = ctas_for(1ull << rp.log_h, io.nb);
+        rp.partials = part; rp.tickets = tick; rp.ps = ps;
+        rp.round_evals = (uint64_t *)io.round_evals; rp.challenges = (uint64_t *)io.challenges;
+        rp.claims = (uint64_t *)io.claims;
+        if (i == 1) { rp.src = tab; rp.dst = nullptr; }
+        else {
+            rp.src = (i == 2) ? tab : ((i - 1) % 2 == 0 ? bufX : bufY);
+            rp.dst = (i % 2 == 0) ? bufX : bufY;
+        }
+        dim3 grid(rp.ctas, (uint32_t)io.nb);
+        ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
+        cudaError_t e = gl_launch_round(D, P.order, i == 1, grid, kThreads, s, rp);
+        ++ctx->launches;
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "k_gl_round launch");
+    }
+    {
+        gl::TailParams tp;
+        memset(&tp, 0, sizeof tp);
+        tp.i0 = P.i0; tp.log_h0 = P.log_h0; tp.k = k; tp.order = P.order; tp.ps = ps; tp.given = P.given;
+        tp.round_evals = (uint64_t *)io.round_evals; tp.challenges = (uint64_t *)io.challenges;
+        tp.final_evals = (uint64_t *)io.final_evals; tp.claims = (uint64_t *)io.claims;
+        tp.src = (P.i0 <= 2) ? tab : (((P.i0 - 1) % 2 == 0) ? bufX : bufY);
+        size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 8;
+        ProfScope ps_(ctx, s, 2);
+        cudaError_t e = gl_launch_tail(D, P.order, (uint32_t)io.nb, kThreads, smem, s, tp);
+        ++ctx->launches;
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "k_gl_tail launch");
+    }
+    return BZK_OK;
+}
 
 bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
     char *ws = (char *)ctx->ws;
@@ -307,7 +368,8 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
     uint32_t *tick = (uint32_t *)(ws + P.off_tick);
     fe *part = (fe *)(ws + P.off_part);
     fe *bufX = (fe *)(ws + P.off_bufX);
-    fe *bufY = P.bufY_alias_input ? io.tables : (fe *)(ws + P.off_bufY);
+    fe *tab = (fe *)io.tables;
+    fe *bufY = P.bufY_alias_input ? tab : (fe *)(ws + P.off_bufY);
     const uint32_t D = P.D, k = P.k;
     {
         ProfScope ps_(ctx, s, 3);
@@ -324,13 +386,13 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         const uint64_t h = 1ull << rp.log_h;
         rp.ctas = ctas_for(h, io.nb);
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
-        rp.round_evals = io.round_evals; rp.challenges = io.challenges; rp.claims = io.claims;
+        rp.round_evals = (fe *)io.round_evals; rp.challenges = (fe *)io.challenges; rp.claims = (fe *)io.claims;
         rp.consts = ctx->consts;
         rp.prefetch = knobs().prefetch;
         rp.given = P.given;
-        if (i == 1) { rp.src = io.tables; rp.dst = nullptr; }
+        if (i == 1) { rp.src = tab; rp.dst = nullptr; }
         else {
-            rp.src = (i == 2) ? io.tables : ((i - 1) % 2 == 0 ? bufX : bufY);
+            rp.src = (i == 2) ? tab : ((i - 1) % 2 == 0 ? bufX : bufY);
             rp.dst = (i % 2 == 0) ? bufX : bufY;
         }
         dim3 grid(rp.ctas, (uint32_t)io.nb);
@@ -343,11 +405,11 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         TailParams tp;
         memset(&tp, 0, sizeof tp);
         tp.i0 = P.i0; tp.log_h0 = P.log_h0; tp.k = k; tp.order = P.order; tp.ps = ps;
-        tp.round_evals = io.round_evals; tp.challenges = io.challenges;
-        tp.final_evals = io.final_evals; tp.claims = io.claims;
+        tp.round_evals = (fe *)io.round_evals; tp.challenges = (fe *)io.challenges;
+        tp.final_evals = (fe *)io.final_evals; tp.claims = (fe *)io.claims;
         tp.consts = ctx->consts;
         tp.given = P.given;
-        if (P.i0 <= 2) tp.src = io.tables;
+        if (P.i0 <= 2) tp.src = tab;
         else tp.src = ((P.i0 - 1) % 2 == 0) ? bufX : bufY;
         size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 32;
         ProfScope ps_(ctx, s, 2);
@@ -369,16 +431,17 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
     if (validate) CK(cudaMemsetAsync(ctx->d_flag, 0, 4, s));
 
-    const size_t ev_pp = (size_t)P.k * (P.D + 1), ch_pp = P.k, fi_pp = P.D;
-    fe *o_ev, *o_ch, *o_fi, *o_cl;
+    const size_t E = P.esz;
+    const size_t ev_pp = (size_t)P.k * (P.D + 1) * E, ch_pp = P.k * E, fi_pp = P.D * E;   // bytes per proof
+    char *o_ev, *o_ch, *o_fi, *o_cl;
     if (P.host_outputs) {
-        fe *base = (fe *)(ws + P.off_out);
+        char *base = ws + P.off_out;
         o_ev = base; o_ch = o_ev + P.B * ev_pp; o_fi = o_ch + P.B * ch_pp; o_cl = o_fi + P.B * fi_pp;
         if (P.given && P.k)
-            CK(cudaMemcpyAsync(o_ch, b->challenges, P.B * ch_pp * 32, cudaMemcpyHostToDevice, s));
+            CK(cudaMemcpyAsync(o_ch, b->challenges, P.B * ch_pp, cudaMemcpyHostToDevice, s));
     } else {
-        o_ev = (fe *)b->round_evals; o_ch = (fe *)b->challenges; o_fi = (fe *)b->final_evals;
-        o_cl = (fe *)b->claims;
+        o_ev = (char *)b->round_evals; o_ch = (char *)b->challenges; o_fi = (char *)b->final_evals;
+        o_cl = (char *)b->claims;
     }
     for (uint64_t w = 0; w < P.nwaves; ++w) {
         WaveIO io;
@@ -388,8 +451,8 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
         io.first_index = b->first_index + b0;
         io.round_evals = o_ev + b0 * ev_pp;
         io.challenges = o_ch + b0 * ch_pp;
-        io.final_evals = o_fi + b0 * fi_pp;
-        io.claims = (P.host_outputs || o_cl) ? o_cl + b0 : nullptr;
+        io.final_evals = o_fi + b0 * fi_pp;   // (byte offsets)
+        io.claims = (P.host_outputs || o_cl) ? o_cl + b0 * E : nullptr;
         int slot = -1;
         if (P.host_tables) {
             slot = ctx->next_slot;
@@ -402,17 +465,18 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
             }
             CK(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
             CK(cudaStreamWaitEvent(s, ctx->ev_copied[slot], 0));
-            io.tables = (fe *)ctx->stage[slot];
+            io.tables = (char *)ctx->stage[slot];
         } else {
-            io.tables = (fe *)((char *)b->tables + b0 * P.elem_table);
+            io.tables = (char *)b->tables + b0 * P.elem_table;
         }
         if (validate) {
             ProfScope ps_(ctx, s, 4);
-            k_validate<<<kSMs * 8, 256, 0, s>>>(io.tables, io.nb * P.D * P.N, ctx->d_flag);
+            if (P.gl) k_validate_gl<<<kSMs * 8, 256, 0, s>>>((const uint64_t *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
+            else      k_validate<<<kSMs * 8, 256, 0, s>>>((const fe *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
             ++ctx->launches;
             CK(cudaGetLastError());
         }
-        bzk_status st = run_wave(ctx, P, io, s);
+        bzk_status st = P.gl ? run_wave_gl(ctx, P, io, s) : run_wave(ctx, P, io, s);
         if (st) return st;
         if (slot >= 0) {
             CK(cudaEventRecord(ctx->ev_consumed[slot], s));
@@ -421,11 +485,11 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     }
     if (P.host_outputs) {
         if (P.k) {
-            CK(cudaMemcpyAsync(b->round_evals, o_ev, P.B * ev_pp * 32, cudaMemcpyDeviceToHost, s));
-            if (!P.given) CK(cudaMemcpyAsync(b->challenges, o_ch, P.B * ch_pp * 32, cudaMemcpyDeviceToHost, s));
+            CK(cudaMemcpyAsync(b->round_evals, o_ev, P.B * ev_pp, cudaMemcpyDeviceToHost, s));
+            if (!P.given) CK(cudaMemcpyAsync(b->challenges, o_ch, P.B * ch_pp, cudaMemcpyDeviceToHost, s));
         }
-        CK(cudaMemcpyAsync(b->final_evals, o_fi, P.B * fi_pp * 32, cudaMemcpyDeviceToHost, s));
-        if (b->claims) CK(cudaMemcpyAsync(b->claims, o_cl, P.B * 32, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(b->final_evals, o_fi, P.B * fi_pp, cudaMemcpyDeviceToHost, s));
+        if (b->claims) CK(cudaMemcpyAsync(b->claims, o_cl, P.B * E, cudaMemcpyDeviceToHost, s));
     }
     if (validate) {
         uint32_t flag = 0;
@@ -690,6 +754,7 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
     set_kernel_attrs<2>();
     set_kernel_attrs<3>();
     set_kernel_attrs<4>();
+    gl_set_attrs();
     k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
     if (cudaStreamSynchronize(ctx->copy_stream) != cudaSuccess) {
         delete ctx;
@@ -759,7 +824,7 @@ bzk_status bzk_sync(bzk_ctx *ctx) {
 
 bzk_status bzk_generate(uint64_t *dst, uint64_t batch, uint32_t d, uint32_t k, uint64_t first_index,
                         uint32_t dist, uint64_t data_seed, void *cuda_stream) {
-    if (!dst || k > 30 || d < 1 || d > 15 || dist > 2 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
+    if (!dst || k > 30 || d < 1 || d > 15 || dist > 3 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
     k_generate<<<kSMs * 16, 256, 0, (cudaStream_t)cuda_stream>>>(dst, batch, d, k, first_index, dist, data_seed);
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }

@@ -24,6 +24,10 @@ static __global__ void k_generate(uint64_t *dst, uint64_t batch, uint32_t d, uin
         uint64_t m = bm % d, b = bm / d;
         uint64_t I = first_index + b;
         uint64_t base = (I << 36) | (m << 32) | (x << 2);
+        if (dist == 3) {   // Goldilocks: one word per element, masked to 63 bits
+            dst[e] = splitmix64_ctr(base, seed) & ((1ull << 63) - 1);
+            continue;
+        }
         bool small = dist == 1 || (dist == 2 && m == 0);
         uint64_t w0, w1, w2, w3;
         if (small) {

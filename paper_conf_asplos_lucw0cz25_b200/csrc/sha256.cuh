@@ -94,8 +94,9 @@ __device__ __forceinline__ fe digest_to_fe_raw(const uint32_t s[8]) {
 }
 
 // state_0 for proof I (64-byte init block + 1 padding block)
+// field_id: 0 = BN254 Fr, 1 = Goldilocks (reading R15; the last LE16 of the init block)
 __device__ __forceinline__ void transcript_init(uint32_t state[8], const uint8_t seed[32], uint64_t I,
-                                                uint32_t k, uint32_t d, uint32_t order) {
+                                                uint32_t k, uint32_t d, uint32_t order, uint32_t field_id = 0) {
     sha256_words sh;
     sh.init();
     // "BZK-SUMCHECK-V1\0" as big-endian words
@@ -110,7 +111,7 @@ __device__ __forceinline__ void transcript_init(uint32_t state[8], const uint8_t
     sh.push(bswap32((uint32_t)I));
     sh.push(bswap32((uint32_t)(I >> 32)));
     sh.push(bswap32((k & 0xffffu) | ((d & 0xffffu) << 16)));
-    sh.push(bswap32(order & 0xffffu));
+    sh.push(bswap32((order & 0xffffu) | ((field_id & 0xffffu) << 16)));
     sh.finish(state);
 }
 
