@@ -43,6 +43,8 @@ CONFIGS = {
                                       "k=20, MSB order = Alg. 1 pairing"),
     "m0lit": (1024, 1, 20, 1, "uniform", "paper-literal Table 4 analogue: 1024 proofs x single multilinear (d=1), "
                                          "k=20, MSB = Alg. 1 pairing, challenges given (no Fiat-Shamir, P:111)"),
+    "g2": (1024, 2, 20, 0, "gl", "NEXT-2 second field instance: 1024 proofs x product of 2 multilinears, k=20, "
+                                 "Goldilocks p = 2^64 - 2^32 + 1 (8-byte elements: the HBM-bound regime)"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -85,14 +87,14 @@ def alg_mulmods(d: int, k: int, kind: str) -> int:
     raise ValueError(kind)
 
 
-def alg_bytes_kind(d: int, k: int, kind: str) -> int:
+def alg_bytes_kind(d: int, k: int, kind: str, esz: int = 32) -> int:
     """Algorithmic HBM bytes per proof of a kernel kind: round 1 reads d 2^k x 32 B; a fused round
     i reads 4 d h_i x 32 B and writes 2 d h_i x 32 B (ping-pong)."""
     tail_log = 8
     i0 = 1 if k - 1 <= tail_log else k - tail_log
     if kind == "round1":
-        return d * (1 << k) * 32
-    return sum(6 * d * (1 << (k - i)) * 32 for i in range(2, i0))
+        return d * (1 << k) * esz
+    return sum(6 * d * (1 << (k - i)) * esz for i in range(2, i0))
 
 
 class ClockSampler:
@@ -159,11 +161,19 @@ def cpu_baseline(cfg, max_proofs=8):
     B, d, k, order, dist, _ = CONFIGS[cfg]
     cores = len(os.sched_getaffinity(0))
     n = max(1, min(max_proofs, cores, B))
-    tabs = inputs.gen_tables(n, d, k, 0, dist)
     oracle.build()
-    t0 = time.perf_counter()
-    oracle.prove_batch(tabs, k, d, order, inputs.DEFAULT_SEED, 0, nthreads=n)
-    dt = time.perf_counter() - t0
+    if dist == "gl":
+        import concurrent.futures as cf
+        tabs = inputs.gen_tables_gl(n, d, k, 0)
+        t0 = time.perf_counter()
+        with cf.ThreadPoolExecutor(n) as ex:     # ctypes releases the GIL: one proof per thread
+            list(ex.map(lambda b: oracle.gl_prove(tabs[b], k, d, order, inputs.DEFAULT_SEED, b), range(n)))
+        dt = time.perf_counter() - t0
+    else:
+        tabs = inputs.gen_tables(n, d, k, 0, dist)
+        t0 = time.perf_counter()
+        oracle.prove_batch(tabs, k, d, order, inputs.DEFAULT_SEED, 0, nthreads=n)
+        dt = time.perf_counter() - t0
     return {"value": n / dt, "unit": "proofs/s", "cores": n, "kind": "oracle",
             "sample": f"{n} proofs of {cfg} (d={d}, k={k}), one per thread, {dt:.1f} s wall"}
 
@@ -336,14 +346,21 @@ def main():
         B = args.batch
     first, _ = shard.weak_range(B, rank)
     consume = args.config == "c3"
+    gl = gen_dist == "gl"
+    esz = 8 if gl else 32
     flags = 0 if consume else bzk.BZK_F_PRESERVE_INPUT
+    if gl:
+        flags |= bzk.BZK_F_FIELD_GOLDILOCKS
+
+    def tshape(n):
+        return (n, d, 1 << k) if gl else (n, d, 1 << k, 4)
     if args.config == "m0lit":
         flags |= bzk.BZK_F_GIVEN_CHALLENGES
     stream = torch.cuda.Stream()
-    tables = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+    tables = torch.empty(tshape(B), dtype=torch.int64, device="cuda")
     bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
     prover = bzk.Prover(local)
-    out = bzk.Prover.alloc_outputs(B, k, d)
+    out = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(B, k, d)
     if flags & bzk.BZK_F_GIVEN_CHALLENGES:
         # pre-seeded challenges (the paper's PRG output): any canonical values < 2^253
         kk = max(1, (k - 1).bit_length())          # generator tables have 2^kk >= k entries
@@ -419,7 +436,7 @@ def main():
     total_alg = alg_mulmods(d, k, "total") * B
     step_gmulmod = total_alg / (ms_per_step / 1000.0) / 1e9
     # HBM: algorithmic bytes (read each input once) and the streaming schedule's bytes
-    alg_bytes = d * (1 << k) * 32 * B
+    alg_bytes = d * (1 << k) * esz * B
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
@@ -429,22 +446,32 @@ def main():
             tj = json.load(f)
         if tj.get("config") == args.config and tj.get("kernel_kind") == dom and tj.get("batch") == B:
             traffic = tj["dram_bytes_per_launch"]
+    bytes_per_launch = alg_bytes_kind(d, k, kinds[dom], esz) * B / max(1, dom_cnt / args.steps)
     roofline = {"bound": "alu", "kernel": dom, "achieved": round(achieved, 2), "peak": round(int_peak, 2),
                 "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": traffic,
-                "alg_bytes_per_launch": alg_bytes_kind(d, k, kinds[dom]) * B / max(1, dom_cnt / args.steps),
+                "alg_bytes_per_launch": bytes_per_launch,
                 "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} MHz "
                                f"({peak_src} max clock) / {IMAD_PER_MULMOD} IMAD per mulmod",
                 "step_frac": round(step_gmulmod / int_peak, 4),
                 "hbm_alg_frac": round(alg_bytes / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
                 "hbm_peak_gbs": hbm_peak}
+    if gl:
+        # Goldilocks (8-byte elements): the dominant kernel streams; its roof is HBM bandwidth
+        ach_gbs = bytes_per_launch / avg_launch_s / 1e9
+        roofline.update({"bound": "hbm", "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
+                         "frac": round(ach_gbs / hbm_peak, 4),
+                         "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); achieved = algorithmic bytes per "
+                                        "launch (reads 4dh + writes 2dh elements per proof for a fused round, 2dh "
+                                        "reads for round 1) / CUDA-event launch time",
+                         "alu_gmulmod_s": round(achieved, 2)})
 
     kernel_ms = {n: round(v[0] / args.steps, 3) for n, v in prof.items() if v[1]}
     line = {"metric": METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64" if gl else "u32", "data": "synthetic",
             "config": {"workload": desc, "batch_per_gpu": B, "global_batch": B * world, "d": d, "k": k,
-                       "order": "LSB" if order == 0 else "MSB", "field": "BN254 Fr",
-                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * d * (1 << k) * 32 / 2**30)},
+                       "order": "LSB" if order == 0 else "MSB", "field": "Goldilocks" if gl else "BN254 Fr",
+                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * d * (1 << k) * esz / 2**30)},
             "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
             "kernel_ms_per_step": kernel_ms, "ms_per_step_kernel_by_kernel": round(sum(step_ms_prof) / args.steps, 3),
             "roofline": roofline, "clocks": clocks,
@@ -454,9 +481,9 @@ def main():
     if not args.no_e2e and not consume:
         del tables
         torch.cuda.empty_cache()
-        host_t = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, pin_memory=True)
+        host_t = torch.empty(tshape(B), dtype=torch.int64, pin_memory=True)
         chunk = max(1, B // 16)
-        tmp = torch.empty((chunk, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+        tmp = torch.empty(tshape(chunk), dtype=torch.int64, device="cuda")
         for c0 in range(0, B, chunk):
             n = min(chunk, B - c0)
             bzk.bzk_generate(tmp, n, d, k, first + c0, gen_dist, stream=stream)
@@ -464,10 +491,11 @@ def main():
             host_t[c0:c0 + n].copy_(tmp[:n])
         del tmp
         torch.cuda.empty_cache()
-        out_h = bzk.Prover.alloc_outputs(B, k, d, device="cpu", pin=True)
+        out_h = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(B, k, d, device="cpu", pin=True)
         if flags & bzk.BZK_F_GIVEN_CHALLENGES:
             out_h["challenges"].copy_(out["challenges"])
-        hb = prover.batch(host_t, k, d, order, None, first, flags & bzk.BZK_F_GIVEN_CHALLENGES, out_h)
+        hb = prover.batch(host_t, k, d, order, None, first,
+                          flags & (bzk.BZK_F_GIVEN_CHALLENGES | bzk.BZK_F_FIELD_GOLDILOCKS), out_h)
         bzk.bzk_prove(prover.ctx, hb, stream)   # warm-up (allocates staging)
         barrier()
         t0 = time.perf_counter()

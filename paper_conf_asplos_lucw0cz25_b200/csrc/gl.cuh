@@ -185,8 +185,15 @@ __device__ __forceinline__ void load_pair(const uint64_t *src, uint64_t *dst, ui
     }
 }
 
+#ifndef GL_MLP
+#define GL_MLP 4
+#endif
+#ifndef GL_OCC
+#define GL_OCC 3
+#endif
+
 template <int D, int ORDER, bool FIRST>
-__global__ void __launch_bounds__(256) k_gl_round(RoundParams P) {
+__global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
     __shared__ uint64_t s_red[32 * (D + 1)];
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
@@ -199,15 +206,15 @@ __global__ void __launch_bounds__(256) k_gl_round(RoundParams P) {
     const uint64_t r = FIRST ? 0 : P.ps[b].r;
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    // two pairs in flight per iteration (memory-level parallelism)
-    for (; j + stride < h; j += 2 * stride) {
-        uint64_t a0[D], b0[D], a1[D], b1[D];
-        load_pair<D, ORDER, FIRST>(src, dst, h, j, r, a0, b0);
-        load_pair<D, ORDER, FIRST>(src, dst, h, j + stride, r, a1, b1);
-        eval_pair<D>(a0, b0, acc);
-        eval_pair<D>(a1, b1, acc);
+    // GL_MLP pairs in flight per iteration (memory-level parallelism: the kernel streams)
+    for (; j + (GL_MLP - 1) * stride < h; j += GL_MLP * stride) {
+        uint64_t a[GL_MLP][D], bb[GL_MLP][D];
+#pragma unroll
+        for (int q = 0; q < GL_MLP; ++q) load_pair<D, ORDER, FIRST>(src, dst, h, j + q * stride, r, a[q], bb[q]);
+#pragma unroll
+        for (int q = 0; q < GL_MLP; ++q) eval_pair<D>(a[q], bb[q], acc);
     }
-    if (j < h) {
+    for (; j < h; j += stride) {
         uint64_t a0[D], b0[D];
         load_pair<D, ORDER, FIRST>(src, dst, h, j, r, a0, b0);
         eval_pair<D>(a0, b0, acc);
