@@ -284,7 +284,9 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
     if (round == 1 && claims) st_fe(claims, fe_add(g[0], g[1]));
     fe rm = mont_mul(r, fe_const(2));
     ps.rmont = rm;
-    ps.claim = lagrange_at<D>(g, rm, consts);
+    // the next claim feeds g(1) = claim - g(0) of a fused global round; the on-chip tail (MODE 0)
+    // sums every point directly, so it skips the interpolation (9-16 serial products per round)
+    if (MODE != 0) ps.claim = lagrange_at<D>(g, rm, consts);
     if (rmont_out) *rmont_out = rm;
 }
 

@@ -60,3 +60,61 @@ def test_config3_full_size(orc):
     rng = np.random.default_rng(3)
     sample = sorted({0, 255, *rng.choice(256, size=2, replace=False).tolist()})
     run_full(orc, 256, 3, 22, 0, 0, sample)
+
+
+def test_m0_and_g2_full_size(orc):
+    """m0 (paper shape: 1024 x d=1, k=20, MSB) and g2 (Goldilocks 1024 x d=2, k=20) at full size in
+    bench.py's launch configuration: sampled proofs vs the oracle."""
+    rng = np.random.default_rng(4)
+    sample = sorted({0, 1023, *rng.choice(1024, size=2, replace=False).tolist()})
+    torch.cuda.empty_cache()
+    # m0
+    t = torch.empty((1024, 1, 1 << 20, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(t, 1024, 1, 20, 0, "uniform")
+    p = bzk.Prover(0)
+    out = p.prove(t, 20, 1, 1, flags=bzk.BZK_F_PRESERVE_INPUT)
+    p.sync()
+    del t
+    for i in sample:
+        ref = orc.prove(inputs.gen_tables(1, 1, 20, first_index=i)[0], 20, 1, 1, SEED, i)
+        for key in KEYS:
+            assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), ("m0", key, i)
+    torch.cuda.empty_cache()
+    # g2
+    t = torch.empty((1024, 2, 1 << 20), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(t, 1024, 2, 20, 0, "gl")
+    out = p.prove(t, 20, 2, 0, flags=bzk.BZK_F_PRESERVE_INPUT | bzk.BZK_F_FIELD_GOLDILOCKS)
+    p.sync()
+    host = np64(t[sample])
+    for n, i in enumerate(sample):
+        ref = orc.gl_prove(host[n], 20, 2, 0, SEED, i)
+        for key in KEYS:
+            assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), ("g2", key, i)
+    p.close()
+    del t
+    torch.cuda.empty_cache()
+
+
+def test_vml_image_shapes(orc):
+    """configs[3]: the 32 sum-checks of one VGG-16/CIFAR-10-shaped image (k per layer as bench.py),
+    streamed from pinned host memory through bzk_prove_ragged, every proof vs the oracle."""
+    ks = [16, 16, 15, 15, 14, 14, 14, 13, 13, 13, 11, 11, 11, 9, 9, 9]
+    p = bzk.Prover(0)
+    jobs, outs, tabs = [], [], []
+    for li, k in enumerate(ks):
+        I = 5000 + 2 * li
+        t = torch.empty((2, 2, 1 << k, 4), dtype=torch.int64, device="cuda")
+        bzk.bzk_generate(t, 2, 2, k, I, "vml")
+        ht = t.cpu().pin_memory()
+        o = bzk.Prover.alloc_outputs(2, k, 2, device="cpu", pin=True)
+        tabs.append(ht)
+        outs.append(o)
+        jobs.append(p.batch(ht, k, 2, 0, None, I, 0, o))
+    bzk.bzk_prove_ragged(p.ctx, jobs)
+    for li, k in enumerate(ks):
+        host = tabs[li].numpy().view(np.uint64)
+        for b in range(2):
+            ref = orc.prove(host[b], k, 2, 0, SEED, 5000 + 2 * li + b)
+            for key in KEYS:
+                assert np.array_equal(outs[li][key][b].numpy().view(np.uint64).reshape(ref[key].shape), ref[key])
+    p.close()
