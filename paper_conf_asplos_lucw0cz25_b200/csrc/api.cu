@@ -25,6 +25,7 @@ using namespace bzk;
 namespace {
 
 constexpr uint32_t kThreads = 256;
+constexpr uint32_t kRoundThreads = BZK_RT;   // k_round CTA size (sumcheck.cuh)
 constexpr uint32_t kTailLog = 8;          // rounds with h <= 2^kTailLog pairs run in k_tail
 constexpr uint32_t kSMs = 148;
 
@@ -139,9 +140,9 @@ const Knobs &knobs() { static Knobs k; return k; }
 uint32_t ctas_for(uint64_t h, uint64_t nb) {
     // enough CTAs to fill 148 SMs x 2 resident CTAs x `waves` waves, at most ppt_max pairs per thread
     const uint64_t target = (uint64_t)kSMs * 2 * knobs().waves;
-    uint64_t ppt = (nb * h) / ((uint64_t)kThreads * target);
+    uint64_t ppt = (nb * h) / ((uint64_t)kRoundThreads * target);
     ppt = std::max<uint64_t>(1, std::min<uint64_t>(knobs().ppt_max, ppt));
-    uint64_t c = (h + kThreads * ppt - 1) / (kThreads * ppt);
+    uint64_t c = (h + kRoundThreads * ppt - 1) / (kRoundThreads * ppt);
     return (uint32_t)std::max<uint64_t>(1, c);
 }
 
@@ -270,10 +271,10 @@ bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
 cudaError_t dispatch_round(uint32_t D, uint32_t order, bool first, dim3 grid, cudaStream_t s,
                            const RoundParams &p) {
     switch (D) {
-        case 1: return launch_round<1>(order, first, grid, kThreads, s, p);
-        case 2: return launch_round<2>(order, first, grid, kThreads, s, p);
-        case 3: return launch_round<3>(order, first, grid, kThreads, s, p);
-        case 4: return launch_round<4>(order, first, grid, kThreads, s, p);
+        case 1: return launch_round<1>(order, first, grid, kRoundThreads, s, p);
+        case 2: return launch_round<2>(order, first, grid, kRoundThreads, s, p);
+        case 3: return launch_round<3>(order, first, grid, kRoundThreads, s, p);
+        case 4: return launch_round<4>(order, first, grid, kRoundThreads, s, p);
     }
     return cudaErrorInvalidValue;
 }

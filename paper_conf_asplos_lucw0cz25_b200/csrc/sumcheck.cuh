@@ -26,6 +26,9 @@
 #include <stdint.h>
 #include "field.cuh"
 
+#ifndef BZK_RT
+#define BZK_RT 256        // threads per CTA of k_round
+#endif
 #ifndef BZK_ROUND_OCC
 #define BZK_ROUND_OCC 2   // resident CTAs per SM requested for k_round (d <= 2)
 #endif
@@ -502,7 +505,7 @@ constexpr size_t round_smem_bytes(uint32_t threads) {
 }
 
 template <int D, int ORDER, bool FIRST>
-__global__ void __launch_bounds__(256, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
+__global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
     constexpr bool DERIVE = !FIRST;
     constexpr int NV = Pts<D, DERIVE>::NV;
     __shared__ fe s_red[32 * NV];
