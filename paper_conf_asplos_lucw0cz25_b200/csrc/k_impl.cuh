@@ -3,18 +3,37 @@
 
 namespace bzk {
 
+template <int ORDER, bool FIRST>
+static cudaError_t launch_round_cl(dim3 grid, uint32_t threads, size_t sm, cudaStream_t s, const RoundParams &p,
+                                   uint32_t cluster) {
+    if (cluster <= 1) {
+        k_round<BZK_D, ORDER, FIRST><<<grid, threads, sm, s>>>(p);
+        return cudaGetLastError();
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(threads, 1, 1);
+    cfg.dynamicSmemBytes = sm;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = cluster;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_round<BZK_D, ORDER, FIRST>, p);
+}
+
 template <>
 cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
                                 const RoundParams &p) {
     const size_t sm = first ? round_smem_bytes<BZK_D, true>(threads) : round_smem_bytes<BZK_D, false>(threads);
-    if (order == 0) {
-        if (first) k_round<BZK_D, 0, true><<<grid, threads, sm, s>>>(p);
-        else       k_round<BZK_D, 0, false><<<grid, threads, sm, s>>>(p);
-    } else {
-        if (first) k_round<BZK_D, 1, true><<<grid, threads, sm, s>>>(p);
-        else       k_round<BZK_D, 1, false><<<grid, threads, sm, s>>>(p);
-    }
-    return cudaGetLastError();
+    const uint32_t cl = p.cluster;
+    if (order == 0) return first ? launch_round_cl<0, true>(grid, threads, sm, s, p, cl)
+                                 : launch_round_cl<0, false>(grid, threads, sm, s, p, cl);
+    return first ? launch_round_cl<1, true>(grid, threads, sm, s, p, cl)
+                 : launch_round_cl<1, false>(grid, threads, sm, s, p, cl);
 }
 
 template <>

@@ -23,6 +23,7 @@
 //   k_tail<D,ORDER>  one CTA per proof finishes the remaining rounds (h <= tail threshold) in
 //       shared memory, including the final fold that yields final_m = f_m(rho).
 #pragma once
+#include <cooperative_groups.h>
 #include <stdint.h>
 #include "field.cuh"
 
@@ -65,6 +66,7 @@ struct RoundParams {
     const fe *consts;     // kNumConsts
     uint32_t prefetch;    // 1: bulk-prefetch the next iteration's tiles into L2
     uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
+    uint32_t cluster;     // thread-block cluster size along x (1 = none); divides ctas
 };
 
 // ---------------------------------------------------------------- reductions
@@ -509,6 +511,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     constexpr bool DERIVE = !FIRST;
     constexpr int NV = Pts<D, DERIVE>::NV;
     __shared__ fe s_red[32 * NV];
+    __shared__ fe s_clu[NV];
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
     const uint64_t h = 1ull << P.log_h;
@@ -597,13 +600,36 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
             finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr, P.given);
         return;
     }
+    // Thread-block cluster (launched with cluster dims (cs, 1, 1), cs <= 8, all CTAs of one proof):
+    // the cluster's CTA sums are combined through distributed shared memory, so only one partial
+    // per cluster goes to global memory and through the last-CTA ticket.
+    namespace cg = cooperative_groups;
+    cg::cluster_group cluster = cg::this_cluster();
+    const uint32_t cs = cluster.num_blocks();
+    if (cs > 1) {
+        if (threadIdx.x == 0)
+#pragma unroll
+            for (int t = 0; t < NV; ++t) s_clu[t] = acc[t];
+        cluster.sync();
+        const bool leader = cluster.block_rank() == 0;
+        if (leader && threadIdx.x == 0) {
+            for (uint32_t r = 1; r < cs; ++r) {
+                const fe *rem = cluster.map_shared_rank(s_clu, r);
+#pragma unroll
+                for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], rem[t]);
+            }
+        }
+        cluster.sync();   // remote shared memory must outlive the leader's reads
+        if (!leader) return;
+    }
+    const uint32_t nparts = P.ctas / cs, pidx = blockIdx.x / cs;
     fe *part = P.partials + (size_t)b * P.ctas * NV;
     if (threadIdx.x == 0) {
 #pragma unroll
-        for (int t = 0; t < NV; ++t) st_fe_cg(&part[(size_t)blockIdx.x * NV + t], acc[t]);
+        for (int t = 0; t < NV; ++t) st_fe_cg(&part[(size_t)pidx * NV + t], acc[t]);
         __threadfence();
         uint32_t old = atomicAdd(&P.tickets[b], 1u);
-        s_last = (old == P.ctas - 1);
+        s_last = (old == nparts - 1);
     }
     __syncthreads();
     if (!s_last) return;
@@ -611,7 +637,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     // last CTA of proof b: cooperative sum of all partials
 #pragma unroll
     for (int t = 0; t < NV; ++t) acc[t] = fe_zero();
-    for (uint32_t c = threadIdx.x; c < P.ctas; c += blockDim.x)
+    for (uint32_t c = threadIdx.x; c < nparts; c += blockDim.x)
 #pragma unroll
         for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], ld_fe_cg(&part[(size_t)c * NV + t]));
     block_reduce<NV>(acc, s_red);
