@@ -176,6 +176,15 @@ bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
     if (!b->final_evals) return fail(ctx, BZK_EINVAL, "final_evals is NULL");
     if (b->tables_mem > 1 || b->outputs_mem > 1) return fail(ctx, BZK_EINVAL, "bad *_mem value");
     if (b->first_index + b->batch > (1ull << 28)) return fail(ctx, BZK_EINVAL, "global index must be < 2^28");
+    // BN254 kernels access elements with 256-bit loads/stores: device buffers must be 32-byte aligned
+    if (!(b->flags & BZK_F_FIELD_GOLDILOCKS)) {
+        auto mis = [](const void *q) { return q && ((uintptr_t)q & 31u); };
+        if (b->tables_mem == BZK_MEM_DEVICE && mis(b->tables))
+            return fail(ctx, BZK_EINVAL, "device tables must be 32-byte aligned");
+        if (b->outputs_mem == BZK_MEM_DEVICE &&
+            (mis(b->round_evals) || mis(b->challenges) || mis(b->final_evals) || mis(b->claims)))
+            return fail(ctx, BZK_EINVAL, "device outputs must be 32-byte aligned");
+    }
     return BZK_OK;
 }
 

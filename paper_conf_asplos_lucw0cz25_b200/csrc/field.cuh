@@ -488,6 +488,113 @@ __device__ __forceinline__ fe mont_mul2_lz(const fe &x, const fe &y, const fe &u
     return r;
 }
 
+// ---------------------------------------------------------------- fixed-multiplier product (folds)
+//
+// Every fold of one proof in one round multiplies by the SAME challenge r (Alg. 1
+// line 5), so the product r * x can use a per-(proof, round) table instead of a CIOS product:
+//   K_i = r * 2^(32 i + 64) mod p,  i = 0..7  (canonical, in shared memory, built once per CTA)
+//   V   = sum_i x_i K_i   (x_i = 32-bit limbs of x; any x < 2^256)   ->  V < 8 * 2^32 * p < 2^289
+//   two Montgomery word steps: (V + q p) / 2^64 == r x (mod p),  result < p (1 + 2^-29) < 2p.
+// 64 + 18 limb products instead of 136 for mont_mul_lz (the rows need no reduction in between).
+
+// 8 words of K_i from shared memory (broadcast).  The address carries a false data dependency on
+// a word of the previous row (dep & zmask, zmask = 0 from a kernel parameter ptxas cannot see
+// through), so the loads stay one row ahead instead of the whole 64-word table being hoisted into
+// registers.
+__device__ __forceinline__ void lds_k(uint32_t k[8], const fe *Ki, uint32_t dep, uint32_t zmask) {
+    const uint32_t a = (uint32_t)__cvta_generic_to_shared(Ki) + (dep & zmask);
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%8];\n\t"
+                 "ld.shared.v4.u32 {%4, %5, %6, %7}, [%8+16];"
+                 : "=r"(k[0]), "=r"(k[1]), "=r"(k[2]), "=r"(k[3]), "=r"(k[4]), "=r"(k[5]), "=r"(k[6]), "=r"(k[7])
+                 : "r"(a));
+}
+
+// carry-propagating add of a pending word at column 0 of A (A[q] at column q)
+__device__ __forceinline__ void add_l(uint32_t A[9], uint32_t L) {
+    asm("add.cc.u32  %0, %0, %9;\n\t"
+        "addc.cc.u32 %1, %1, 0;\n\t"
+        "addc.cc.u32 %2, %2, 0;\n\t"
+        "addc.cc.u32 %3, %3, 0;\n\t"
+        "addc.cc.u32 %4, %4, 0;\n\t"
+        "addc.cc.u32 %5, %5, 0;\n\t"
+        "addc.cc.u32 %6, %6, 0;\n\t"
+        "addc.cc.u32 %7, %7, 0;\n\t"
+        "addc.u32    %8, %8, 0;"
+        : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
+          "+r"(A[8])
+        : "r"(L));
+}
+
+__device__ __forceinline__ fe fixmul_lz(const fe &x, const fe *K, uint32_t zmask) {
+    uint32_t A[9], B[9], k[8];
+    lds_k(k, K, x.l[0], zmask);
+    // row 0: A (columns 0..8) = K0_even * x0, B (columns 1..9) = K0_odd * x0
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]), "=r"(A[4]), "=r"(A[5]), "=r"(A[6]), "=r"(A[7]),
+          "=r"(A[8])
+        : "r"(k[0]), "r"(k[2]), "r"(k[4]), "r"(k[6]), "r"(x.l[0]));
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(B[0]), "=r"(B[1]), "=r"(B[2]), "=r"(B[3]), "=r"(B[4]), "=r"(B[5]), "=r"(B[6]), "=r"(B[7]),
+          "=r"(B[8])
+        : "r"(k[1]), "r"(k[3]), "r"(k[5]), "r"(k[7]), "r"(x.l[0]));
+    // rows 1..7: every row lands on the same columns (K_i already carries the 2^(32 i) weight)
+#pragma unroll
+    for (int i = 1; i < 8; ++i) {
+        lds_k(k, K + i, A[0], zmask);
+        row_a(A, k, x.l[i]);
+        row_b_nl(B, k, x.l[i]);
+    }
+    // two Montgomery word steps (divide by 2^64); same column bookkeeping as mont_mul_lz
+    uint32_t L = 0;
+#pragma unroll
+    for (int s = 0; s < 2; ++s) {
+        if (s > 0) add_l(A, L);
+        const uint32_t m = mont_m(A[0]);
+        red_a(A, m);
+        red_b(B, m);
+        L = A[1];
+        uint32_t nA[9], nB[9];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) nA[q] = B[q];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) nB[q] = A[q + 2];
+        nB[7] = 0;
+        nB[8] = 0;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) { A[q] = nA[q]; B[q] = nB[q]; }
+    }
+    fe r;   // A + L + (B << 32) < 2^255: A8, B7, B8 are zero
+    asm("add.cc.u32  %0, %8,  %16;\n\t"
+        "addc.cc.u32 %1, %9,  %17;\n\t"
+        "addc.cc.u32 %2, %10, %18;\n\t"
+        "addc.cc.u32 %3, %11, %19;\n\t"
+        "addc.cc.u32 %4, %12, %20;\n\t"
+        "addc.cc.u32 %5, %13, %21;\n\t"
+        "addc.cc.u32 %6, %14, %22;\n\t"
+        "addc.u32    %7, %15, %23;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
+          "=r"(r.l[7])
+        : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
+          "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
+    return r;
+}
+
 // (x*y + u*v) * R^{-1} mod p, canonical; x, y, u, v canonical (result of the lazy form < 3p)
 __device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, const fe &v) {
     return fe_reduce_once(fe_reduce_once(mont_mul2_lz(x, y, u, v)));
@@ -598,6 +705,103 @@ __device__ __forceinline__ void acc9_add(acc9 &a, const fe &x) {
         : "r"(x.l[0]), "r"(x.l[1]), "r"(x.l[2]), "r"(x.l[3]), "r"(x.l[4]), "r"(x.l[5]), "r"(x.l[6]), "r"(x.l[7]));
 }
 
+// ---------------------------------------------------------------- unreduced product sums
+//
+// A round sum  S = sum_j x_j y_j  needs only ONE Montgomery reduction per thread, after the loop:
+// the 512-bit products are added into a 544-bit accumulator (17 words; room for 2^32 products of
+// values < 4p) and acc17_to_fe returns S * R^{-1} mod p -- the same value (and scale) as summing
+// mont_mul(x_j, y_j).  64 limb products per product instead of 100 (mont_mul2) or 136 (mont_mul).
+struct acc17 { uint32_t w[17]; };
+__device__ __forceinline__ acc17 acc17_zero() {
+    acc17 a;
+#pragma unroll
+    for (int i = 0; i < 17; ++i) a.w[i] = 0;
+    return a;
+}
+
+// acc += x * y   (x * y < 2^512).  Row-scanned product on the parity-aligned A/B chains of
+// mont_mul_lz without the reduction rows: after row i the lowest relative column (A0) is final
+// and is emitted to out[i]; the shift re-pairs the chains exactly as in mont_mul_lz.
+__device__ __forceinline__ void mul_acc(acc17 &acc, const fe &x, const fe &y) {
+    uint32_t A[9], B[9], L, out[8];
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]), "=r"(A[4]), "=r"(A[5]), "=r"(A[6]), "=r"(A[7]),
+          "=r"(A[8])
+        : "r"(x.l[0]), "r"(x.l[2]), "r"(x.l[4]), "r"(x.l[6]), "r"(y.l[0]));
+    asm("mul.lo.u32 %0, %9,  %13;\n\t"
+        "mul.hi.u32 %1, %9,  %13;\n\t"
+        "mul.lo.u32 %2, %10, %13;\n\t"
+        "mul.hi.u32 %3, %10, %13;\n\t"
+        "mul.lo.u32 %4, %11, %13;\n\t"
+        "mul.hi.u32 %5, %11, %13;\n\t"
+        "mul.lo.u32 %6, %12, %13;\n\t"
+        "mul.hi.u32 %7, %12, %13;\n\t"
+        "mov.u32    %8, 0;"
+        : "=r"(B[0]), "=r"(B[1]), "=r"(B[2]), "=r"(B[3]), "=r"(B[4]), "=r"(B[5]), "=r"(B[6]), "=r"(B[7]),
+          "=r"(B[8])
+        : "r"(x.l[1]), "r"(x.l[3]), "r"(x.l[5]), "r"(x.l[7]), "r"(y.l[0]));
+#pragma unroll
+    for (int i = 1; i < 8; ++i) {
+        out[i - 1] = A[0];
+        L = A[1];
+        uint32_t nA[9], nB[9];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) nA[q] = B[q];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) nB[q] = A[q + 2];
+        nB[7] = 0;
+        nB[8] = 0;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) { A[q] = nA[q]; B[q] = nB[q]; }
+        row_b_z(A, B, L, x.l, y.l[i]);
+        row_a(A, x.l, y.l[i]);
+    }
+    out[7] = A[0];
+    // acc[0..7] += out, acc[8..15] += A[1..8], carry -> acc[16]; then acc[8..16] += B[0..8]
+    asm("add.cc.u32  %0,  %0,  %17;\n\t"
+        "addc.cc.u32 %1,  %1,  %18;\n\t"
+        "addc.cc.u32 %2,  %2,  %19;\n\t"
+        "addc.cc.u32 %3,  %3,  %20;\n\t"
+        "addc.cc.u32 %4,  %4,  %21;\n\t"
+        "addc.cc.u32 %5,  %5,  %22;\n\t"
+        "addc.cc.u32 %6,  %6,  %23;\n\t"
+        "addc.cc.u32 %7,  %7,  %24;\n\t"
+        "addc.cc.u32 %8,  %8,  %25;\n\t"
+        "addc.cc.u32 %9,  %9,  %26;\n\t"
+        "addc.cc.u32 %10, %10, %27;\n\t"
+        "addc.cc.u32 %11, %11, %28;\n\t"
+        "addc.cc.u32 %12, %12, %29;\n\t"
+        "addc.cc.u32 %13, %13, %30;\n\t"
+        "addc.cc.u32 %14, %14, %31;\n\t"
+        "addc.cc.u32 %15, %15, %32;\n\t"
+        "addc.u32    %16, %16, 0;"
+        : "+r"(acc.w[0]), "+r"(acc.w[1]), "+r"(acc.w[2]), "+r"(acc.w[3]), "+r"(acc.w[4]), "+r"(acc.w[5]),
+          "+r"(acc.w[6]), "+r"(acc.w[7]), "+r"(acc.w[8]), "+r"(acc.w[9]), "+r"(acc.w[10]), "+r"(acc.w[11]),
+          "+r"(acc.w[12]), "+r"(acc.w[13]), "+r"(acc.w[14]), "+r"(acc.w[15]), "+r"(acc.w[16])
+        : "r"(out[0]), "r"(out[1]), "r"(out[2]), "r"(out[3]), "r"(out[4]), "r"(out[5]), "r"(out[6]), "r"(out[7]),
+          "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]), "r"(A[8]));
+    asm("add.cc.u32  %0, %0, %9;\n\t"
+        "addc.cc.u32 %1, %1, %10;\n\t"
+        "addc.cc.u32 %2, %2, %11;\n\t"
+        "addc.cc.u32 %3, %3, %12;\n\t"
+        "addc.cc.u32 %4, %4, %13;\n\t"
+        "addc.cc.u32 %5, %5, %14;\n\t"
+        "addc.cc.u32 %6, %6, %15;\n\t"
+        "addc.cc.u32 %7, %7, %16;\n\t"
+        "addc.u32    %8, %8, %17;"
+        : "+r"(acc.w[8]), "+r"(acc.w[9]), "+r"(acc.w[10]), "+r"(acc.w[11]), "+r"(acc.w[12]), "+r"(acc.w[13]),
+          "+r"(acc.w[14]), "+r"(acc.w[15]), "+r"(acc.w[16])
+        : "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]), "r"(B[7]), "r"(B[8]));
+}
+
 __device__ __forceinline__ fe fe_const(int which) {
     fe r;
     switch (which) {
@@ -665,13 +869,29 @@ __device__ __forceinline__ fe ld_fe(const fe *p) {
     return r;
 }
 
-// streaming (evict-first) load for data read exactly once
+// 256-bit global accesses (sm_100: LDG/STG.E.ENL2.256): one instruction per element, and every
+// store writes whole 32-byte sectors (with two 128-bit stores per element the fused rounds read
+// ~60 % of their written bytes back from DRAM: partial-sector write fills, ncu r01g)
+#ifndef BZK_V8
+#define BZK_V8 1
+#endif
+#define BZK_LD8(MOD, r, ptr)                                                                      \
+    asm("ld.global" MOD ".v8.u32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"                          \
+        : "=r"((r).l[0]), "=r"((r).l[1]), "=r"((r).l[2]), "=r"((r).l[3]), "=r"((r).l[4]), "=r"((r).l[5]), \
+          "=r"((r).l[6]), "=r"((r).l[7])                                                            \
+        : "l"(ptr))
+
+// streaming load for data read exactly once (evict-first)
 __device__ __forceinline__ fe ld_fe_stream(const fe *p) {
+    fe r;
+#if BZK_V8
+    BZK_LD8(".cs", r, p);
+#else
     const uint4 *q = reinterpret_cast<const uint4 *>(p);
     uint4 x = __ldcs(q), y = __ldcs(q + 1);
-    fe r;
     r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
     r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+#endif
     return r;
 }
 
@@ -686,9 +906,15 @@ __device__ __forceinline__ fe ld_fe_cg(const fe *p) {
 }
 
 __device__ __forceinline__ void st_fe(fe *p, const fe &v) {
+#if BZK_V8
+    asm volatile("st.global.v8.u32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "r"(v.l[0]), "r"(v.l[1]),
+                 "r"(v.l[2]), "r"(v.l[3]), "r"(v.l[4]), "r"(v.l[5]), "r"(v.l[6]), "r"(v.l[7])
+                 : "memory");
+#else
     uint4 *q = reinterpret_cast<uint4 *>(p);
     q[0] = make_uint4(v.l[0], v.l[1], v.l[2], v.l[3]);
     q[1] = make_uint4(v.l[4], v.l[5], v.l[6], v.l[7]);
+#endif
 }
 
 __device__ __forceinline__ void st_fe_cg(fe *p, const fe &v) {

@@ -46,9 +46,11 @@ struct ProofState {
 // Device constants (filled once per context by k_init_consts):
 //   [0..4]        l * R mod p, l = 0..4          (Montgomery form of the node l)
 //   [5 + 5D + j]  w_{D,j}^{-1} * R mod p, w_{D,j} = prod_{l != j, 0<=l<=D} (j - l)   (Lagrange)
+//   [30 + i]      2^(32 i + 64) mod p, i = 0..7   (fixed-multiplier fold table: K_i = r * this)
 constexpr int kConstLR = 0;
 constexpr int kConstInvW = 5;
-constexpr int kNumConsts = 5 + 5 * 5;
+constexpr int kConstPow2 = 30;
+constexpr int kNumConsts = 5 + 5 * 5 + 8;
 
 struct RoundParams {
     const fe *src;        // FIRST: [Bw][D][2h]; else [Bw][D][4h]
@@ -67,6 +69,7 @@ struct RoundParams {
     uint32_t prefetch;    // 1: bulk-prefetch the next iteration's tiles into L2
     uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
     uint32_t cluster;     // thread-block cluster size along x (1 = none); divides ctas
+    uint32_t zero;        // always 0 (opaque to the compiler: orders the fold-table loads, fixmul_lz)
 };
 
 // ---------------------------------------------------------------- reductions
@@ -172,6 +175,85 @@ __device__ __forceinline__ fe acc9_to_fe(const acc9 &a) {
     return fe_add(fe_reduce_256(a.lo), mont_mul(h, fe_const(2)));   // hi * R^2 * R^-1 = hi * R
 }
 
+// 544-bit accumulator -> S * R^{-1} mod p, canonical (once per thread after the loop; plain code)
+__device__ __forceinline__ fe acc17_to_fe(const acc17 &a) {
+    const uint32_t P[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
+    uint32_t t[18];
+#pragma unroll
+    for (int i = 0; i < 17; ++i) t[i] = a.w[i];
+    t[17] = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {   // Montgomery REDC: t += m p 2^(32 i) clears word i
+        const uint32_t m = t[i] * BZK_NP0;
+        uint64_t c = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const uint64_t x = (uint64_t)m * P[j] + t[i + j] + c;
+            t[i + j] = (uint32_t)x;
+            c = x >> 32;
+        }
+#pragma unroll
+        for (int j = i + 8; j < 18; ++j) {
+            const uint64_t x = (uint64_t)t[j] + c;
+            t[j] = (uint32_t)x;
+            c = x >> 32;
+        }
+    }
+    // W = t[8..17] = (S + q p) / R < 2^288 + p:  W = lo + hi 2^256,  hi 2^256 = mont_mul(hi, R^2)
+    fe lo, hi = fe_zero();
+#pragma unroll
+    for (int i = 0; i < 8; ++i) lo.l[i] = t[8 + i];
+    hi.l[0] = t[16];
+    hi.l[1] = t[17];
+    return fe_add(fe_reduce_256(lo), mont_mul(hi, fe_const(2)));
+}
+
+// BZK_UNRED (d >= 2): the last product of every summed point goes into a 544-bit accumulator
+// (mul_acc) and is reduced once per thread, instead of two pairs sharing one reduction (eval_two).
+#ifndef BZK_UNRED
+#define BZK_UNRED 1
+#endif
+template <int D> struct UseUnred { static constexpr bool v = BZK_UNRED && D >= 2; };
+
+// one pair at the summed points (same point sets and lazy bounds as eval_two)
+template <int D, bool DERIVE>
+__device__ __forceinline__ void eval_one(const fe (&a)[D], const fe (&s)[D], acc17 (&acc)[Pts<D, DERIVE>::NV]) {
+    constexpr int NV = Pts<D, DERIVE>::NV;
+    fe v[D], dl[D];
+#pragma unroll
+    for (int idx = 0; idx < NV; ++idx) {
+        const int t = point_t<D, DERIVE>(idx);
+        if ((t < 0 || t == 2) && !DERIVE) {   // round 1: delta = b - a on demand
+#pragma unroll
+            for (int m = 0; m < D; ++m) {
+                dl[m] = lz_sub(s[m], a[m]);
+                if (!(D == 2 && m == 0)) dl[m] = lz_red(dl[m]);
+            }
+        }
+        const fe *x;
+        if (t == 0) x = a;
+        else if (t == 1) x = s;                                    // FIRST only: s = b
+        else if (t < 0) x = DERIVE ? s : dl;
+        else {
+#pragma unroll
+            for (int m = 0; m < D; ++m) {
+                const fe &d1 = DERIVE ? s[m] : dl[m];
+                if (t == 2) {
+                    v[m] = lz_red(lz_add(DERIVE ? a[m] : s[m], d1));
+                    if (DERIVE) v[m] = lz_red(lz_add(v[m], d1));
+                } else {
+                    v[m] = lz_red(lz_add(v[m], d1));
+                }
+            }
+            x = v;
+        }
+        fe p = x[0];
+#pragma unroll
+        for (int m = 1; m < D - 1; ++m) p = mont_mul_lz(p, x[m]);
+        mul_acc(acc[idx], p, x[D - 1]);
+    }
+}
+
 // single pair, every point t = 0..D (used by the on-chip tail)
 template <int D>
 __device__ __forceinline__ void eval_pair(const fe (&a)[D], const fe (&b)[D], fe (&acc)[D + 1]) {
@@ -202,6 +284,20 @@ __device__ __forceinline__ fe fold1(const fe &a, const fe &b, const fe &rmont) {
 __device__ __forceinline__ fe fold_lz(const fe &a, const fe &b, const fe &rmont) {
     return lz_red(lz_add(a, mont_mul_lz(rmont, lz_sub(b, a))));
 }
+
+// the same fold through the fixed-multiplier table K of r (field.cuh fixmul_lz; K in shared memory)
+__device__ __forceinline__ fe fold_fx(const fe &a, const fe &b, const fe *K, uint32_t zmask) {
+    return lz_red(lz_add(a, fixmul_lz(lz_sub(b, a), K, zmask)));
+}
+
+#ifndef BZK_FIXMUL
+#define BZK_FIXMUL 1   // 1: fused-round folds use the per-(proof, round) table K_i = r 2^(32i+64)
+#endif
+#if BZK_FIXMUL
+#define BZK_FOLD(a, b) fold_fx(a, b, sK, zmask)
+#else
+#define BZK_FOLD(a, b) fold_lz(a, b, rm)
+#endif
 
 // ---------------------------------------------------------------- per-round finalisation
 
@@ -331,6 +427,12 @@ static __global__ void k_init_consts(fe *c) {
     } else if (t < 25) {
         c[kConstInvW + t] = fe_zero();
     }
+    if (t < 8) {   // 2^(32 t + 64) mod p by doubling
+        fe v = fe_zero();
+        v.l[0] = 1;
+        for (int e = 0; e < 32 * t + 64; ++e) v = fe_add(v, v);
+        c[kConstPow2 + t] = v;
+    }
 }
 
 struct Seed32 { uint8_t b[32]; };
@@ -349,7 +451,7 @@ static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed3
 
 template <int D, int ORDER, bool FIRST>
 __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, uint64_t j, const fe &rm,
-                                          fe (&a)[D], fe (&sv)[D]) {
+                                          const fe *sK, uint32_t zmask, fe (&a)[D], fe (&sv)[D]) {
 #pragma unroll
     for (int m = 0; m < D; ++m) {
         fe lo, hi;
@@ -363,16 +465,16 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
             if (ORDER == 0) {
                 fe x0 = ld_fe_stream(T + 4 * j), x1 = ld_fe_stream(T + 4 * j + 1);
                 fe x2 = ld_fe_stream(T + 4 * j + 2), x3 = ld_fe_stream(T + 4 * j + 3);
-                lo = fold_lz(x0, x1, rm);
-                hi = fold_lz(x2, x3, rm);
+                lo = BZK_FOLD(x0, x1);
+                hi = BZK_FOLD(x2, x3);
                 st_fe(U + 2 * j, lo);
                 st_fe(U + 2 * j + 1, hi);
             } else {
                 // previous round paired (x, x + 2h); this round pairs (j, j + h)
                 fe x0 = ld_fe_stream(T + j), x1 = ld_fe_stream(T + j + 2 * h);
                 fe x2 = ld_fe_stream(T + j + h), x3 = ld_fe_stream(T + j + 3 * h);
-                lo = fold_lz(x0, x1, rm);
-                hi = fold_lz(x2, x3, rm);
+                lo = BZK_FOLD(x0, x1);
+                hi = BZK_FOLD(x2, x3);
                 st_fe(U + j, lo);
                 st_fe(U + j + h, hi);
             }
@@ -522,6 +624,11 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     const fe *src = P.src + (size_t)b * D * (FIRST ? 2 * h : 4 * h);
     fe *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const fe rm = FIRST ? fe_zero() : P.ps[b].rmont;
+    __shared__ __align__(16) fe sK[8];   // fixed-multiplier table of r_{i-1} (fused rounds)
+    if (!FIRST && BZK_FIXMUL) {
+        if (threadIdx.x < 8) sK[threadIdx.x] = mont_mul(rm, P.consts[kConstPow2 + threadIdx.x]);   // r 2^(32t+64)
+        __syncthreads();
+    }
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     const uint32_t lane = threadIdx.x & 31;
 #ifdef BZK_STAGGER_NS
@@ -564,13 +671,25 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     // One pair per loop iteration (keeps the loop body -- 2d folds + one two-pair evaluation -- small
     // enough for the instruction cache); every second pair is held in registers and evaluated
     // together with the next one, so the two pairs' products share one Montgomery reduction.
-    {
+    if constexpr (UseUnred<D>::v) {
+        acc17 uacc[NV];
+#pragma unroll
+        for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
+        for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
+            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
+            fe a[D], sv[D];
+            load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
+            eval_one<D, DERIVE>(a, sv, uacc);
+        }
+#pragma unroll
+        for (int t = 0; t < NV; ++t) { wacc[t].lo = acc17_to_fe(uacc[t]); wacc[t].hi = 0; }
+    } else {
         fe ha[D], hs[D];
         bool held = false;
         for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
             if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
             fe a[D], sv[D];
-            load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, a, sv);
+            load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
             if (held) {
                 eval_two<D, DERIVE>(ha, hs, a, sv, wacc);
             } else {
