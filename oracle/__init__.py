@@ -52,6 +52,12 @@ def lib():
         L.orc_mu.argtypes = [u64p]
         L.orc_gl_prove.argtypes = [u32, u32, u32, u8p, u64, u64p, u64p, u64p, u64p, u64p, u64p]
         L.orc_gl_op.argtypes = [ctypes.c_int, u64, u64p, u64p, u64p]
+        vp = ctypes.c_void_p
+        L.orc_sha256_compress.argtypes = [vp, vp, vp]
+        L.orc_merkle.argtypes = [u32, ctypes.c_int, vp, vp, vp]
+        L.orc_merkle_batch.argtypes = [u32, ctypes.c_int, u64, vp, vp, vp, ctypes.c_int]
+        L.orc_merkle_path.argtypes = [u32, vp, u64, vp]
+        L.orc_merkle_verify_path.argtypes = [u32, ctypes.c_int, vp, u64, vp, vp]
         _lib = L
     return _lib
 
@@ -210,3 +216,69 @@ def gl_op(op: str, a: np.ndarray, b: np.ndarray) -> np.ndarray:
     out = np.zeros_like(a)
     lib().orc_gl_op(code, a.shape[0], _p(a), _p(b), _p(out))
     return out
+
+
+# ---------------------------------------------------------------- Merkle trees (NEXT-3, readings R17-R19)
+
+MERKLE_COMPRESS = 0   # H = one SHA-256 compression of the 512-bit block from the FIPS IV
+MERKLE_FIPS = 1       # H = FIPS 180-4 SHA-256 of the 64-byte message
+
+
+def _u8(a: np.ndarray):
+    assert a.dtype == np.uint8 and a.flags["C_CONTIGUOUS"]
+    return a.ctypes.data
+
+
+def sha256_compress(state, block: bytes):
+    """One SHA-256 compression: state = 8 uint32 words, block = 64 bytes -> 8 words."""
+    h = np.ascontiguousarray(np.asarray(state, dtype=np.uint32))
+    b = np.frombuffer(bytes(block), dtype=np.uint8).copy()
+    assert h.shape == (8,) and b.shape == (64,)
+    out = np.zeros(8, np.uint32)
+    lib().orc_sha256_compress(h.ctypes.data, b.ctypes.data, out.ctypes.data)
+    return [int(x) for x in out]
+
+
+def merkle(blocks: np.ndarray, n: int, mode: int = MERKLE_COMPRESS, nodes: bool = True):
+    """One tree: blocks uint8 [2^n][64] -> (root bytes, nodes uint8 [2^(n+1)-1][32] or None)."""
+    blocks = np.ascontiguousarray(blocks, dtype=np.uint8).reshape(-1)
+    assert blocks.size == (64 << n)
+    root = np.zeros(32, np.uint8)
+    nd = np.zeros(((2 << n) - 1) * 32, np.uint8) if nodes else None
+    s = lib().orc_merkle(n, mode, _u8(blocks), None if nd is None else _u8(nd), _u8(root))
+    if s:
+        raise ValueError(f"orc_merkle failed: {s}")
+    return root.tobytes(), (None if nd is None else nd.reshape(-1, 32))
+
+
+def merkle_batch(blocks: np.ndarray, n: int, mode: int = MERKLE_COMPRESS, nodes: bool = False,
+                 nthreads: int | None = None):
+    """Batch: blocks uint8 [B][2^n][64] -> (roots uint8 [B][32], nodes uint8 [B][2^(n+1)-1][32] or None)."""
+    blocks = np.ascontiguousarray(blocks, dtype=np.uint8)
+    B = blocks.shape[0]
+    assert blocks.size == B * (64 << n)
+    roots = np.zeros((B, 32), np.uint8)
+    nd = np.zeros((B, (2 << n) - 1, 32), np.uint8) if nodes else None
+    if nthreads is None:
+        nthreads = min(B, len(os.sched_getaffinity(0))) or 1
+    s = lib().orc_merkle_batch(n, mode, B, _u8(blocks.reshape(-1)), None if nd is None else _u8(nd),
+                               _u8(roots), nthreads)
+    if s:
+        raise ValueError(f"orc_merkle_batch failed: {s}")
+    return roots, nd
+
+
+def merkle_path(nodes: np.ndarray, n: int, x: int) -> np.ndarray:
+    nodes = np.ascontiguousarray(nodes, dtype=np.uint8)
+    path = np.zeros((max(n, 1), 32), np.uint8)
+    lib().orc_merkle_path(n, _u8(nodes), x, _u8(path))
+    return path[:n]
+
+
+def merkle_verify_path(n: int, mode: int, block: bytes, x: int, path: np.ndarray, root: bytes) -> bool:
+    b = np.frombuffer(bytes(block), dtype=np.uint8).copy()
+    p = np.ascontiguousarray(path, dtype=np.uint8).reshape(-1)
+    if p.size == 0:
+        p = np.zeros(32, np.uint8)
+    r = np.frombuffer(bytes(root), dtype=np.uint8).copy()
+    return bool(lib().orc_merkle_verify_path(n, mode, _u8(b), x, _u8(p), _u8(r)))

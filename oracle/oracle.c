@@ -28,6 +28,11 @@
  *                   plain definition (independent of folding).
  *   orc_hsum     -- H = sum_{x in {0,1}^k} prod_m T_m[x].
  *   orc_sha256   -- FIPS 180-4 SHA-256 (the paper's hash).
+ *   orc_merkle   -- Merkle tree of N = 2^n 512-bit blocks, level by level as
+ *                   P:91-97 (Sec. 2.2, Fig. 2) describes it; H = one SHA-256
+ *                   compression of the block (reading R18) or full
+ *                   FIPS SHA-256; orc_merkle_path / orc_merkle_verify_path
+ *                   open and check one leaf ("efficient verifiability").
  *
  * Pins (tests/test_oracle_*.py, -m "not gpu"): Python exact integers for the
  * field, FIPS 180-4 vectors + hashlib for SHA-256, brute-force hypercube sums,
@@ -712,4 +717,126 @@ int orc_gl_op(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t
         }
     }
     return ORC_OK;
+}
+
+/* ------------------------------------------------------------------ */
+/* Merkle trees (readings R17-R19)       */
+/*   P:91-97 Sec. 2.2 Fig. 2: "divides input data into multiple blocks  */
+/*   and then hashes each block to create the leaf node ... iteratively */
+/*   combines pairs of these hash values ... until only one hash value  */
+/*   remains at the top, known as the Merkle root".                     */
+/*   P:137 Sec. 3.1: N 512-bit blocks, log N rounds; 2N hashes.  */
+/* Hash H of a 512-bit block (reading R18):                             */
+/*   mode 0 (paper-literal, "produces a fixed-size 256-bit hash    */
+/*     value from a 512-bit block"): one SHA-256 compression of the     */
+/*     block from the FIPS 180-4 initial value, digest = the 8 state    */
+/*     words big-endian;                                                */
+/*   mode 1: the full FIPS 180-4 SHA-256 of the 64-byte message.        */
+/* Nodes, level-major (reading R19): level 0 = N leaf digests           */
+/* H(block_x); level l+1 [j] = H(level_l[2j] || level_l[2j+1]); the     */
+/* root is level n [0]; 2N-1 digests per tree.                          */
+/* ------------------------------------------------------------------ */
+
+/* one compression from an arbitrary state (exposed for the pins)     */
+void orc_sha256_compress(const uint32_t h_in[8], const uint8_t blk[64], uint32_t h_out[8]) {
+    uint32_t h[8];
+    memcpy(h, h_in, sizeof h);
+    sha256_block(h, blk);
+    memcpy(h_out, h, sizeof h);
+}
+
+static void merkle_hash(const uint8_t blk[64], int mode, uint8_t out[32]) {
+    if (mode == 1) { orc_sha256(blk, 64, out); return; }
+    static const uint32_t IV[8] = {0x6a09e667, 0xbb67ae85, 0x3c6ef372, 0xa54ff53a,
+                                   0x510e527f, 0x9b05688c, 0x1f83d9ab, 0x5be0cd19};
+    uint32_t h[8];
+    memcpy(h, IV, sizeof h);
+    sha256_block(h, blk);
+    for (int i = 0; i < 8; ++i) {
+        out[4 * i] = (uint8_t)(h[i] >> 24); out[4 * i + 1] = (uint8_t)(h[i] >> 16);
+        out[4 * i + 2] = (uint8_t)(h[i] >> 8); out[4 * i + 3] = (uint8_t)h[i];
+    }
+}
+
+/* One tree of N = 2^n blocks (64 bytes each).  nodes: (2N-1) x 32 bytes, level-major, or NULL.
+ * root: 32 bytes.  Level by level exactly as P:97 describes it. */
+int orc_merkle(uint32_t n, int mode, const uint8_t *blocks, uint8_t *nodes, uint8_t root[32]) {
+    if (n > 24 || (mode != 0 && mode != 1)) return 1;
+    const uint64_t N = (uint64_t)1 << n;
+    uint8_t *lv = (uint8_t *)malloc((size_t)(2 * N - 1) * 32);
+    if (!lv) return 2;
+    /* level 0: leaf digests */
+    for (uint64_t x = 0; x < N; ++x) merkle_hash(blocks + 64 * x, mode, lv + 32 * x);
+    /* level l+1 from level l: the concatenation of two adjacent digests is a 512-bit block */
+    uint64_t off = 0, cnt = N;
+    while (cnt > 1) {
+        uint8_t *cur = lv + 32 * off, *nxt = lv + 32 * (off + cnt);
+        for (uint64_t j = 0; j < cnt / 2; ++j) {
+            uint8_t blk[64];
+            memcpy(blk, cur + 64 * j, 32);
+            memcpy(blk + 32, cur + 64 * j + 32, 32);
+            merkle_hash(blk, mode, nxt + 32 * j);
+        }
+        off += cnt;
+        cnt /= 2;
+    }
+    memcpy(root, lv + 32 * off, 32);
+    if (nodes) memcpy(nodes, lv, (size_t)(2 * N - 1) * 32);
+    free(lv);
+    return 0;
+}
+
+/* Authentication path of block x (siblings from the leaf level up, n x 32 bytes), read from a
+ * level-major node array, and its check: recompute the root from the block and the path. */
+int orc_merkle_path(uint32_t n, const uint8_t *nodes, uint64_t x, uint8_t *path) {
+    uint64_t off = 0, cnt = (uint64_t)1 << n;
+    for (uint32_t l = 0; l < n; ++l) {
+        memcpy(path + 32 * l, nodes + 32 * (off + (x ^ 1)), 32);
+        off += cnt; cnt /= 2; x /= 2;
+    }
+    return 0;
+}
+
+int orc_merkle_verify_path(uint32_t n, int mode, const uint8_t blk[64], uint64_t x, const uint8_t *path,
+                           const uint8_t root[32]) {
+    uint8_t cur[32], buf[64];
+    merkle_hash(blk, mode, cur);
+    for (uint32_t l = 0; l < n; ++l) {
+        if (x & 1) { memcpy(buf, path + 32 * l, 32); memcpy(buf + 32, cur, 32); }
+        else       { memcpy(buf, cur, 32); memcpy(buf + 32, path + 32 * l, 32); }
+        merkle_hash(buf, mode, cur);
+        x /= 2;
+    }
+    return memcmp(cur, root, 32) == 0;
+}
+
+typedef struct {
+    uint32_t n; int mode; uint64_t batch; const uint8_t *blocks; uint8_t *nodes, *roots;
+    uint64_t next; pthread_mutex_t lock; int status;
+} merkle_job;
+
+static void *merkle_worker(void *arg) {
+    merkle_job *j = (merkle_job *)arg;
+    const uint64_t N = (uint64_t)1 << j->n;
+    for (;;) {
+        pthread_mutex_lock(&j->lock);
+        uint64_t b = j->next++;
+        pthread_mutex_unlock(&j->lock);
+        if (b >= j->batch) break;
+        int s = orc_merkle(j->n, j->mode, j->blocks + b * N * 64,
+                           j->nodes ? j->nodes + b * (2 * N - 1) * 32 : NULL, j->roots + b * 32);
+        if (s) { pthread_mutex_lock(&j->lock); j->status = s; pthread_mutex_unlock(&j->lock); }
+    }
+    return NULL;
+}
+
+int orc_merkle_batch(uint32_t n, int mode, uint64_t batch, const uint8_t *blocks, uint8_t *nodes,
+                     uint8_t *roots, int nthreads) {
+    if (nthreads < 1) nthreads = 1;
+    merkle_job j = {n, mode, batch, blocks, nodes, roots, 0, PTHREAD_MUTEX_INITIALIZER, 0};
+    pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)nthreads);
+    for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, merkle_worker, &j);
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    free(th);
+    return j.status;
 }

@@ -45,4 +45,16 @@ static __global__ void k_generate(uint64_t *dst, uint64_t batch, uint32_t d, uin
     }
 }
 
+// Merkle blocks (inputs.py gen_blocks): dst [batch][2^n][64] bytes = 8 LE64 words per block,
+// word w of block x of tree I = splitmix64((I << 36) | (x << 3) | w).  One thread per word.
+static __global__ void k_generate_blocks(uint64_t *dst, uint64_t batch, uint32_t n, uint64_t first_index,
+                                         uint64_t seed) {
+    const uint64_t words = batch << (n + 3);
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < words;
+         e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t xw = e & ((8ull << n) - 1), b = e >> (n + 3);
+        dst[e] = splitmix64_ctr(((first_index + b) << 36) | xw, seed);
+    }
+}
+
 }  // namespace bzk

@@ -79,3 +79,22 @@ def gen_tables(batch: int, d: int, k: int, first_index: int = 0, dist: str | int
                 words[:, 3] &= MASK61
                 out[bi, m] = words
     return out
+
+
+# ---------------------------------------------------------------- Merkle blocks (NEXT-3)
+# ctr(I, x, w) = (I << 36) | (x << 3) | w   (I < 2^28, x < 2^33, w < 8); a block is the 8 words
+# LE64-serialised, 64 bytes.  Device twin: gen.cuh k_generate_blocks (bzk_generate_blocks).
+MERKLE_DATA_SEED = 0x42415443485A4B4D   # "BATCHZKM"
+
+
+def gen_blocks(batch: int, n: int, first_index: int = 0, data_seed: int = MERKLE_DATA_SEED) -> np.ndarray:
+    """uint8 [B][2^n][64] Merkle input blocks for global tree indices first_index.."""
+    N = 1 << n
+    out = np.empty((batch, N, 8), dtype=np.uint64)
+    x = np.arange(N, dtype=np.uint64)
+    w = np.arange(8, dtype=np.uint64)
+    for bi in range(batch):
+        I = np.uint64(first_index + bi)
+        ctr = (I << np.uint64(36)) | (x[:, None] << np.uint64(3)) | w[None, :]
+        out[bi] = splitmix64(ctr, data_seed)
+    return out.astype("<u8").view(np.uint8).reshape(batch, N, 64)
