@@ -45,6 +45,11 @@ CONFIGS = {
                                          "k=20, MSB = Alg. 1 pairing, challenges given (no Fiat-Shamir, P:111)"),
     "g2": (1024, 2, 20, 0, "gl", "NEXT-2 second field instance: 1024 proofs x product of 2 multilinears, k=20, "
                                  "Goldilocks p = 2^64 - 2^32 + 1 (8-byte elements: the HBM-bound regime)"),
+    "mk20": (256, 0, 20, 0, "blocks", "NEXT-3 batched Merkle trees: 256 trees x 2^20 512-bit blocks (64 MiB per tree, "
+                                     "P:295 Table 3 shape), H = one SHA-256 compression per block (P:97), every "
+                                     "node level written to HBM"),
+    "mk20f": (256, 1, 20, 0, "blocks", "NEXT-3 batched Merkle trees: 256 trees x 2^20 512-bit blocks, H = FIPS "
+                                       "SHA-256 of the 64-byte block (two compressions), every node level written"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -152,6 +157,15 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+MERKLE_METRIC = "Merkle trees/s @2^20 512-bit blocks (NEXT-3, P:295 Table 3 shape)"
+# ALU-pipe roof of one SHA-256 compression: the rotations/shifts (SHF) and the
+# 3-input logic (LOP3) can only issue to the ALU pipe (B300_MICROARCH.md: IADD3/LOP3/SHF/PRMT on the
+# alu pipe, rt_SMSP = 2 -> 64 lanes/clk/SM); the additions may go to the FMA pipe.  Per compression:
+# 64 rounds x (6 SHF + 4 LOP3) + 48 schedule steps x (6 SHF + 2 LOP3) = 1024 ALU-only instructions.
+ALU_PER_CLK_SM = 64
+ALU_OPS_PER_COMPRESSION = 64 * 10 + 48 * 8
+
+
 def cpu_baseline(cfg, max_proofs=8):
     """The oracle as it stands on this box's host cores: a bounded sample of the same workload."""
     import numpy as np  # noqa: F401
@@ -162,6 +176,14 @@ def cpu_baseline(cfg, max_proofs=8):
     cores = len(os.sched_getaffinity(0))
     n = max(1, min(max_proofs, cores, B))
     oracle.build()
+    if dist == "blocks":
+        blocks = inputs.gen_blocks(n, k, 0)
+        t0 = time.perf_counter()
+        oracle.merkle_batch(blocks, k, d, nodes=True, nthreads=n)
+        dt = time.perf_counter() - t0
+        return {"value": n / dt, "unit": "trees/s", "cores": n, "kind": "oracle",
+                "sample": f"{n} trees of {cfg} (2^{k} blocks, hash mode {d}), one per thread, {dt:.1f} s wall "
+                          f"= {n * dt:.0f} CPU-seconds"}
     if dist == "gl":
         import concurrent.futures as cf
         tabs = inputs.gen_tables_gl(n, d, k, 0)
@@ -193,13 +215,15 @@ def run_reference(args, rank, world):
         times.append(cb["cores"] / cb["value"])
     nproofs = cb["cores"]
     value = nproofs * len(times) / sum(times)
-    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "proofs/s", "n_gpus": args.gpus,
+    unit = cb["unit"]
+    line = {"impl": "reference", "metric": MERKLE_METRIC if dist == "blocks" else METRIC, "value": value,
+            "unit": unit, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * sum(times) / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
             "data": "synthetic", "config": {"workload": desc, "batch_sampled": nproofs, "d": d, "k": k},
-            "cpu_baseline": {"value": value, "unit": "proofs/s", "cores": nproofs, "kind": "oracle",
+            "cpu_baseline": {"value": value, "unit": unit, "cores": nproofs, "kind": "oracle",
                              "sample": cb["sample"]},
-            "e2e": {"value": value, "unit": "proofs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
@@ -298,6 +322,131 @@ def run_vml(args, rank, world):
     prover.close()
 
 
+def run_merkle(args, rank, world):
+    """NEXT-3: batched Merkle trees (bzk_merkle).  A step builds every tree of the batch: all 2N - 1
+    hashes per tree, every node level written to HBM (the tree is what a prover opens later)."""
+    import torch
+
+    from paper_conf_asplos_lucw0cz25_b200 import bzk
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if os.environ.get("BZK_BENCH_DEVICE") is not None:
+        local = int(os.environ["BZK_BENCH_DEVICE"])
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    B, mode, n, _, _, desc = CONFIGS[args.config]
+    if args.batch:
+        B = args.batch
+    first, _ = shard.weak_range(B, rank)
+    N = 1 << n
+    stream = torch.cuda.Stream()
+    blocks = torch.empty((B, N, 64), dtype=torch.uint8, device="cuda")
+    bzk.bzk_generate_blocks(blocks, B, n, first, stream=stream)
+    roots = torch.empty((B, 32), dtype=torch.uint8, device="cuda")
+    nodes = torch.empty((B, 2 * N - 1, 32), dtype=torch.uint8, device="cuda")
+    mb = bzk.MerkleBuilder(local)
+    batch = mb.batch(blocks, n, mode, roots, nodes)
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        bzk.bzk_merkle(mb.ctx, batch, stream)
+    stream.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    bzk.bzk_launch_count(mb.ctx, reset=True)
+    barrier()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            bzk.bzk_merkle(mb.ctx, batch, stream)
+            ev[i][1].record(stream)
+        stream.synchronize()
+        barrier()
+    launches = bzk.bzk_launch_count(mb.ctx, reset=True)
+    my_ms = float(sum(a.elapsed_time(b) for a, b in ev))
+    # per-stage device time (roofline of the dominant stage kernel), outside the headline region
+    bzk.bzk_profile_enable(mb.ctx, True)
+    bzk.bzk_profile_read(mb.ctx, reset=True)
+    for _ in range(args.steps):
+        bzk.bzk_merkle(mb.ctx, batch, stream)
+    prof = bzk.bzk_profile_read(mb.ctx, reset=True)
+    bzk.bzk_profile_enable(mb.ctx, False)
+    digest = shard.output_digest([roots.cpu()])
+    max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
+    digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
+    ms_per_step = max_ms / args.steps
+    value = B * world * args.steps / (max_ms / 1000.0)
+    hbm_peak, sm_max_mhz, peak_src = peaks()
+    comps_per_tree = (2 * N - 1) * (2 if mode == 1 else 1)
+    stage_ms, stage_cnt = prof["merkle_stage"]
+    launches_per_step = max(1, stage_cnt // args.steps)
+    # the dominant launch is stage 0 (all but 2^-10 of the hashes); its share of the step's compressions
+    # is (2N - 1 - top) / (2N - 1); report the step as the conservative whole-step roof fraction
+    achieved = B * comps_per_tree / (stage_ms / args.steps / 1000.0) / 1e9
+    peak = SMS * ALU_PER_CLK_SM * sm_max_mhz * 1e6 / ALU_OPS_PER_COMPRESSION / 1e9
+    bytes_step = B * (N * 64 + (2 * N - 1) * 32 + 32)
+    line = {"metric": MERKLE_METRIC, "value": round(value, 2), "unit": "trees/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": desc, "trees_per_gpu": B, "global_trees": B * world, "log_blocks": n,
+                       "hash": "sha256-compress" if mode == 0 else "sha256-fips",
+                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * N * 64 / 2**30)},
+            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
+            "kernel_ms_per_step": {"merkle_stages": round(stage_ms / args.steps, 3),
+                                   "launches_per_step": launches_per_step},
+            "roofline": {"bound": "alu", "kernel": "k_merkle_stage (all stages of a step)",
+                         "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "Gcompress/s",
+                         "frac": round(achieved / peak, 4), "traffic": None,
+                         "alg_compressions_per_step": B * comps_per_tree,
+                         "peak_source": f"guide unit counts: {SMS} SMs x {ALU_PER_CLK_SM} ALU lanes/clk x "
+                                        f"{sm_max_mhz:.0f} MHz ({peak_src} max clock) / "
+                                        f"{ALU_OPS_PER_COMPRESSION} ALU-only instructions per SHA-256 compression",
+                         "hbm_alg_frac": round(bytes_step / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
+                         "hbm_peak_gbs": hbm_peak},
+            "clocks": clk.summary(), "digest_rank0": digests[0], "digests_per_rank": len(digests),
+            "context": "paper Table 3 (P:251-261): 6.536 trees/ms at 2^20 on GH200 as printed (unit garbled; "
+                       "DESIGN.md R20)"}
+    if not args.no_e2e:
+        # e2e: pinned host blocks in, host roots + node arrays out, through bzk_merkle's loader
+        Be = max(1, min(B, 32))
+        host_b = blocks[:Be].cpu().pin_memory()
+        hr = torch.empty((Be, 32), dtype=torch.uint8, pin_memory=True)
+        hn = torch.empty((Be, 2 * N - 1, 32), dtype=torch.uint8, pin_memory=True)
+        hb = mb.batch(host_b, n, mode, hr, hn)
+        bzk.bzk_merkle(mb.ctx, hb, stream)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            bzk.bzk_merkle(mb.ctx, hb, stream)
+        e1.record(stream)
+        stream.synchronize()
+        e2e_ms = shard.max_over_ranks(e0.elapsed_time(e1), dist, device="cuda")
+        same = torch.equal(hr, roots[:Be].cpu()) and torch.equal(hn[-1], nodes[Be - 1].cpu())
+        line["e2e"] = {"value": round(Be * world * args.e2e_steps / (e2e_ms / 1000.0), 2), "unit": "trees/s",
+                       "trees_per_gpu": Be, "h2d_bytes_per_step": int(host_b.numel()),
+                       "d2h_bytes_per_step": int(hr.numel() + hn.numel()), "steps": args.e2e_steps,
+                       "matches_device_run": bool(same),
+                       "path": "bzk_merkle(blocks_mem=HOST pinned, outputs_mem=HOST): H2D waves and D2H of node "
+                               "levels on two side streams overlapping compute (P:145-147)"}
+    if rank == 0 and world == 1 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(args.config)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    mb.close()
+    if dist:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -326,6 +475,9 @@ def main():
         return
     if args.config == "c4":
         run_vml(args, rank, world)
+        return
+    if CONFIGS[args.config][4] == "blocks":
+        run_merkle(args, rank, world)
         return
 
     import numpy as np

@@ -25,12 +25,15 @@ BZK_ORDER_LSB, BZK_ORDER_MSB = 0, 1
 BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
 BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
 BZK_F_FIELD_GOLDILOCKS = 32
-BZK_PROF_KINDS = 6
-PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy"]
+BZK_PROF_KINDS = 8
+PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy",
+                   "merkle_stage", "d2h_copy"]
+BZK_MERKLE_COMPRESS, BZK_MERKLE_SHA256 = 0, 1
 
 EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
            "bzk_strerror", "bzk_last_error", "bzk_generate", "bzk_profile_enable", "bzk_profile_read",
-           "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version"]
+           "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version",
+           "bzk_merkle", "bzk_generate_blocks"]
 
 
 class BzkError(RuntimeError):
@@ -45,6 +48,13 @@ class bzk_batch(ctypes.Structure):
                 ("seed", ctypes.c_void_p), ("tables", ctypes.c_void_p), ("tables_mem", ctypes.c_uint32),
                 ("outputs_mem", ctypes.c_uint32), ("round_evals", ctypes.c_void_p),
                 ("challenges", ctypes.c_void_p), ("final_evals", ctypes.c_void_p), ("claims", ctypes.c_void_p)]
+
+
+class bzk_merkle_batch(ctypes.Structure):
+    _fields_ = [("log_blocks", ctypes.c_uint32), ("hash", ctypes.c_uint32), ("flags", ctypes.c_uint32),
+                ("blocks_mem", ctypes.c_uint32), ("batch", ctypes.c_uint64), ("blocks", ctypes.c_void_p),
+                ("outputs_mem", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("roots", ctypes.c_void_p),
+                ("nodes", ctypes.c_void_p)]
 
 
 _lib = None
@@ -79,9 +89,11 @@ def lib():
         L.bzk_debug_sha256.argtypes = [vp, u32, u64, vp, vp]
         L.bzk_debug_bench.argtypes = [i32, u32, ctypes.POINTER(ctypes.c_double), vp]
         L.bzk_version.restype = ctypes.c_char_p
+        L.bzk_merkle.argtypes = [vp, ctypes.POINTER(bzk_merkle_batch), vp]
+        L.bzk_generate_blocks.argtypes = [vp, u64, u32, u64, u64, vp]
         for name in ("bzk_create", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
                      "bzk_generate", "bzk_profile_enable", "bzk_profile_read", "bzk_debug_field",
-                     "bzk_debug_sha256", "bzk_debug_bench"):
+                     "bzk_debug_sha256", "bzk_debug_bench", "bzk_merkle", "bzk_generate_blocks"):
             getattr(L, name).restype = i32
         _lib = L
     return _lib
@@ -170,6 +182,16 @@ def bzk_generate(dst, batch, d, k, first_index=0, dist=0, data_seed=None, stream
         dist = DISTS[dist]
     _check(lib().bzk_generate(ptr(dst), batch, d, k, first_index, dist,
                               DATA_SEED if data_seed is None else data_seed, _stream_handle(stream)))
+
+
+def bzk_merkle(ctx, b: bzk_merkle_batch, stream=None) -> None:
+    _check(lib().bzk_merkle(ctx, ctypes.byref(b), _stream_handle(stream)), ctx)
+
+
+def bzk_generate_blocks(dst, batch, n, first_index=0, data_seed=None, stream=None) -> None:
+    from .inputs import MERKLE_DATA_SEED
+    _check(lib().bzk_generate_blocks(ptr(dst), batch, n, first_index,
+                                     MERKLE_DATA_SEED if data_seed is None else data_seed, _stream_handle(stream)))
 
 
 def bzk_profile_enable(ctx, on: bool) -> None:
@@ -274,3 +296,48 @@ class Prover:
 
     def sync(self):
         bzk_sync(self.ctx)
+
+
+class MerkleBuilder:
+    """Owns a bzk context; builds batches of Merkle trees held in torch tensors (device or pinned host).
+
+    blocks: uint8 tensor [B][2^n][64].  Returns (roots uint8 [B][32], nodes uint8 [B][2^(n+1)-1][32] or None).
+    """
+
+    def __init__(self, device: int = 0, workspace_limit: int = 0, ctx=None):
+        self.device = device
+        self._own = ctx is None
+        self.ctx = bzk_create(device, workspace_limit) if ctx is None else ctx
+
+    def close(self):
+        if self.ctx and self._own:
+            bzk_destroy(self.ctx)
+        self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    @staticmethod
+    def batch(blocks, n, hash_mode=BZK_MERKLE_COMPRESS, roots=None, nodes=None, flags=0, batch=None):
+        B = batch if batch is not None else blocks.shape[0]
+        host_in = hasattr(blocks, "is_cuda") and not blocks.is_cuda
+        host_out = hasattr(roots, "is_cuda") and not roots.is_cuda
+        return bzk_merkle_batch(n, hash_mode, flags, BZK_MEM_HOST if host_in else BZK_MEM_DEVICE, B, ptr(blocks),
+                                BZK_MEM_HOST if host_out else BZK_MEM_DEVICE, 0, ptr(roots), ptr(nodes))
+
+    def build(self, blocks, n, hash_mode=BZK_MERKLE_COMPRESS, with_nodes=True, roots=None, nodes=None,
+              flags=0, stream=None):
+        import torch
+        B = blocks.shape[0]
+        dev = "cuda" if blocks.is_cuda else "cpu"
+        pin = dev == "cpu"
+        if roots is None:
+            roots = torch.empty((B, 32), dtype=torch.uint8, device=dev, pin_memory=pin)
+        if with_nodes and nodes is None:
+            nodes = torch.empty((B, (2 << n) - 1, 32), dtype=torch.uint8, device=dev, pin_memory=pin)
+        b = self.batch(blocks, n, hash_mode, roots, nodes if with_nodes else None, flags)
+        bzk_merkle(self.ctx, b, stream)
+        return roots, (nodes if with_nodes else None)

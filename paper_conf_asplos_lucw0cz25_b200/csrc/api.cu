@@ -17,6 +17,7 @@
 #include "field_f64.cuh"
 #include "gl.cuh"
 #include "gen.cuh"
+#include "merkle.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
 
@@ -41,6 +42,10 @@ struct bzk_ctx {
     cudaStream_t copy_stream = nullptr;
     cudaEvent_t ev_copied[2] = {nullptr, nullptr};
     cudaEvent_t ev_consumed[2] = {nullptr, nullptr};
+    // Merkle loader (NEXT-3): device->host stream for node levels, per-slot events
+    cudaStream_t d2h_stream = nullptr;
+    cudaEvent_t ev_nodes_ready[2] = {nullptr, nullptr};
+    cudaEvent_t ev_nodes_copied[2] = {nullptr, nullptr};
     // loader ring: two device staging slots for host tables, reused across waves, jobs and calls
     void *stage[2] = {nullptr, nullptr};
     size_t stage_size = 0;
@@ -592,6 +597,186 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
     return BZK_OK;
 }
 
+
+// ---------------------------------------------------------------- Merkle trees (NEXT-3)
+//
+// Plan: a chain of stage launches (merkle.cuh).  Stage s hashes M_s 64-byte blocks per tree (the
+// input blocks for s = 0, pairs of level-(lvl0_s - 1) digests after that); each thread covers 2^lt
+// blocks and produces one digest of level lvl0_s + lt.  Host blocks stream through the loader ring
+// in waves (H2D on copy_stream); host node arrays stream back per wave on d2h_stream while the next
+// wave computes ("dynamic loading and storing", multi-stream).
+
+struct MkStage { uint32_t lt, lg_tpt, lvl0; };
+
+// blocks per thread = 2^lt (BZK_MK_LT, default 3: tuned on B200)
+uint32_t mk_lt_max() {
+    static uint32_t v = [] {
+        const char *e = getenv("BZK_MK_LT");
+        return e ? (uint32_t)std::max(0, std::min(4, atoi(e))) : 3u;
+    }();
+    return v;
+}
+
+std::vector<MkStage> merkle_stages(uint32_t n) {
+    std::vector<MkStage> v;
+    uint32_t lgM = n, lvl0 = 0;
+    for (;;) {
+        MkStage st;
+        st.lt = std::min(mk_lt_max(), lgM);
+        st.lg_tpt = lgM - st.lt;
+        st.lvl0 = lvl0;
+        v.push_back(st);
+        if (st.lg_tpt == 0) break;
+        lvl0 = lvl0 + st.lt + 1;     // the next stage's leaf hashes are H(pair of thread roots)
+        lgM = st.lg_tpt - 1;
+    }
+    return v;
+}
+
+bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) {
+    if (!m) return fail(ctx, BZK_EINVAL, "batch is NULL");
+    if (m->log_blocks > 30) return fail(ctx, BZK_EINVAL, "log_blocks must be <= 30");
+    if (m->hash > 1) return fail(ctx, BZK_EINVAL, "hash must be BZK_MERKLE_COMPRESS or BZK_MERKLE_SHA256");
+    if (m->batch == 0) return fail(ctx, BZK_EINVAL, "batch must be >= 1");
+    if (!m->blocks || !m->roots) return fail(ctx, BZK_EINVAL, "blocks/roots is NULL");
+    if (m->blocks_mem > 1 || m->outputs_mem > 1) return fail(ctx, BZK_EINVAL, "bad *_mem value");
+    auto mis = [](const void *q) { return q && ((uintptr_t)q & 31u); };
+    if ((m->blocks_mem == BZK_MEM_DEVICE && mis(m->blocks)) ||
+        (m->outputs_mem == BZK_MEM_DEVICE && (mis(m->roots) || mis(m->nodes))))
+        return fail(ctx, BZK_EINVAL, "device buffers must be 32-byte aligned");
+    const uint32_t n = m->log_blocks;
+    const uint64_t N = 1ull << n, B = m->batch;
+    const size_t blk_bytes = (size_t)N * 64, nodes_bytes = (size_t)(2 * N - 1) * 32;
+    const bool host_in = m->blocks_mem == BZK_MEM_HOST, host_out = m->outputs_mem == BZK_MEM_HOST;
+    const bool want_nodes = m->nodes != nullptr;
+    const std::vector<MkStage> stages = merkle_stages(n);
+    // scratch for CTA roots between stages when the node array is not kept on the device
+    const bool dev_nodes = want_nodes;   // host_out stages the node array per wave on the device
+    const size_t scratch_pt = dev_nodes ? 0 : (size_t)32 << stages[0].lg_tpt;
+
+    size_t limit = ctx->workspace_limit;
+    if (limit == 0) {
+        if (ctx->auto_limit == 0) {
+            size_t fr = 0, tot = 0;
+            cudaMemGetInfo(&fr, &tot);
+            fr += ctx->ws_size + 2 * ctx->stage_size;
+            ctx->auto_limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
+        }
+        limit = ctx->auto_limit;
+    }
+    auto per_tree = [&]() {
+        size_t t = 2 * scratch_pt;
+        if (host_in) t += 2 * blk_bytes;
+        if (host_out && want_nodes) t += 2 * nodes_bytes;
+        return t;
+    };
+    const size_t fixed = 4096 + (host_out ? align_up(B * 32) : 0);
+    uint64_t bw = B;
+    if ((host_in || host_out) && B >= 8 && B * (blk_bytes + nodes_bytes) > (1ull << 30)) bw = (B + 7) / 8;
+    while (bw > 1 && fixed + per_tree() * bw + 1024 > limit) bw = (bw + 1) / 2;
+    if (fixed + per_tree() * bw + 1024 > limit) return fail(ctx, BZK_ENOMEM, "workspace_limit too small for one tree");
+    const uint64_t nw = (B + bw - 1) / bw;
+    bw = (B + nw - 1) / nw;
+
+    size_t off = 0;
+    const size_t off_roots = off; if (host_out) off = align_up(off + B * 32);
+    const size_t off_scr = off; off = align_up(off + 2 * bw * scratch_pt);
+    const size_t off_nodes = off; if (host_out && want_nodes) off = align_up(off + 2 * bw * nodes_bytes);
+    bzk_status st = ensure_ws(ctx, std::max<size_t>(off, 256));
+    if (st) return st;
+    st = ensure_stage(ctx, host_in ? align_up(bw * blk_bytes) : 0);
+    if (st) return st;
+    char *ws = (char *)ctx->ws;
+    uint8_t *roots_all = host_out ? (uint8_t *)(ws + off_roots) : m->roots;
+
+    bool nslot_used[2] = {false, false};
+    for (uint64_t w = 0; w < nw; ++w) {
+        const uint64_t b0 = w * bw, nb = std::min<uint64_t>(bw, B - b0);
+        const uint8_t *blocks;
+        int slot = -1;
+        if (host_in) {
+            slot = ctx->next_slot;
+            ctx->next_slot ^= 1;
+            if (ctx->slot_used[slot]) CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
+            {
+                ProfScope ps_(ctx, ctx->copy_stream, 5);
+                CK(cudaMemcpyAsync(ctx->stage[slot], m->blocks + b0 * blk_bytes, nb * blk_bytes,
+                                   cudaMemcpyHostToDevice, ctx->copy_stream));
+            }
+            CK(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
+            CK(cudaStreamWaitEvent(s, ctx->ev_copied[slot], 0));
+            blocks = (const uint8_t *)ctx->stage[slot];
+        } else {
+            blocks = m->blocks + b0 * blk_bytes;
+        }
+        uint8_t *nodes = nullptr;
+        const int ns = (int)(w & 1);
+        if (want_nodes) {
+            if (host_out) {
+                nodes = (uint8_t *)(ws + off_nodes) + (size_t)ns * bw * nodes_bytes;
+                if (nslot_used[ns]) CK(cudaStreamWaitEvent(s, ctx->ev_nodes_copied[ns], 0));
+            } else {
+                nodes = m->nodes + b0 * nodes_bytes;
+            }
+        }
+        uint8_t *scr[2] = {(uint8_t *)(ws + off_scr), (uint8_t *)(ws + off_scr) + bw * scratch_pt};
+        const uint8_t *in = blocks;
+        uint64_t in_stride = blk_bytes;
+        for (size_t si = 0; si < stages.size(); ++si) {
+            const MkStage &g = stages[si];
+            const bool last = si + 1 == stages.size();
+            mk::StageParams p;
+            p.in = in; p.in_stride = in_stride;
+            p.nodes = nodes; p.nodes_stride = nodes_bytes;
+            p.n = n; p.lvl0 = g.lvl0; p.lg_tpt = g.lg_tpt;
+            p.threads = nb << g.lg_tpt;
+            const uint32_t top = g.lvl0 + g.lt;      // level of the thread roots
+            if (last) { p.out = roots_all + b0 * 32; p.out_stride = 32; }
+            else if (dev_nodes) { p.out = nullptr; p.out_stride = 0; }
+            else { p.out = scr[si & 1]; p.out_stride = (uint64_t)32 << g.lg_tpt; }
+            const uint32_t tpb = 256;
+            const uint64_t grid = (p.threads + tpb - 1) / tpb;
+            if (grid > 0x7fffffffull) return fail(ctx, BZK_EINVAL, "too many CTAs in one stage launch");
+            {
+                ProfScope ps_(ctx, s, 6);
+                cudaError_t e = merkle_launch_stage(m->hash, g.lt, (uint32_t)grid, tpb, s, p);
+                ++ctx->launches;
+                if (e != cudaSuccess) return cuda_fail(ctx, e, "k_merkle_stage");
+            }
+            if (!last) {
+                if (dev_nodes) {
+                    in = nodes + (((2ull << n) - (2ull << (n - top))) * 32);
+                    in_stride = nodes_bytes;
+                } else {
+                    in = p.out;
+                    in_stride = p.out_stride;
+                }
+            }
+        }
+        if (slot >= 0) {
+            CK(cudaEventRecord(ctx->ev_consumed[slot], s));
+            ctx->slot_used[slot] = true;
+        }
+        if (want_nodes && host_out) {
+            CK(cudaEventRecord(ctx->ev_nodes_ready[ns], s));
+            CK(cudaStreamWaitEvent(ctx->d2h_stream, ctx->ev_nodes_ready[ns], 0));
+            {
+                ProfScope ps_(ctx, ctx->d2h_stream, 7);
+                CK(cudaMemcpyAsync(m->nodes + b0 * nodes_bytes, nodes, nb * nodes_bytes, cudaMemcpyDeviceToHost,
+                                   ctx->d2h_stream));
+            }
+            CK(cudaEventRecord(ctx->ev_nodes_copied[ns], ctx->d2h_stream));
+            nslot_used[ns] = true;
+        }
+    }
+    if (host_out) {
+        CK(cudaMemcpyAsync(m->roots, roots_all, B * 32, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(ctx->d2h_stream));
+    }
+    if (host_in || host_out || (m->flags & BZK_F_SYNC)) CK(cudaStreamSynchronize(s));
+    return BZK_OK;
+}
+
 // ---------------------------------------------------------------- debug kernels
 
 __global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *out) {
@@ -741,7 +926,7 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
 
 extern "C" {
 
-const char *bzk_version(void) { return "bzk 0.1 sm_100a (BN254 Fr, SHA-256 Fiat-Shamir)"; }
+const char *bzk_version(void) { return "bzk 0.2 sm_100a (BN254 Fr + Goldilocks sum-check, SHA-256 Fiat-Shamir, batched Merkle trees)"; }
 
 const char *bzk_strerror(bzk_status s) {
     switch (s) {
@@ -789,6 +974,12 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
     for (int i = 0; i < 2; ++i) {
         cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming);
         cudaEventCreateWithFlags(&ctx->ev_consumed[i], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&ctx->ev_nodes_ready[i], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&ctx->ev_nodes_copied[i], cudaEventDisableTiming);
+    }
+    if (cudaStreamCreateWithFlags(&ctx->d2h_stream, cudaStreamNonBlocking) != cudaSuccess) {
+        delete ctx;
+        return BZK_ECUDA;
     }
     *out = ctx;
     return BZK_OK;
@@ -806,7 +997,10 @@ void bzk_destroy(bzk_ctx *ctx) {
     for (int i = 0; i < 2; ++i) {
         if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
         if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
+        if (ctx->ev_nodes_ready[i]) cudaEventDestroy(ctx->ev_nodes_ready[i]);
+        if (ctx->ev_nodes_copied[i]) cudaEventDestroy(ctx->ev_nodes_copied[i]);
     }
+    if (ctx->d2h_stream) cudaStreamDestroy(ctx->d2h_stream);
     if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
     for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
     for (auto e : ctx->ev_pool) cudaEventDestroy(e);
@@ -852,6 +1046,20 @@ bzk_status bzk_generate(uint64_t *dst, uint64_t batch, uint32_t d, uint32_t k, u
                         uint32_t dist, uint64_t data_seed, void *cuda_stream) {
     if (!dst || k > 30 || d < 1 || d > 15 || dist > 3 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
     k_generate<<<kSMs * 16, 256, 0, (cudaStream_t)cuda_stream>>>(dst, batch, d, k, first_index, dist, data_seed);
+    return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+}
+
+bzk_status bzk_merkle(bzk_ctx *ctx, const bzk_merkle_batch *batch, void *cuda_stream) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    return merkle_impl(ctx, batch, (cudaStream_t)cuda_stream);
+}
+
+bzk_status bzk_generate_blocks(uint8_t *dst, uint64_t batch, uint32_t n, uint64_t first_index, uint64_t data_seed,
+                               void *cuda_stream) {
+    if (!dst || n > 30 || batch == 0 || first_index + batch > (1ull << 28) || ((uintptr_t)dst & 7u)) return BZK_EINVAL;
+    k_generate_blocks<<<kSMs * 16, 256, 0, (cudaStream_t)cuda_stream>>>((uint64_t *)dst, batch, n, first_index,
+                                                                       data_seed);
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }
 
