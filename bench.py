@@ -343,6 +343,9 @@ def run_merkle(args, rank, world):
     B, mode, n, _, _, desc = CONFIGS[args.config]
     if args.batch:
         B = args.batch
+    if args.log_blocks is not None:
+        n = args.log_blocks
+        desc = desc.replace("2^20", "2^%d" % n)
     first, _ = shard.weak_range(B, rank)
     N = 1 << n
     stream = torch.cuda.Stream()
@@ -394,6 +397,16 @@ def run_merkle(args, rank, world):
     achieved = B * comps_per_tree / (stage_ms / args.steps / 1000.0) / 1e9
     peak = SMS * ALU_PER_CLK_SM * sm_max_mhz * 1e6 / ALU_OPS_PER_COMPRESSION / 1e9
     bytes_step = B * (N * 64 + (2 * N - 1) * 32 + 32)
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic_merkle.json")
+    if os.path.exists(tpath) and n == 20:
+        # DRAM bytes of the dominant launch (stage 0) from one `ncu --set full` capture, scaled to B trees
+        with open(tpath) as f:
+            tj = json.load(f)
+        if tj.get("config") == args.config:
+            traffic = {"stage0_dram_bytes": int(tj["dram_bytes_per_launch"] * B / tj["batch"]),
+                       "stage0_alg_bytes": int(tj["algorithmic_bytes_per_launch"] * B / tj["batch"]),
+                       "source": tj["source"]}
     line = {"metric": MERKLE_METRIC, "value": round(value, 2), "unit": "trees/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
@@ -405,7 +418,7 @@ def run_merkle(args, rank, world):
                                    "launches_per_step": launches_per_step},
             "roofline": {"bound": "alu", "kernel": "k_merkle_stage (all stages of a step)",
                          "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "Gcompress/s",
-                         "frac": round(achieved / peak, 4), "traffic": None,
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
                          "alg_compressions_per_step": B * comps_per_tree,
                          "peak_source": f"guide unit counts: {SMS} SMs x {ALU_PER_CLK_SM} ALU lanes/clk x "
                                         f"{sm_max_mhz:.0f} MHz ({peak_src} max clock) / "
@@ -454,7 +467,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--batch", type=int, default=None, help="override proofs per GPU")
+    ap.add_argument("--batch", type=int, default=None, help="override proofs (trees) per GPU")
+    ap.add_argument("--log-blocks", type=int, default=None, help="Merkle configs: override n (2^n blocks per tree)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
