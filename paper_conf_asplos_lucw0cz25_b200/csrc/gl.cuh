@@ -107,6 +107,61 @@ __device__ __forceinline__ void eval_pair(const uint64_t (&a)[D], const uint64_t
     }
 }
 
+// Lazy evaluation sums (GL_LAZY, default on): the last product of every point is accumulated
+// unreduced into a 192-bit accumulator (lo, hi, top) and reduced once per thread, instead of a
+// 128 -> 64-bit reduction plus a canonical addition per product (the round kernels were ALU-bound
+// on those, ncu r01).  2^128 = -2^32 (mod p), so top * C128 folds the third word back.
+#ifndef GL_LAZY
+#define GL_LAZY 1
+#endif
+constexpr uint64_t C128 = 0xfffffffe00000001ull;   // 2^128 mod p
+
+struct Wide { uint64_t lo, hi, top; };
+
+__device__ __forceinline__ void wide_mac(Wide &A, uint64_t x, uint64_t y) {
+    const uint64_t lo = x * y, hi = __umul64hi(x, y);
+    asm("add.cc.u64 %0, %0, %3;\n\taddc.cc.u64 %1, %1, %4;\n\taddc.u64 %2, %2, 0;"
+        : "+l"(A.lo), "+l"(A.hi), "+l"(A.top)
+        : "l"(lo), "l"(hi));
+}
+
+__device__ __forceinline__ uint64_t wide_reduce(const Wide &A) {   // top < 2^32 (fewer than 2^32 products)
+    return add(reduce128(A.hi, A.lo), mul(A.top, C128));
+}
+
+// x + y reduced only to 64 bits (congruent mod p, not necessarily canonical): a multiplication
+// input needs no more
+__device__ __forceinline__ uint64_t add_lazy(uint64_t x, uint64_t y) {
+    const uint64_t s = x + y;
+    return s < x ? s + EPS : s;       // x + y - 2^64 + (2^64 mod p) < 2^64
+}
+
+template <int D>
+__device__ __forceinline__ void eval_pair(const uint64_t (&a)[D], const uint64_t (&b)[D], Wide (&acc)[D + 1]) {
+    uint64_t v[D], dl[D];
+#pragma unroll
+    for (int m = 0; m < D; ++m) { v[m] = a[m]; dl[m] = sub(b[m], a[m]); }
+#pragma unroll
+    for (int t = 0; t <= D; ++t) {
+        // v_m = a_m + t (b_m - a_m): t = 1 is b_m itself; later points are lazy sums (< 2^64)
+        if (t == 1) {
+#pragma unroll
+            for (int m = 0; m < D; ++m) v[m] = b[m];
+        } else if (t > 1) {
+#pragma unroll
+            for (int m = 0; m < D; ++m) v[m] = add_lazy(v[m], dl[m]);
+        }
+        if (D == 1) {
+            wide_mac(acc[t], v[0], 1ull);
+        } else {
+            uint64_t prod = v[0];
+#pragma unroll
+            for (int m = 1; m + 1 < D; ++m) prod = mul(prod, v[m]);
+            wide_mac(acc[t], prod, v[D - 1]);
+        }
+    }
+}
+
 __device__ __forceinline__ uint64_t fold(uint64_t a, uint64_t b, uint64_t r) { return add(a, mul(r, sub(b, a))); }
 
 // transcript round over LE64 evaluations; r_i = LE64(state_i[0..8]) mod p  (reading R15)
@@ -198,27 +253,43 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
     const uint64_t h = 1ull << P.log_h;
+#if GL_LAZY
+    Wide wacc[D + 1];
+#pragma unroll
+    for (int t = 0; t <= D; ++t) wacc[t] = Wide{0, 0, 0};
+#define GL_ACC wacc
+#else
     uint64_t acc[D + 1];
 #pragma unroll
     for (int t = 0; t <= D; ++t) acc[t] = 0;
+#define GL_ACC acc
+#endif
     const uint64_t *src = P.src + (size_t)b * D * (FIRST ? 2 * h : 4 * h);
     uint64_t *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const uint64_t r = FIRST ? 0 : P.ps[b].r;
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    // GL_MLP pairs in flight per iteration (memory-level parallelism: the kernel streams)
-    for (; j + (GL_MLP - 1) * stride < h; j += GL_MLP * stride) {
-        uint64_t a[GL_MLP][D], bb[GL_MLP][D];
+    // MLP pairs in flight per iteration (memory-level parallelism: the kernel streams); fewer for
+    // d >= 3, whose wider accumulators would otherwise spill
+    constexpr int MLP = D <= 2 ? GL_MLP : (GL_MLP > 2 ? 2 : GL_MLP);
+    for (; j + (MLP - 1) * stride < h; j += MLP * stride) {
+        uint64_t a[MLP][D], bb[MLP][D];
 #pragma unroll
-        for (int q = 0; q < GL_MLP; ++q) load_pair<D, ORDER, FIRST>(src, dst, h, j + q * stride, r, a[q], bb[q]);
+        for (int q = 0; q < MLP; ++q) load_pair<D, ORDER, FIRST>(src, dst, h, j + q * stride, r, a[q], bb[q]);
 #pragma unroll
-        for (int q = 0; q < GL_MLP; ++q) eval_pair<D>(a[q], bb[q], acc);
+        for (int q = 0; q < MLP; ++q) eval_pair<D>(a[q], bb[q], GL_ACC);
     }
     for (; j < h; j += stride) {
         uint64_t a0[D], b0[D];
         load_pair<D, ORDER, FIRST>(src, dst, h, j, r, a0, b0);
-        eval_pair<D>(a0, b0, acc);
+        eval_pair<D>(a0, b0, GL_ACC);
     }
+#undef GL_ACC
+#if GL_LAZY
+    uint64_t acc[D + 1];
+#pragma unroll
+    for (int t = 0; t <= D; ++t) acc[t] = wide_reduce(wacc[t]);
+#endif
     block_reduce<D + 1>(acc, s_red);
     uint64_t *evals = P.round_evals + (size_t)b * P.k * (D + 1);
     uint64_t *chals = P.challenges + (size_t)b * P.k;
