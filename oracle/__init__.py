@@ -58,6 +58,8 @@ def lib():
         L.orc_merkle_batch.argtypes = [u32, ctypes.c_int, u64, vp, vp, vp, ctypes.c_int]
         L.orc_merkle_path.argtypes = [u32, vp, u64, vp]
         L.orc_merkle_verify_path.argtypes = [u32, ctypes.c_int, vp, u64, vp, vp]
+        L.orc_encode.argtypes = [u32, u32, vp, vp, vp, vp, vp]
+        L.orc_encode_batch.argtypes = [u32, u32, vp, vp, vp, u64, vp, vp, ctypes.c_int]
         _lib = L
     return _lib
 
@@ -282,3 +284,54 @@ def merkle_verify_path(n: int, mode: int, block: bytes, x: int, path: np.ndarray
         p = np.zeros(32, np.uint8)
     r = np.frombuffer(bytes(root), dtype=np.uint8).copy()
     return bool(lib().orc_merkle_verify_path(n, mode, _u8(b), x, _u8(p), _u8(r)))
+
+
+# ---------------------------------------------------------------- linear-time encoder (NEXT-4, readings R21-R24)
+
+class _Csr(ctypes.Structure):
+    _fields_ = [("rows", ctypes.c_uint32), ("cols", ctypes.c_uint32), ("row_ptr", ctypes.c_void_p),
+                ("col", ctypes.c_void_p), ("val", ctypes.c_void_p)]
+
+
+def _csr(m: dict) -> _Csr:
+    for k_ in ("row_ptr", "col", "val"):
+        assert m[k_].flags["C_CONTIGUOUS"]
+    return _Csr(m["rows"], m["cols"], m["row_ptr"].ctypes.data, m["col"].ctypes.data, m["val"].ctypes.data)
+
+
+def _code_args(code: dict):
+    L = code["levels"]
+    A = (_Csr * max(1, L))(*[_csr(a) for a in code["A"]])
+    B = (_Csr * max(1, L))(*[_csr(b) for b in code["B"]])
+    G0 = _csr(code["G0"])
+    return A, B, G0
+
+
+def encode(code: dict, msg: np.ndarray) -> np.ndarray:
+    """One message [n][4] (canonical) -> codeword [2n][4] (oracle/oracle.c orc_encode)."""
+    msg = np.ascontiguousarray(msg, dtype=np.uint64)
+    n = 1 << code["log_n"]
+    assert msg.shape == (n, 4)
+    out = np.zeros((2 * n, 4), np.uint64)
+    A, B, G0 = _code_args(code)
+    s = lib().orc_encode(code["log_n"], code["levels"], ctypes.addressof(A), ctypes.addressof(B),
+                         ctypes.addressof(G0), msg.ctypes.data, out.ctypes.data)
+    if s:
+        raise ValueError(f"orc_encode failed: {s}")
+    return out
+
+
+def encode_batch(code: dict, msgs: np.ndarray, nthreads: int | None = None) -> np.ndarray:
+    msgs = np.ascontiguousarray(msgs, dtype=np.uint64)
+    Bn = msgs.shape[0]
+    n = 1 << code["log_n"]
+    assert msgs.shape == (Bn, n, 4)
+    out = np.zeros((Bn, 2 * n, 4), np.uint64)
+    if nthreads is None:
+        nthreads = min(Bn, len(os.sched_getaffinity(0))) or 1
+    A, B, G0 = _code_args(code)
+    s = lib().orc_encode_batch(code["log_n"], code["levels"], ctypes.addressof(A), ctypes.addressof(B),
+                               ctypes.addressof(G0), Bn, msgs.ctypes.data, out.ctypes.data, nthreads)
+    if s:
+        raise ValueError(f"orc_encode_batch failed: {s}")
+    return out

@@ -33,6 +33,8 @@
  *                   compression of the block (reading R18) or full
  *                   FIPS SHA-256; orc_merkle_path / orc_merkle_verify_path
  *                   open and check one leaf ("efficient verifiability").
+ *   orc_encode   -- Spielman-style linear-time encoder, recursively as P:113-117
+ *                   (Sec. 2.4, Fig. 3) describes it; graphs are inputs (R21-R24).
  *
  * Pins (tests/test_oracle_*.py, -m "not gpu"): Python exact integers for the
  * field, FIPS 180-4 vectors + hashlib for SHA-256, brute-force hypercube sums,
@@ -836,6 +838,97 @@ int orc_merkle_batch(uint32_t n, int mode, uint64_t batch, const uint8_t *blocks
     merkle_job j = {n, mode, batch, blocks, nodes, roots, 0, PTHREAD_MUTEX_INITIALIZER, 0};
     pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)nthreads);
     for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, merkle_worker, &j);
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    free(th);
+    return j.status;
+}
+
+/* ------------------------------------------------------------------ */
+/* Linear-time (Spielman-style) encoder (readings   */
+/* R21-R24).  P:113-117 Sec. 2.4, Fig. 3: each stage         */
+/* multiplies its input by the first bipartite graph's sparse matrix,    */
+/* encodes the result recursively ("forwarded to the subsequent stage"), */
+/* multiplies the returned vector by the second graph's matrix; "the     */
+/* result, combined with the input vector and the vector returned from   */
+/* the subsequent stage, forms the output of this stage".  Rows = right  */
+/* vertices, columns = left vertices.  Written recursively,      */
+/* exactly in that order (the GPU path is iterative).         */
+/*   Enc_l(x), |x| = n_l:  l == L: x || G0 x  (base code)                */
+/*                         else    y = A_l x; z = Enc_{l+1}(y);          */
+/*                                 w = B_l z; return x || z || w         */
+/* ------------------------------------------------------------------ */
+
+typedef struct { uint32_t rows, cols; const uint32_t *row_ptr, *col; const uint64_t *val; } orc_csr;
+
+/* y[r] = sum over the row's edges (r, j) of val * x[j]  (plain: fr_mul, fr_add per edge) */
+static void csr_apply(const orc_csr *M, const fr *x, fr *y) {
+    for (uint32_t r = 0; r < M->rows; ++r) {
+        fr acc = fr_zero();
+        for (uint32_t e = M->row_ptr[r]; e < M->row_ptr[r + 1]; ++e) {
+            fr w; memcpy(w.v, M->val + 4 * (uint64_t)e, 32);
+            acc = fr_add(acc, fr_mul(w, x[M->col[e]]));
+        }
+        y[r] = acc;
+    }
+}
+
+static int enc_rec(uint32_t l, uint32_t levels, const orc_csr *A, const orc_csr *B, const orc_csr *G0,
+                   const fr *x, uint64_t n, fr *out) {
+    memcpy(out, x, n * sizeof(fr));                    /* the input vector is part of the output */
+    if (l == levels) {                                 /* base code: x || G0 x */
+        if (G0->cols != n || G0->rows != n) return 1;
+        csr_apply(G0, x, out + n);
+        return 0;
+    }
+    if (A[l].cols != n || A[l].rows != n / 4 || B[l].cols != n / 2 || B[l].rows != n / 2) return 1;
+    fr *y = (fr *)malloc((n / 4) * sizeof(fr));
+    if (!y) return 2;
+    csr_apply(&A[l], x, y);                            /* first vector-matrix multiplication */
+    int s = enc_rec(l + 1, levels, A, B, G0, y, n / 4, out + n);   /* z = Enc(y), length n/2 */
+    free(y);
+    if (s) return s;
+    csr_apply(&B[l], out + n, out + n + n / 2);        /* second: w = B z */
+    return 0;
+}
+
+/* msg: n = 2^log_n canonical elements [n][4]; out: codeword [2n][4] = x || z || w */
+int orc_encode(uint32_t log_n, uint32_t levels, const orc_csr *A, const orc_csr *B, const orc_csr *G0,
+               const uint64_t *msg, uint64_t *out) {
+    ensure_mu();
+    const uint64_t n = (uint64_t)1 << log_n;
+    for (uint64_t i = 0; i < n; ++i) {
+        fr t; memcpy(t.v, msg + 4 * i, 32);
+        if (!fr_is_canon(&t)) return 3;
+    }
+    return enc_rec(0, levels, A, B, G0, (const fr *)msg, n, (fr *)out);
+}
+
+typedef struct {
+    uint32_t log_n, levels; const orc_csr *A, *B, *G0; uint64_t batch; const uint64_t *msgs; uint64_t *out;
+    uint64_t next; pthread_mutex_t lock; int status;
+} enc_job;
+
+static void *enc_worker(void *arg) {
+    enc_job *j = (enc_job *)arg;
+    const uint64_t n = (uint64_t)1 << j->log_n;
+    for (;;) {
+        pthread_mutex_lock(&j->lock);
+        uint64_t b = j->next++;
+        pthread_mutex_unlock(&j->lock);
+        if (b >= j->batch) break;
+        int s = orc_encode(j->log_n, j->levels, j->A, j->B, j->G0, j->msgs + b * n * 4, j->out + b * 2 * n * 4);
+        if (s) { pthread_mutex_lock(&j->lock); j->status = s; pthread_mutex_unlock(&j->lock); }
+    }
+    return NULL;
+}
+
+int orc_encode_batch(uint32_t log_n, uint32_t levels, const orc_csr *A, const orc_csr *B, const orc_csr *G0,
+                     uint64_t batch, const uint64_t *msgs, uint64_t *out, int nthreads) {
+    if (nthreads < 1) nthreads = 1;
+    ensure_mu();
+    enc_job j = {log_n, levels, A, B, G0, batch, msgs, out, 0, PTHREAD_MUTEX_INITIALIZER, 0};
+    pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)nthreads);
+    for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, enc_worker, &j);
     for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
     free(th);
     return j.status;

@@ -98,3 +98,75 @@ def gen_blocks(batch: int, n: int, first_index: int = 0, data_seed: int = MERKLE
         ctr = (I << np.uint64(36)) | (x[:, None] << np.uint64(3)) | w[None, :]
         out[bi] = splitmix64(ctr, data_seed)
     return out.astype("<u8").view(np.uint8).reshape(batch, N, 64)
+
+
+# ---------------------------------------------------------------- linear-time encoder graphs (NEXT-4)
+# The Spielman-style code's random bipartite graphs are INPUTS of the method (the random draws are
+# passed in, readings R21-R24).  Counter: ctr = ((((l << 2 | mat) << 24 | j) << 8 | t) << 3) | w
+# for level l < 16, matrix mat (0 = A_l, 1 = B_l, 2 = base G0), left vertex j < 2^24, edge t < 256,
+# word w (0..3 weight limbs, 4 = row pick).  Left-regular graphs: every left vertex (input) picks
+# `deg` distinct right vertices (rows); a duplicate pick moves to the next row (mod rows).
+# Weights: uniform < 2^253, limb 0 | 1 (nonzero).  Rows = right vertices.
+ENC_DATA_SEED = 0x42415443485A4B45     # "BATCHZKE"
+ENC_C, ENC_D = 10, 20                  # left degrees of A_l and B_l (reading R22)
+
+
+def enc_levels(log_n: int, log_n0: int) -> int:
+    """Recursion depth L: level l encodes n_l = n / 4^l elements; the base code takes n_L <= n0."""
+    L = 0
+    while log_n - 2 * L > log_n0:
+        L += 1
+    return L
+
+
+def _enc_ctr(l, mat, j, t, w):
+    j = np.asarray(j, dtype=np.uint64)
+    t = np.asarray(t, dtype=np.uint64)
+    return (((((np.uint64(l) << np.uint64(2) | np.uint64(mat)) << np.uint64(24) | j) << np.uint64(8) | t)
+             << np.uint64(3)) | np.uint64(w))
+
+
+def _left_regular_csr(l, mat, cols, rows, deg, seed):
+    j = np.arange(cols, dtype=np.uint64)[:, None]
+    t = np.arange(deg, dtype=np.uint64)[None, :]
+    r = (splitmix64(_enc_ctr(l, mat, j, t, 4), seed) % np.uint64(rows)).astype(np.int64)
+    for q in range(1, deg):
+        dup = (r[:, :q] == r[:, q:q + 1]).any(axis=1)
+        while dup.any():
+            r[dup, q] = (r[dup, q] + 1) % rows
+            dup = (r[:, :q] == r[:, q:q + 1]).any(axis=1)
+    w = np.stack([splitmix64(_enc_ctr(l, mat, j, t, k), seed) for k in range(4)], axis=-1)
+    w[..., 3] &= MASK61
+    w[..., 0] |= np.uint64(1)
+    rr = r.reshape(-1)
+    cc = np.repeat(np.arange(cols, dtype=np.int64), deg)
+    order = np.lexsort((cc, rr))
+    row_ptr = np.zeros(rows + 1, dtype=np.uint32)
+    np.cumsum(np.bincount(rr, minlength=rows), out=row_ptr[1:])
+    return {"rows": rows, "cols": cols, "row_ptr": row_ptr, "col": cc[order].astype(np.uint32),
+            "val": np.ascontiguousarray(w.reshape(-1, 4)[order])}
+
+
+def _dense_csr(l, m, seed):
+    i = np.arange(m, dtype=np.uint64)[:, None]
+    jj = np.arange(m, dtype=np.uint64)[None, :]
+    idx = i * np.uint64(m) + jj
+    w = np.stack([splitmix64(_enc_ctr(l, 2, idx, 0, k), seed) for k in range(4)], axis=-1)
+    w[..., 3] &= MASK61
+    w[..., 0] |= np.uint64(1)
+    return {"rows": m, "cols": m, "row_ptr": (np.arange(m + 1, dtype=np.uint32) * np.uint32(m)),
+            "col": np.tile(np.arange(m, dtype=np.uint32), m), "val": np.ascontiguousarray(w.reshape(-1, 4))}
+
+
+def gen_code(log_n: int, log_n0: int = 6, c: int = ENC_C, d: int = ENC_D, seed: int = ENC_DATA_SEED) -> dict:
+    """Graphs of the code for messages of n = 2^log_n elements: per level l < L, A_l (n_l/4 rows x n_l
+    cols, left degree c) and B_l (n_l/2 x n_l/2, left degree d); the base G0 (m x m dense, m = n_L)."""
+    assert 6 <= log_n0 and log_n <= 24
+    L = enc_levels(log_n, log_n0)
+    A, B = [], []
+    for l in range(L):
+        nl = 1 << (log_n - 2 * l)
+        A.append(_left_regular_csr(l, 0, nl, nl // 4, c, seed))
+        B.append(_left_regular_csr(l, 1, nl // 2, nl // 2, d, seed))
+    m = 1 << (log_n - 2 * L)
+    return {"log_n": log_n, "log_n0": log_n0, "levels": L, "A": A, "B": B, "G0": _dense_csr(L, m, seed), "m": m}
