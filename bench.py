@@ -50,6 +50,8 @@ CONFIGS = {
                                      "node level written to HBM"),
     "mk20f": (256, 1, 20, 0, "blocks", "NEXT-3 batched Merkle trees: 256 trees x 2^20 512-bit blocks, H = FIPS "
                                        "SHA-256 of the 64-byte block (two compressions), every node level written"),
+    "enc20": (256, 0, 20, 0, "code", "NEXT-4 linear-time encoder: 256 messages x 2^20 BN254 Fr elements (P:320 Table 5 "
+                                     "shape), Spielman-style rate-1/2 code, left degrees 10/20, base 64 (readings R21-R24)"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -166,6 +168,17 @@ ALU_PER_CLK_SM = 64
 ALU_OPS_PER_COMPRESSION = 64 * 10 + 48 * 8
 
 
+ENC_METRIC = "linear-time encodings/s @2^20 BN254 Fr elements (NEXT-4, P:320 Table 5 shape)"
+# IMAD roof of an edge product: a 256 x 256-bit product accumulated unreduced = 64 IMAD.WIDE = 128 IMAD
+# slots (the Montgomery reduction is amortised over a whole row: one per output element)
+IMAD_PER_EDGE_PRODUCT = 128
+
+
+def enc_edges(code) -> int:
+    return sum(int(a["row_ptr"][-1]) for a in code["A"]) + sum(int(b["row_ptr"][-1]) for b in code["B"]) + \
+        int(code["G0"]["row_ptr"][-1])
+
+
 def cpu_baseline(cfg, max_proofs=8):
     """The oracle as it stands on this box's host cores: a bounded sample of the same workload."""
     import numpy as np  # noqa: F401
@@ -176,6 +189,15 @@ def cpu_baseline(cfg, max_proofs=8):
     cores = len(os.sched_getaffinity(0))
     n = max(1, min(max_proofs, cores, B))
     oracle.build()
+    if dist == "code":
+        code = inputs.gen_code(k, 6)
+        ms = inputs.gen_tables(n, 1, k, 0)[:, 0]
+        t0 = time.perf_counter()
+        oracle.encode_batch(code, ms, nthreads=n)
+        dt = time.perf_counter() - t0
+        return {"value": n / dt, "unit": "codes/s", "cores": n, "kind": "oracle",
+                "sample": f"{n} codewords of {cfg} (2^{k} elements), one per thread, {dt:.1f} s wall "
+                          f"= {n * dt:.0f} CPU-seconds"}
     if dist == "blocks":
         blocks = inputs.gen_blocks(n, k, 0)
         t0 = time.perf_counter()
@@ -216,7 +238,8 @@ def run_reference(args, rank, world):
     nproofs = cb["cores"]
     value = nproofs * len(times) / sum(times)
     unit = cb["unit"]
-    line = {"impl": "reference", "metric": MERKLE_METRIC if dist == "blocks" else METRIC, "value": value,
+    metric = {"blocks": MERKLE_METRIC, "code": ENC_METRIC}.get(dist, METRIC)
+    line = {"impl": "reference", "metric": metric, "value": value,
             "unit": unit, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * sum(times) / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
@@ -389,13 +412,16 @@ def run_merkle(args, rank, world):
     ms_per_step = max_ms / args.steps
     value = B * world * args.steps / (max_ms / 1000.0)
     hbm_peak, sm_max_mhz, peak_src = peaks()
-    comps_per_tree = (2 * N - 1) * (2 if mode == 1 else 1)
+    hashes_per_tree = 2 * N - 1
+    # FIPS mode: the second compression of every hash is the constant padding block, whose message
+    # schedule is folded into constants (64 x (6 SHF + 4 LOP3) = 640 ALU-only instructions)
+    alu_per_hash = ALU_OPS_PER_COMPRESSION + (64 * 10 if mode == 1 else 0)
     stage_ms, stage_cnt = prof["merkle_stage"]
     launches_per_step = max(1, stage_cnt // args.steps)
     # the dominant launch is stage 0 (all but 2^-10 of the hashes); its share of the step's compressions
     # is (2N - 1 - top) / (2N - 1); report the step as the conservative whole-step roof fraction
-    achieved = B * comps_per_tree / (stage_ms / args.steps / 1000.0) / 1e9
-    peak = SMS * ALU_PER_CLK_SM * sm_max_mhz * 1e6 / ALU_OPS_PER_COMPRESSION / 1e9
+    achieved = B * hashes_per_tree / (stage_ms / args.steps / 1000.0) / 1e9
+    peak = SMS * ALU_PER_CLK_SM * sm_max_mhz * 1e6 / alu_per_hash / 1e9
     bytes_step = B * (N * 64 + (2 * N - 1) * 32 + 32)
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic_merkle.json")
@@ -417,12 +443,13 @@ def run_merkle(args, rank, world):
             "kernel_ms_per_step": {"merkle_stages": round(stage_ms / args.steps, 3),
                                    "launches_per_step": launches_per_step},
             "roofline": {"bound": "alu", "kernel": "k_merkle_stage (all stages of a step)",
-                         "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "Gcompress/s",
+                         "achieved": round(achieved, 3), "peak": round(peak, 3), "unit": "Ghash/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
-                         "alg_compressions_per_step": B * comps_per_tree,
+                         "alg_hashes_per_step": B * hashes_per_tree, "alu_ops_per_hash": alu_per_hash,
                          "peak_source": f"guide unit counts: {SMS} SMs x {ALU_PER_CLK_SM} ALU lanes/clk x "
                                         f"{sm_max_mhz:.0f} MHz ({peak_src} max clock) / "
-                                        f"{ALU_OPS_PER_COMPRESSION} ALU-only instructions per SHA-256 compression",
+                                        f"{alu_per_hash} ALU-only instructions per hash (SHF + LOP3 of the "
+                                        "SHA-256 compression(s); additions may issue to the FMA pipe)",
                          "hbm_alg_frac": round(bytes_step / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
                          "hbm_peak_gbs": hbm_peak},
             "clocks": clk.summary(), "digest_rank0": digests[0], "digests_per_rank": len(digests),
@@ -460,6 +487,137 @@ def run_merkle(args, rank, world):
         dist.destroy_process_group()
 
 
+def run_encoder(args, rank, world):
+    """NEXT-4: batched linear-time encoding (bzk_encode), in place on [B][2n] codeword buffers."""
+    import torch
+
+    from paper_conf_asplos_lucw0cz25_b200 import bzk, inputs
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if os.environ.get("BZK_BENCH_DEVICE") is not None:
+        local = int(os.environ["BZK_BENCH_DEVICE"])
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    B, _, log_n, _, _, desc = CONFIGS[args.config]
+    if args.batch:
+        B = args.batch
+    if args.log_blocks is not None:
+        log_n = args.log_blocks
+        desc = desc.replace("2^20", "2^%d" % log_n)
+    first, _ = shard.weak_range(B, rank)
+    n = 1 << log_n
+    t_setup = time.perf_counter()
+    code = inputs.gen_code(log_n, 6)
+    enc = bzk.Encoder(code, local)
+    t_setup = time.perf_counter() - t_setup
+    stream = torch.cuda.Stream()
+    msgs = torch.empty((B, 1, n, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(msgs, B, 1, log_n, first, "uniform", stream=stream)
+    stream.synchronize()
+    codes = torch.empty((B, 2 * n, 4), dtype=torch.int64, device="cuda")
+
+    def reset():
+        codes[:, :n].copy_(msgs[:, 0])   # untimed: every step encodes the same messages
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        reset()
+        enc.encode(codes, stream=stream)
+    stream.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    bzk.bzk_launch_count(enc.ctx, reset=True)
+    barrier()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                reset()
+            ev[i][0].record(stream)
+            enc.encode(codes, stream=stream)
+            ev[i][1].record(stream)
+        stream.synchronize()
+        barrier()
+    launches = bzk.bzk_launch_count(enc.ctx, reset=True)
+    my_ms = float(sum(a.elapsed_time(b) for a, b in ev))
+    bzk.bzk_profile_enable(enc.ctx, True)
+    bzk.bzk_profile_read(enc.ctx, reset=True)
+    for _ in range(args.steps):
+        enc.encode(codes, stream=stream)
+    prof = bzk.bzk_profile_read(enc.ctx, reset=True)
+    bzk.bzk_profile_enable(enc.ctx, False)
+    with torch.cuda.stream(stream):
+        reset()
+    enc.encode(codes, stream=stream)
+    stream.synchronize()
+    digest = shard.output_digest([codes[:, :, :].cpu()]) if B * n <= (1 << 24) else \
+        shard.output_digest([codes[:, n:n + 1024].cpu()])
+    max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
+    digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
+    ms_per_step = max_ms / args.steps
+    value = B * world * args.steps / (max_ms / 1000.0)
+    hbm_peak, sm_max_mhz, peak_src = peaks()
+    edges = enc_edges(code)
+    spmv_ms, spmv_cnt = prof["encoder_spmv"]
+    achieved = B * edges / (spmv_ms / args.steps / 1000.0) / 1e9
+    peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6 / IMAD_PER_EDGE_PRODUCT / 1e9
+    wbytes = edges * 36
+    line = {"metric": ENC_METRIC, "value": round(value, 2), "unit": "codes/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": desc, "codes_per_gpu": B, "global_codes": B * world, "log_n": log_n,
+                       "levels": code["levels"], "edges_per_code": edges, "left_degrees": [inputs.ENC_C, inputs.ENC_D],
+                       "l2": "codewords larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * 2 * n * 32 / 2**30),
+                       "setup_s": round(t_setup, 2)},
+            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
+            "kernel_ms_per_step": {"encoder_spmv": round(spmv_ms / args.steps, 3),
+                                   "launches_per_step": spmv_cnt // max(1, args.steps)},
+            "roofline": {"bound": "alu", "kernel": "k_spmv (all products of a step)", "achieved": round(achieved, 2),
+                         "peak": round(peak, 2), "unit": "Gproduct/s", "frac": round(achieved / peak, 4),
+                         "traffic": None, "alg_products_per_step": B * edges,
+                         "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} "
+                                        f"MHz ({peak_src} max clock) / {IMAD_PER_EDGE_PRODUCT} IMAD slots per "
+                                        "256x256-bit edge product (reduction amortised per output element)",
+                         "weights_bytes": wbytes, "hbm_peak_gbs": hbm_peak},
+            "clocks": clk.summary(), "digest_rank0": digests[0], "digests_per_rank": len(digests),
+            "context": "paper Table 5 (P:281-291): 0.726 codes/ms at 2^20 on GH200 as printed (parameters of "
+                       "the paper's code unknown, R22)"}
+    if not args.no_e2e:
+        Be = max(1, min(B, 16))
+        host = torch.empty((Be, 2 * n, 4), dtype=torch.int64, pin_memory=True)
+        host[:, :n].copy_(msgs[:Be, 0])
+        enc.encode(host)
+        same = torch.equal(host, codes[:Be].cpu())
+        barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            enc.encode(host)       # host buffer: H2D of the messages, D2H of the codewords inside
+        torch.cuda.synchronize()
+        wall = time.perf_counter() - t0
+        e2e_s = shard.max_over_ranks(wall * 1000.0, dist, device="cuda") / 1000.0
+        line["e2e"] = {"value": round(Be * world * args.e2e_steps / e2e_s, 2), "unit": "codes/s",
+                       "codes_per_gpu": Be, "h2d_bytes_per_step": int(Be * n * 32),
+                       "d2h_bytes_per_step": int(Be * 2 * n * 32), "steps": args.e2e_steps,
+                       "matches_device_run": bool(same), "timing": "host wall clock around the synchronous call",
+                       "path": "bzk_encode(codes_mem=HOST pinned): message H2D and codeword D2H waves on side "
+                               "streams overlapping the encoding"}
+    if rank == 0 and world == 1 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(args.config, max_proofs=args.ref_proofs)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    enc.close()
+    if dist:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -492,6 +650,9 @@ def main():
         return
     if CONFIGS[args.config][4] == "blocks":
         run_merkle(args, rank, world)
+        return
+    if CONFIGS[args.config][4] == "code":
+        run_encoder(args, rank, world)
         return
 
     import numpy as np

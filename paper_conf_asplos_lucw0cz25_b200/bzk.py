@@ -25,15 +25,15 @@ BZK_ORDER_LSB, BZK_ORDER_MSB = 0, 1
 BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
 BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
 BZK_F_FIELD_GOLDILOCKS = 32
-BZK_PROF_KINDS = 8
+BZK_PROF_KINDS = 9
 PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy",
-                   "merkle_stage", "d2h_copy"]
+                   "merkle_stage", "d2h_copy", "encoder_spmv"]
 BZK_MERKLE_COMPRESS, BZK_MERKLE_SHA256 = 0, 1
 
 EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
            "bzk_strerror", "bzk_last_error", "bzk_generate", "bzk_profile_enable", "bzk_profile_read",
            "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version",
-           "bzk_merkle", "bzk_generate_blocks"]
+           "bzk_merkle", "bzk_generate_blocks", "bzk_encoder_create", "bzk_encoder_destroy", "bzk_encode"]
 
 
 class BzkError(RuntimeError):
@@ -55,6 +55,16 @@ class bzk_merkle_batch(ctypes.Structure):
                 ("blocks_mem", ctypes.c_uint32), ("batch", ctypes.c_uint64), ("blocks", ctypes.c_void_p),
                 ("outputs_mem", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("roots", ctypes.c_void_p),
                 ("nodes", ctypes.c_void_p)]
+
+
+class bzk_csr(ctypes.Structure):
+    _fields_ = [("rows", ctypes.c_uint32), ("cols", ctypes.c_uint32), ("nnz", ctypes.c_uint64),
+                ("row_ptr", ctypes.c_void_p), ("col", ctypes.c_void_p), ("val", ctypes.c_void_p)]
+
+
+class bzk_code(ctypes.Structure):
+    _fields_ = [("log_n", ctypes.c_uint32), ("levels", ctypes.c_uint32), ("A", ctypes.c_void_p),
+                ("B", ctypes.c_void_p), ("G0", ctypes.c_void_p)]
 
 
 _lib = None
@@ -91,9 +101,14 @@ def lib():
         L.bzk_version.restype = ctypes.c_char_p
         L.bzk_merkle.argtypes = [vp, ctypes.POINTER(bzk_merkle_batch), vp]
         L.bzk_generate_blocks.argtypes = [vp, u64, u32, u64, u64, vp]
+        L.bzk_encoder_create.argtypes = [vp, ctypes.POINTER(bzk_code), ctypes.POINTER(vp)]
+        L.bzk_encoder_destroy.argtypes = [vp]
+        L.bzk_encoder_destroy.restype = None
+        L.bzk_encode.argtypes = [vp, vp, vp, u64, u32, u32, vp]
         for name in ("bzk_create", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
                      "bzk_generate", "bzk_profile_enable", "bzk_profile_read", "bzk_debug_field",
-                     "bzk_debug_sha256", "bzk_debug_bench", "bzk_merkle", "bzk_generate_blocks"):
+                     "bzk_debug_sha256", "bzk_debug_bench", "bzk_merkle", "bzk_generate_blocks",
+                     "bzk_encoder_create", "bzk_encode"):
             getattr(L, name).restype = i32
         _lib = L
     return _lib
@@ -192,6 +207,33 @@ def bzk_generate_blocks(dst, batch, n, first_index=0, data_seed=None, stream=Non
     from .inputs import MERKLE_DATA_SEED
     _check(lib().bzk_generate_blocks(ptr(dst), batch, n, first_index,
                                      MERKLE_DATA_SEED if data_seed is None else data_seed, _stream_handle(stream)))
+
+
+def _csr_struct(m: dict) -> bzk_csr:
+    for k_ in ("row_ptr", "col", "val"):
+        assert m[k_].flags["C_CONTIGUOUS"]
+    return bzk_csr(m["rows"], m["cols"], int(m["row_ptr"][-1]), m["row_ptr"].ctypes.data, m["col"].ctypes.data,
+                   m["val"].ctypes.data)
+
+
+def bzk_encoder_create(ctx, code: dict):
+    """code: the dict of inputs.gen_code (host CSR arrays).  Returns an opaque encoder handle."""
+    L = code["levels"]
+    A = (bzk_csr * max(1, L))(*[_csr_struct(a) for a in code["A"]])
+    B = (bzk_csr * max(1, L))(*[_csr_struct(b) for b in code["B"]])
+    G0 = _csr_struct(code["G0"])
+    c = bzk_code(code["log_n"], L, ctypes.addressof(A), ctypes.addressof(B), ctypes.addressof(G0))
+    h = ctypes.c_void_p()
+    _check(lib().bzk_encoder_create(ctx, ctypes.byref(c), ctypes.byref(h)), ctx)
+    return h
+
+
+def bzk_encoder_destroy(enc) -> None:
+    lib().bzk_encoder_destroy(enc)
+
+
+def bzk_encode(ctx, enc, codes, batch: int, codes_mem: int = BZK_MEM_DEVICE, flags: int = 0, stream=None) -> None:
+    _check(lib().bzk_encode(ctx, enc, ptr(codes), batch, codes_mem, flags, _stream_handle(stream)), ctx)
 
 
 def bzk_profile_enable(ctx, on: bool) -> None:
@@ -341,3 +383,37 @@ class MerkleBuilder:
         b = self.batch(blocks, n, hash_mode, roots, nodes if with_nodes else None, flags)
         bzk_merkle(self.ctx, b, stream)
         return roots, (nodes if with_nodes else None)
+
+
+class Encoder:
+    """Linear-time encoder (NEXT-4) for one code (graphs from inputs.gen_code); encodes batches in place.
+
+    codes: int64 tensor [B][2n][4] (device, or pinned host) whose first n elements per row are the
+    messages; after encode() each row is its codeword.
+    """
+
+    def __init__(self, code: dict, device: int = 0, ctx=None, workspace_limit: int = 0):
+        self.device = device
+        self._own = ctx is None
+        self.ctx = bzk_create(device, workspace_limit) if ctx is None else ctx
+        self.log_n = code["log_n"]
+        self.enc = bzk_encoder_create(self.ctx, code)
+
+    def close(self):
+        if getattr(self, "enc", None):
+            bzk_encoder_destroy(self.enc)
+            self.enc = None
+        if self.ctx and self._own:
+            bzk_destroy(self.ctx)
+        self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    def encode(self, codes, flags: int = 0, stream=None):
+        host = hasattr(codes, "is_cuda") and not codes.is_cuda
+        bzk_encode(self.ctx, self.enc, codes, codes.shape[0], BZK_MEM_HOST if host else BZK_MEM_DEVICE, flags, stream)
+        return codes

@@ -18,6 +18,7 @@
 #include "gl.cuh"
 #include "gen.cuh"
 #include "merkle.cuh"
+#include "encoder.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
 
@@ -777,6 +778,242 @@ bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) 
     return BZK_OK;
 }
 
+
+// ---------------------------------------------------------------- linear-time encoder (NEXT-4)
+//
+// bzk_encoder_create converts every CSR graph to SELL-32 on the host (rows sorted by length, the
+// paper's bucket sort of P:191, 32 rows per warp slice, entries lane-interleaved), uploads it in one
+// allocation and turns the weights into Montgomery form on the device.  bzk_encode then runs the
+// two launch chains of encoder.cuh in place on the codeword buffer.
+
+struct SellDev {
+    uint32_t rows = 0, cols = 0, slices = 0;
+    uint64_t entries = 0;
+    uint32_t *perm = nullptr, *slice_w = nullptr, *col = nullptr;
+    uint64_t *slice_off = nullptr;
+    fe *val = nullptr;
+};
+
+}  // namespace
+
+struct bzk_encoder {
+    int device = 0;
+    uint32_t log_n = 0, levels = 0, m = 0;
+    std::vector<SellDev> A, B;
+    SellDev G0;
+    void *mem = nullptr;
+    size_t bytes = 0;
+};
+
+namespace {
+
+struct SellHost {
+    std::vector<uint32_t> perm, slice_w, col;
+    std::vector<uint64_t> slice_off;
+    std::vector<uint64_t> val;   // 4 words per entry
+};
+
+bzk_status sell_build(bzk_ctx *ctx, const bzk_csr &M, SellHost &H, std::string &why) {
+    if (!M.row_ptr || !M.col || !M.val) { why = "CSR pointer is NULL"; return BZK_EINVAL; }
+    const uint32_t rows = M.rows;
+    std::vector<uint32_t> len(rows);
+    for (uint32_t r = 0; r < rows; ++r) {
+        if (M.row_ptr[r + 1] < M.row_ptr[r]) { why = "row_ptr not monotone"; return BZK_EINVAL; }
+        len[r] = M.row_ptr[r + 1] - M.row_ptr[r];
+    }
+    if (M.row_ptr[rows] != M.nnz) { why = "row_ptr[rows] != nnz"; return BZK_EINVAL; }
+    for (uint64_t e = 0; e < M.nnz; ++e)
+        if (M.col[e] >= M.cols) { why = "column index out of range"; return BZK_EINVAL; }
+    // bucket sort of the rows by length, longest first
+    const uint32_t maxlen = rows ? *std::max_element(len.begin(), len.end()) : 0;
+    std::vector<uint32_t> cnt(maxlen + 2, 0);
+    for (uint32_t r = 0; r < rows; ++r) ++cnt[maxlen - len[r]];
+    std::vector<uint32_t> start(maxlen + 2, 0);
+    for (uint32_t k = 1; k <= maxlen + 1; ++k) start[k] = start[k - 1] + cnt[k - 1];
+    std::vector<uint32_t> order(rows);
+    for (uint32_t r = 0; r < rows; ++r) order[start[maxlen - len[r]]++] = r;
+    const uint32_t slices = (rows + 31) / 32;
+    H.perm.assign((size_t)slices * 32, 0xffffffffu);
+    H.slice_w.assign(slices, 0);
+    H.slice_off.assign(slices, 0);
+    uint64_t total = 0;
+    for (uint32_t sl = 0; sl < slices; ++sl) {
+        H.slice_w[sl] = len[order[(size_t)sl * 32]];
+        H.slice_off[sl] = total;
+        total += (uint64_t)H.slice_w[sl] * 32;
+    }
+    H.col.assign(total, 0);
+    H.val.assign(total * 4, 0);
+    for (uint32_t sl = 0; sl < slices; ++sl) {
+        for (uint32_t ln = 0; ln < 32; ++ln) {
+            const uint64_t i = (uint64_t)sl * 32 + ln;
+            if (i >= rows) break;
+            const uint32_t r = order[i];
+            H.perm[i] = r;
+            for (uint32_t t = 0; t < len[r]; ++t) {
+                const uint64_t src = (uint64_t)M.row_ptr[r] + t, dst = H.slice_off[sl] + (uint64_t)t * 32 + ln;
+                H.col[dst] = M.col[src];
+                memcpy(&H.val[dst * 4], M.val + src * 4, 32);
+            }
+        }
+    }
+    (void)ctx;
+    return BZK_OK;
+}
+
+size_t sell_bytes(const SellHost &H) {
+    return align_up(H.perm.size() * 4) + align_up(H.slice_w.size() * 4) + align_up(H.slice_off.size() * 8) +
+           align_up(H.col.size() * 4) + align_up(H.val.size() * 8);
+}
+
+cudaError_t sell_upload(const SellHost &H, const bzk_csr &M, char *&cur, SellDev &D, cudaStream_t s) {
+    D.rows = M.rows; D.cols = M.cols; D.slices = (uint32_t)H.slice_w.size(); D.entries = H.col.size();
+    auto put = [&](const void *src, size_t n, auto *&dst) -> cudaError_t {
+        dst = reinterpret_cast<std::remove_reference_t<decltype(dst)>>(cur);
+        cur += align_up(n);
+        return n ? cudaMemcpyAsync((void *)dst, src, n, cudaMemcpyHostToDevice, s) : cudaSuccess;
+    };
+    cudaError_t e;
+    if ((e = put(H.perm.data(), H.perm.size() * 4, D.perm)) != cudaSuccess) return e;
+    if ((e = put(H.slice_w.data(), H.slice_w.size() * 4, D.slice_w)) != cudaSuccess) return e;
+    if ((e = put(H.slice_off.data(), H.slice_off.size() * 8, D.slice_off)) != cudaSuccess) return e;
+    if ((e = put(H.col.data(), H.col.size() * 4, D.col)) != cudaSuccess) return e;
+    if ((e = put(H.val.data(), H.val.size() * 8, D.val)) != cudaSuccess) return e;
+    return enc_launch_to_mont(D.val, D.entries, s);
+}
+
+bzk_status encoder_create_impl(bzk_ctx *ctx, const bzk_code *c, bzk_encoder **out) {
+    if (!c || !out) return fail(ctx, BZK_EINVAL, "code/out is NULL");
+    *out = nullptr;
+    if (c->log_n > 26) return fail(ctx, BZK_EINVAL, "log_n must be <= 26");
+    const uint64_t n = 1ull << c->log_n;
+    if (c->levels > 0 && (!c->A || !c->B)) return fail(ctx, BZK_EINVAL, "A/B is NULL");
+    if (!c->G0) return fail(ctx, BZK_EINVAL, "G0 is NULL");
+    // shapes (reading R21): A_l is n_l/4 x n_l, B_l is n_l/2 x n_l/2, G0 is n_L x n_L
+    for (uint32_t l = 0; l < c->levels; ++l) {
+        const uint64_t nl = n >> (2 * l);
+        if (nl < 8 || c->A[l].cols != nl || c->A[l].rows != nl / 4 || c->B[l].cols != nl / 2 || c->B[l].rows != nl / 2)
+            return fail(ctx, BZK_EINVAL, "graph shapes do not match log_n / level " + std::to_string(l));
+    }
+    const uint64_t m = n >> (2 * c->levels);
+    if (m == 0 || c->G0->rows != m || c->G0->cols != m) return fail(ctx, BZK_EINVAL, "G0 must be n_L x n_L");
+    std::vector<SellHost> HA(c->levels), HB(c->levels);
+    SellHost HG;
+    std::string why;
+    size_t bytes = 0;
+    for (uint32_t l = 0; l < c->levels; ++l) {
+        if (sell_build(ctx, c->A[l], HA[l], why) || sell_build(ctx, c->B[l], HB[l], why))
+            return fail(ctx, BZK_EINVAL, "level " + std::to_string(l) + ": " + why);
+        bytes += sell_bytes(HA[l]) + sell_bytes(HB[l]);
+    }
+    if (sell_build(ctx, *c->G0, HG, why)) return fail(ctx, BZK_EINVAL, "G0: " + why);
+    bytes += sell_bytes(HG);
+    bzk_encoder *E = new bzk_encoder();
+    E->device = ctx->device; E->log_n = c->log_n; E->levels = c->levels; E->m = (uint32_t)m; E->bytes = bytes;
+    cudaError_t e = cudaMalloc(&E->mem, std::max<size_t>(bytes, 256));
+    if (e != cudaSuccess) { cudaGetLastError(); delete E; return fail(ctx, BZK_ENOMEM, "cudaMalloc encoder graphs"); }
+    char *cur = (char *)E->mem;
+    E->A.resize(c->levels); E->B.resize(c->levels);
+    cudaStream_t s = ctx->copy_stream;
+    for (uint32_t l = 0; l < c->levels && e == cudaSuccess; ++l) {
+        e = sell_upload(HA[l], c->A[l], cur, E->A[l], s);
+        if (e == cudaSuccess) e = sell_upload(HB[l], c->B[l], cur, E->B[l], s);
+    }
+    if (e == cudaSuccess) e = sell_upload(HG, *c->G0, cur, E->G0, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);   // host SELL arrays die with this scope
+    if (e != cudaSuccess) { cudaFree(E->mem); delete E; return cuda_fail(ctx, e, "encoder upload"); }
+    *out = E;
+    return BZK_OK;
+}
+
+cudaError_t spmv(bzk_ctx *ctx, const SellDev &M, const fe *src, fe *dst, uint64_t stride, uint64_t nb, cudaStream_t s) {
+    enc::SpmvParams p;
+    p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
+    p.slices = M.slices; p.src = src; p.dst = dst; p.stride = stride; p.batch = nb;
+    const uint32_t warps = 8;
+    dim3 grid((M.slices + warps - 1) / warps, (uint32_t)((nb + BZK_ENC_K - 1) / BZK_ENC_K));
+    ProfScope ps_(ctx, s, 8);
+    ++ctx->launches;
+    return enc_launch_spmv(grid, warps * 32, s, p);
+}
+
+// encode nb codewords in place: C[b][0..n) = message on entry, C[b][0..2n) = codeword on exit
+bzk_status encode_wave(bzk_ctx *ctx, const bzk_encoder *E, fe *C, uint64_t nb, cudaStream_t s) {
+    const uint64_t n = 1ull << E->log_n, stride = 2 * n;
+    std::vector<uint64_t> o(E->levels + 1), nl(E->levels + 1);
+    o[0] = 0; nl[0] = n;
+    for (uint32_t l = 0; l < E->levels; ++l) { o[l + 1] = o[l] + nl[l]; nl[l + 1] = nl[l] / 4; }
+    for (uint32_t l = 0; l < E->levels; ++l)             // forward chain: x_{l+1} = A_l x_l
+        CK(spmv(ctx, E->A[l], C + o[l], C + o[l + 1], stride, nb, s));
+    const uint32_t L = E->levels;
+    CK(spmv(ctx, E->G0, C + o[L], C + o[L] + nl[L], stride, nb, s));   // base: x_L || G0 x_L
+    for (int l = (int)L - 1; l >= 0; --l)                 // reverse chain: w_l = B_l c_{l+1}
+        CK(spmv(ctx, E->B[l], C + o[l + 1], C + o[l] + nl[l] + nl[l] / 2, stride, nb, s));
+    return BZK_OK;
+}
+
+bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint64_t batch, uint32_t codes_mem,
+                       uint32_t flags, cudaStream_t s) {
+    if (!E || !codes) return fail(ctx, BZK_EINVAL, "encoder/codes is NULL");
+    if (E->device != ctx->device) return fail(ctx, BZK_EINVAL, "encoder belongs to another device");
+    if (batch == 0) return fail(ctx, BZK_EINVAL, "batch must be >= 1");
+    if (codes_mem > 1) return fail(ctx, BZK_EINVAL, "bad codes_mem");
+    const uint64_t n = 1ull << E->log_n;
+    const size_t cw = (size_t)2 * n * 32;   // bytes per codeword
+    if (codes_mem == BZK_MEM_DEVICE) {
+        if ((uintptr_t)codes & 31u) return fail(ctx, BZK_EINVAL, "device codes must be 32-byte aligned");
+        bzk_status st = encode_wave(ctx, E, (fe *)codes, batch, s);
+        if (st) return st;
+        if (flags & BZK_F_SYNC) CK(cudaStreamSynchronize(s));
+        return BZK_OK;
+    }
+    // host codewords: waves through the loader ring (H2D of the messages on copy_stream, D2H of the
+    // codewords on d2h_stream, overlapping the next wave's encoding)
+    size_t limit = ctx->workspace_limit;
+    if (limit == 0) {
+        size_t fr = 0, tot = 0;
+        cudaMemGetInfo(&fr, &tot);
+        fr += 2 * ctx->stage_size;
+        limit = fr > (2ull << 30) ? fr - (2ull << 30) : fr / 2;
+    }
+    uint64_t bw = batch;
+    if (batch >= 8 && batch * cw > (1ull << 30)) bw = (batch + 7) / 8;
+    while (bw > 1 && 2 * bw * cw + 4096 > limit) bw = (bw + 1) / 2;
+    if (2 * bw * cw + 4096 > limit) return fail(ctx, BZK_ENOMEM, "workspace_limit too small for one codeword");
+    const uint64_t nw = (batch + bw - 1) / bw;
+    bw = (batch + nw - 1) / nw;
+    bzk_status st = ensure_stage(ctx, align_up(bw * cw));
+    if (st) return st;
+    for (uint64_t w = 0; w < nw; ++w) {
+        const uint64_t b0 = w * bw, nb = std::min<uint64_t>(bw, batch - b0);
+        const int slot = ctx->next_slot;
+        ctx->next_slot ^= 1;
+        if (ctx->slot_used[slot]) CK(cudaStreamWaitEvent(ctx->copy_stream, ctx->ev_consumed[slot], 0));
+        char *dev = (char *)ctx->stage[slot];
+        {
+            ProfScope ps_(ctx, ctx->copy_stream, 5);
+            // messages only (the first n elements of every codeword)
+            CK(cudaMemcpy2DAsync(dev, cw, (const char *)codes + b0 * cw, cw, n * 32, nb, cudaMemcpyHostToDevice,
+                                 ctx->copy_stream));
+        }
+        CK(cudaEventRecord(ctx->ev_copied[slot], ctx->copy_stream));
+        CK(cudaStreamWaitEvent(s, ctx->ev_copied[slot], 0));
+        st = encode_wave(ctx, E, (fe *)dev, nb, s);
+        if (st) return st;
+        CK(cudaEventRecord(ctx->ev_nodes_ready[slot], s));
+        CK(cudaStreamWaitEvent(ctx->d2h_stream, ctx->ev_nodes_ready[slot], 0));
+        {
+            ProfScope ps_(ctx, ctx->d2h_stream, 7);
+            CK(cudaMemcpyAsync((char *)codes + b0 * cw, dev, nb * cw, cudaMemcpyDeviceToHost, ctx->d2h_stream));
+        }
+        CK(cudaEventRecord(ctx->ev_consumed[slot], ctx->d2h_stream));
+        ctx->slot_used[slot] = true;
+    }
+    CK(cudaStreamSynchronize(ctx->d2h_stream));
+    CK(cudaStreamSynchronize(s));
+    return BZK_OK;
+}
+
 // ---------------------------------------------------------------- debug kernels
 
 __global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *out) {
@@ -926,7 +1163,7 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
 
 extern "C" {
 
-const char *bzk_version(void) { return "bzk 0.2 sm_100a (BN254 Fr + Goldilocks sum-check, SHA-256 Fiat-Shamir, batched Merkle trees)"; }
+const char *bzk_version(void) { return "bzk 0.3 sm_100a (BN254 Fr + Goldilocks sum-check, SHA-256 Fiat-Shamir, batched Merkle trees, linear-time encoder)"; }
 
 const char *bzk_strerror(bzk_status s) {
     switch (s) {
@@ -1053,6 +1290,27 @@ bzk_status bzk_merkle(bzk_ctx *ctx, const bzk_merkle_batch *batch, void *cuda_st
     if (!ctx) return BZK_EINVAL;
     cudaSetDevice(ctx->device);
     return merkle_impl(ctx, batch, (cudaStream_t)cuda_stream);
+}
+
+bzk_status bzk_encoder_create(bzk_ctx *ctx, const bzk_code *code, bzk_encoder **out) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    return encoder_create_impl(ctx, code, out);
+}
+
+void bzk_encoder_destroy(bzk_encoder *enc) {
+    if (!enc) return;
+    cudaSetDevice(enc->device);
+    cudaDeviceSynchronize();
+    if (enc->mem) cudaFree(enc->mem);
+    delete enc;
+}
+
+bzk_status bzk_encode(bzk_ctx *ctx, const bzk_encoder *enc, uint64_t *codes, uint64_t batch, uint32_t codes_mem,
+                      uint32_t flags, void *cuda_stream) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    return encode_impl(ctx, enc, codes, batch, codes_mem, flags, (cudaStream_t)cuda_stream);
 }
 
 bzk_status bzk_generate_blocks(uint8_t *dst, uint64_t batch, uint32_t n, uint64_t first_index, uint64_t data_seed,
