@@ -930,7 +930,7 @@ cudaError_t spmv(bzk_ctx *ctx, const SellDev &M, const fe *src, fe *dst, uint64_
     enc::SpmvParams p;
     p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
     p.slices = M.slices; p.src = src; p.dst = dst; p.stride = stride; p.batch = nb;
-    const uint32_t warps = 8;
+    const uint32_t warps = BZK_ENC_TPB / 32;
     dim3 grid((M.slices + warps - 1) / warps, (uint32_t)((nb + BZK_ENC_K - 1) / BZK_ENC_K));
     ProfScope ps_(ctx, s, 8);
     ++ctx->launches;

@@ -40,11 +40,18 @@ struct SpmvParams {
 };
 
 #ifndef BZK_ENC_K
-#define BZK_ENC_K 2
+#define BZK_ENC_K 2      // codewords per thread (share every weight load)
+#endif
+#ifndef BZK_ENC_U
+#define BZK_ENC_U 2      // entries per loop iteration (their gathers are in flight together)
 #endif
 
-template <int K>
-__global__ void __launch_bounds__(256) k_spmv(SpmvParams p) {
+#ifndef BZK_ENC_TPB
+#define BZK_ENC_TPB 128  // threads per CTA (4 warp slices; finer occupancy steps at ~100 registers)
+#endif
+
+template <int K, int U>
+__global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t slice = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (slice >= p.slices) return;
@@ -58,8 +65,26 @@ __global__ void __launch_bounds__(256) k_spmv(SpmvParams p) {
     const fe *src[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) src[q] = p.src + (b0 + q < p.batch ? b0 + q : b0) * p.stride;
+    uint32_t t = 0;
 #pragma unroll 1
-    for (uint32_t t = 0; t < W; ++t) {
+    for (; U > 1 && t + U <= W; t += U) {
+        uint32_t c[U];
+        fe w[U], x[U][K];
+#pragma unroll
+        for (int u = 0; u < U; ++u) c[u] = __ldg(p.col + off + (uint64_t)(t + u) * 32);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int q = 0; q < K; ++q) BZK_LD8(".nc", x[u][q], src[q] + c[u]);
+#pragma unroll
+        for (int u = 0; u < U; ++u) w[u] = ld_fe_stream(p.val + off + (uint64_t)(t + u) * 32);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+            for (int q = 0; q < K; ++q) mul_acc(acc[q], w[u], x[u][q]);
+    }
+#pragma unroll 1
+    for (; t < W; ++t) {
         const uint64_t e = off + (uint64_t)t * 32;
         const uint32_t c = __ldg(p.col + e);
         const fe w = ld_fe_stream(p.val + e);

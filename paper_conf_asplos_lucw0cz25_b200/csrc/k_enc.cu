@@ -4,7 +4,7 @@
 namespace bzk {
 
 cudaError_t enc_launch_spmv(dim3 grid, uint32_t threads, cudaStream_t s, const enc::SpmvParams &p) {
-    enc::k_spmv<BZK_ENC_K><<<grid, threads, 0, s>>>(p);
+    enc::k_spmv<BZK_ENC_K, BZK_ENC_U><<<grid, threads, 0, s>>>(p);
     return cudaGetLastError();
 }
 
