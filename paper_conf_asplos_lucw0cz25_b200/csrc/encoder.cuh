@@ -46,6 +46,38 @@ struct SpmvParams {
 #define BZK_ENC_U 2      // entries per loop iteration (their gathers are in flight together)
 #endif
 
+// BZK_ENC_L2HINT=1: gathers carry an L2 evict_last policy and the weight stream evict_first, so the
+// streamed weights do not push the live source vectors out of L2.
+#ifndef BZK_ENC_L2HINT
+#define BZK_ENC_L2HINT 1
+#endif
+
+__device__ __forceinline__ uint64_t l2_policy_last() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint64_t l2_policy_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ fe ld_fe_hint(const fe *p, uint64_t pol) {
+    fe r;
+    asm("ld.global.nc.L2::cache_hint.v8.u32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8], %9;"
+        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
+          "=r"(r.l[7])
+        : "l"(p), "l"(pol));
+    return r;
+}
+#if BZK_ENC_L2HINT
+#define BZK_ENC_GATHER(x, ptr) (x) = ld_fe_hint((ptr), pol_last)
+#define BZK_ENC_WEIGHT(ptr) ld_fe_hint((ptr), pol_first)
+#else
+#define BZK_ENC_GATHER(x, ptr) BZK_LD8(".nc", x, ptr)
+#define BZK_ENC_WEIGHT(ptr) ld_fe_stream(ptr)
+#endif
+
 #ifndef BZK_ENC_TPB
 #define BZK_ENC_TPB 128  // threads per CTA (4 warp slices; finer occupancy steps at ~100 registers)
 #endif
@@ -59,6 +91,9 @@ __global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
     const uint32_t row = p.perm[(size_t)slice * 32 + lane];
     const uint32_t W = p.slice_w[slice];
     const uint64_t off = p.slice_off[slice] + lane;
+#if BZK_ENC_L2HINT
+    const uint64_t pol_last = l2_policy_last(), pol_first = l2_policy_first();
+#endif
     acc17 acc[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) acc[q] = acc17_zero();
@@ -75,9 +110,9 @@ __global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
-            for (int q = 0; q < K; ++q) BZK_LD8(".nc", x[u][q], src[q] + c[u]);
+            for (int q = 0; q < K; ++q) BZK_ENC_GATHER(x[u][q], src[q] + c[u]);
 #pragma unroll
-        for (int u = 0; u < U; ++u) w[u] = ld_fe_stream(p.val + off + (uint64_t)(t + u) * 32);
+        for (int u = 0; u < U; ++u) w[u] = BZK_ENC_WEIGHT(p.val + off + (uint64_t)(t + u) * 32);
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
@@ -87,11 +122,11 @@ __global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
     for (; t < W; ++t) {
         const uint64_t e = off + (uint64_t)t * 32;
         const uint32_t c = __ldg(p.col + e);
-        const fe w = ld_fe_stream(p.val + e);
+        const fe w = BZK_ENC_WEIGHT(p.val + e);
 #pragma unroll
         for (int q = 0; q < K; ++q) {
             fe x;
-            BZK_LD8(".nc", x, src[q] + c);
+            BZK_ENC_GATHER(x, src[q] + c);
             mul_acc(acc[q], w, x);
         }
     }
