@@ -747,6 +747,22 @@ def main():
 
     max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
     digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
+    # the proofs themselves are gathered to rank 0 over NCCL (NVLink) after the timed region
+    # (north star: "NCCL is used only to gather proofs and timing"); rank 0 digests the global batch
+    gathered = None
+    if dist:
+        torch.cuda.synchronize()
+        g0 = time.perf_counter()
+        allp = shard.gather_outputs({k_: out[k_] for k_ in ("round_evals", "challenges", "final_evals", "claims")},
+                                    dist, dst=0)
+        torch.cuda.synchronize()
+        g_ms = (time.perf_counter() - g0) * 1000.0
+        if rank == 0:
+            gbytes = sum(v.numel() * v.element_size() for v in allp.values())
+            gathered = {"proofs": B * world, "bytes": int(gbytes), "ms": round(g_ms, 3),
+                        "backend": dist.get_backend(),
+                        "global_digest": shard.output_digest([allp[k_].cpu() for k_ in
+                                                              ("round_evals", "challenges", "final_evals", "claims")])}
 
     total_proofs = B * world * args.steps
     value = total_proofs / (max_ms / 1000.0)
@@ -804,6 +820,8 @@ def main():
             "kernel_ms_per_step": kernel_ms, "ms_per_step_kernel_by_kernel": round(sum(step_ms_prof) / args.steps, 3),
             "roofline": roofline, "clocks": clocks,
             "digest_rank0": digests[0], "digests_per_rank": len(digests)}
+    if gathered:
+        line["proofs_gathered"] = gathered
 
     # ---------------- e2e: host (pinned) tables in, host outputs out, through bzk_prove
     if not args.no_e2e and not consume:

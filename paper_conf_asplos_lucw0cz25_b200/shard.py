@@ -65,8 +65,11 @@ def gather_outputs(tensors: dict, dist, dst: int = 0):
         return tensors
     world, rank = dist.get_world_size(), dist.get_rank()
     out = {}
+    nccl = dist.get_backend() == "nccl"
     for key in sorted(tensors):
         t = tensors[key].contiguous()
+        if not nccl and t.is_cuda:
+            t = t.cpu()                      # gloo: host tensors
         parts = [torch.empty_like(t) for _ in range(world)]
         dist.all_gather(parts, t)
         if rank == dst:
