@@ -174,6 +174,19 @@ ENC_METRIC = "linear-time encodings/s @2^20 BN254 Fr elements (NEXT-4, P:320 Tab
 IMAD_PER_EDGE_PRODUCT = 128
 
 
+def enc_traffic(cfg, B):
+    """average DRAM bytes per k_spmv launch from profiles/traffic.json (ncu capture of one step)"""
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if not os.path.exists(tpath):
+        return None
+    with open(tpath) as f:
+        tj = json.load(f)
+    for e in (tj if isinstance(tj, list) else [tj]):
+        if e.get("config") == cfg and e.get("kernel_kind") == "encoder_spmv" and e.get("batch") == B:
+            return e["dram_bytes_per_launch"]
+    return None
+
+
 def enc_edges(code) -> int:
     return sum(int(a["row_ptr"][-1]) for a in code["A"]) + sum(int(b["row_ptr"][-1]) for b in code["B"]) + \
         int(code["G0"]["row_ptr"][-1])
@@ -582,7 +595,7 @@ def run_encoder(args, rank, world):
                                    "launches_per_step": spmv_cnt // max(1, args.steps)},
             "roofline": {"bound": "alu", "kernel": "k_spmv (all products of a step)", "achieved": round(achieved, 2),
                          "peak": round(peak, 2), "unit": "Gproduct/s", "frac": round(achieved / peak, 4),
-                         "traffic": None, "alg_products_per_step": B * edges,
+                         "traffic": enc_traffic(args.config, B), "alg_products_per_step": B * edges,
                          "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} "
                                         f"MHz ({peak_src} max clock) / {IMAD_PER_EDGE_PRODUCT} IMAD slots per "
                                         "256x256-bit edge product (reduction amortised per output element)",
@@ -788,8 +801,9 @@ def main():
         # command (scripts/ncu_traffic.sh), if it was taken on this workload
         with open(tpath) as f:
             tj = json.load(f)
-        if tj.get("config") == args.config and tj.get("kernel_kind") == dom and tj.get("batch") == B:
-            traffic = tj["dram_bytes_per_launch"]
+        for e in (tj if isinstance(tj, list) else [tj]):
+            if e.get("config") == args.config and e.get("kernel_kind") == dom and e.get("batch") == B:
+                traffic = e["dram_bytes_per_launch"]
     bytes_per_launch = alg_bytes_kind(d, k, kinds[dom], esz) * B / max(1, dom_cnt / args.steps)
     roofline = {"bound": "alu", "kernel": dom, "achieved": round(achieved, 2), "peak": round(int_peak, 2),
                 "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": traffic,

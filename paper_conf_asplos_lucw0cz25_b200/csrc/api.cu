@@ -131,10 +131,10 @@ struct Plan {
 };
 
 // tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
-// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round, default on)
+// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round, default off)
 struct Knobs {
     uint64_t ppt_max = 64, waves = 4;
-    uint32_t prefetch = 1;
+    uint32_t prefetch = 0;   // BZK_PREFETCH=1: L2 bulk prefetch (measured: fused rounds read 1.5x their bytes, -6 %)
     // BZK_CLUSTER=N: CTAs of a proof form thread-block clusters of up to N (2, 4, 8) that combine
     // their partial sums through DSMEM.  Off by default: measured 10 % slower on B200.
     uint32_t cluster = 1;
