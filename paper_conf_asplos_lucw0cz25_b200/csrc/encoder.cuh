@@ -142,8 +142,10 @@ __global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
 // 3 S 32-byte loads per thread are in flight instead of the 2 U gathers of k_spmv (ncu: k_spmv
 // stalled on gather latency at 82 % fma-heavy busy).  Chunk-major slots (chunk c of thread t at
 // (slot chunk index * blockDim + t) * 16) keep the shared-memory writes and reads conflict-free.
+// Measured SLOWER on B200 (2,897 vs 3,473 codes/s at S = 4: 122 registers and the LDGSTS/LDS overhead
+// cost more than the extra memory-level parallelism gains); bit-exact, kept as an option.
 #ifndef BZK_ENC_ASYNC
-#define BZK_ENC_ASYNC 1
+#define BZK_ENC_ASYNC 0
 #endif
 #ifndef BZK_ENC_S
 #define BZK_ENC_S 4
