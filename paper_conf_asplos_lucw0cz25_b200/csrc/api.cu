@@ -131,10 +131,12 @@ struct Plan {
 };
 
 // tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
-// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round, default off)
+// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round; default: on for d >= 3 only)
 struct Knobs {
     uint64_t ppt_max = 64, waves = 4;
-    uint32_t prefetch = 0;   // BZK_PREFETCH=1: L2 bulk prefetch (measured: fused rounds read 1.5x their bytes, -6 %)
+    // L2 bulk prefetch: -1 = by degree.  d <= 2: off (the fused rounds then read exactly their bytes;
+    // with it 1.5x, -6 % at c2, -2 % at m0); d >= 3: on (IMAD-bound, +2 % at c3).  DESIGN.md sec. 8.
+    int prefetch = -1;
     // BZK_CLUSTER=N: CTAs of a proof form thread-block clusters of up to N (2, 4, 8) that combine
     // their partial sums through DSMEM.  Off by default: measured 10 % slower on B200.
     uint32_t cluster = 1;
@@ -143,6 +145,9 @@ struct Knobs {
         if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_CTA_WAVES")) waves = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_PREFETCH")) prefetch = atoi(e) ? 1 : 0;
+    }
+    uint32_t prefetch_for(uint32_t d) const {
+        return prefetch < 0 ? (d >= 3 ? 1u : 0u) : (uint32_t)prefetch;
     }
 };
 const Knobs &knobs() { static Knobs k; return k; }
@@ -419,7 +424,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = (fe *)io.round_evals; rp.challenges = (fe *)io.challenges; rp.claims = (fe *)io.claims;
         rp.consts = ctx->consts;
-        rp.prefetch = knobs().prefetch;
+        rp.prefetch = knobs().prefetch_for(P.D);
         rp.given = P.given;
         rp.cluster = cluster_for(rp.ctas);
         if (i == 1) { rp.src = tab; rp.dst = nullptr; }
