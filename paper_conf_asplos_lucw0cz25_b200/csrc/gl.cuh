@@ -246,6 +246,12 @@ __device__ __forceinline__ void load_pair(const uint64_t *src, uint64_t *dst, ui
 #ifndef GL_OCC
 #define GL_OCC 3
 #endif
+#ifndef GL_SPLIT
+#define GL_SPLIT 1   // fused LSB rounds: issue every raw load of an iteration before the folds
+#endif
+#ifndef GL_MLP_FUSED
+#define GL_MLP_FUSED 2   // pairs per iteration of the split fused loop (g2: 2 -> fused 0.86 of HBM, 4 -> 0.83)
+#endif
 
 template <int D, int ORDER, bool FIRST>
 __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
@@ -272,6 +278,36 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
     // MLP pairs in flight per iteration (memory-level parallelism: the kernel streams); fewer for
     // d >= 3, whose wider accumulators would otherwise spill
     constexpr int MLP = D <= 2 ? GL_MLP : (GL_MLP > 2 ? 2 : GL_MLP);
+#if GL_SPLIT
+    // all raw loads of the MLP pairs first (LSB fused rounds), then folds + stores, then evaluation:
+    // every load is in flight before the first dependent instruction
+    constexpr int MF = D <= 2 ? GL_MLP_FUSED : 2;
+    if (!FIRST && ORDER == 0) {
+        for (; j + (MF - 1) * stride < h; j += MF * stride) {
+            ulonglong2 raw[MF][D][2];
+#pragma unroll
+            for (int q = 0; q < MF; ++q)
+#pragma unroll
+                for (int m = 0; m < D; ++m) {
+                    const uint64_t *T = src + (size_t)m * (4 * h) + 4 * (j + q * stride);
+                    raw[q][m][0] = __ldcs(reinterpret_cast<const ulonglong2 *>(T));
+                    raw[q][m][1] = __ldcs(reinterpret_cast<const ulonglong2 *>(T + 2));
+                }
+            uint64_t a[MF][D], bb[MF][D];
+#pragma unroll
+            for (int q = 0; q < MF; ++q)
+#pragma unroll
+                for (int m = 0; m < D; ++m) {
+                    a[q][m] = fold(raw[q][m][0].x, raw[q][m][0].y, r);
+                    bb[q][m] = fold(raw[q][m][1].x, raw[q][m][1].y, r);
+                    *reinterpret_cast<ulonglong2 *>(dst + (size_t)m * (2 * h) + 2 * (j + q * stride)) =
+                        make_ulonglong2(a[q][m], bb[q][m]);
+                }
+#pragma unroll
+            for (int q = 0; q < MF; ++q) eval_pair<D>(a[q], bb[q], GL_ACC);
+        }
+    }
+#endif
     for (; j + (MLP - 1) * stride < h; j += MLP * stride) {
         uint64_t a[MLP][D], bb[MLP][D];
 #pragma unroll
