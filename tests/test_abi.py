@@ -65,6 +65,38 @@ def test_argument_errors_without_gpu(libbzk):
         libbzk.bzk_destroy(h)
 
 
+def test_module_entry_points_reject_bad_arguments_without_gpu(libbzk):
+    """NEXT-3 / NEXT-4 entry points: NULL context / destination are rejected before any CUDA call."""
+    from paper_conf_asplos_lucw0cz25_b200 import bzk
+    b = bzk.bzk_merkle_batch(4, 0, 0, 0, 1, None, 0, 0, None, None)
+    assert libbzk.bzk_merkle(None, ctypes.byref(b), None) == bzk.BZK_EINVAL
+    assert libbzk.bzk_generate_blocks(None, 1, 4, 0, 0, None) == bzk.BZK_EINVAL
+    h = ctypes.c_void_p()
+    assert libbzk.bzk_encoder_create(None, None, ctypes.byref(h)) == bzk.BZK_EINVAL
+    assert libbzk.bzk_encode(None, None, None, 1, 0, 0, None) == bzk.BZK_EINVAL
+    libbzk.bzk_encoder_destroy(None)   # no-op
+
+
+def test_abi_struct_layouts_match_header():
+    """ctypes mirrors of the ABI structs have the sizes the C compiler gives the header's structs."""
+    import subprocess
+    import tempfile
+    from paper_conf_asplos_lucw0cz25_b200 import bzk
+    src = """#include <stdio.h>
+#include "bzk.h"
+int main(void) { printf("%zu %zu %zu %zu\\n", sizeof(bzk_batch), sizeof(bzk_merkle_batch), sizeof(bzk_csr),
+                        sizeof(bzk_code)); return 0; }
+"""
+    with tempfile.TemporaryDirectory() as d:
+        c = os.path.join(d, "s.c")
+        open(c, "w").write(src)
+        exe = os.path.join(d, "s")
+        subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
+        sizes = [int(x) for x in subprocess.check_output([exe]).split()]
+    assert sizes == [ctypes.sizeof(bzk.bzk_batch), ctypes.sizeof(bzk.bzk_merkle_batch), ctypes.sizeof(bzk.bzk_csr),
+                     ctypes.sizeof(bzk.bzk_code)]
+
+
 def test_product_package_does_not_touch_the_oracle():
     pkg = os.path.join(ROOT, "paper_conf_asplos_lucw0cz25_b200")
     for dirpath, _, files in os.walk(pkg):
