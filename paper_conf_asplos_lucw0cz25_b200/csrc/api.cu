@@ -12,6 +12,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "bzk.h"
 #include "field.cuh"
 #include "field_f64.cuh"
@@ -32,6 +34,18 @@ constexpr uint32_t kTailLog = 8;          // rounds with h <= 2^kTailLog pairs r
 constexpr uint32_t kSMs = 148;
 
 struct ProfRec { int kind; cudaEvent_t a, b; };
+
+// NVTX ranges (host timeline for nsys: calls, jobs, waves, stage chains), on when BZK_NVTX=1.
+// nvtx3 is header-only: without a profiler attached the calls are no-ops.
+bool nvtx_on() {
+    static const bool on = [] { const char *e = getenv("BZK_NVTX"); return e && atoi(e) != 0; }();
+    return on;
+}
+struct NvtxRange {
+    bool active;
+    explicit NvtxRange(const char *name) : active(nvtx_on()) { if (active) nvtxRangePushA(name); }
+    ~NvtxRange() { if (active) nvtxRangePop(); }
+};
 
 }  // namespace
 
@@ -399,6 +413,7 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
 }
 
 bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
+    NvtxRange nv_("bzk wave");
     char *ws = (char *)ctx->ws;
     ProofState *ps = (ProofState *)(ws + P.off_ps);
     uint32_t *tick = (uint32_t *)(ws + P.off_tick);
@@ -463,6 +478,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
 // ahead of compute across waves AND jobs.  Returns after enqueueing (no synchronisation) unless
 // validation is requested.
 bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStream_t s) {
+    NvtxRange nv_("bzk job");
     char *ws = (char *)ctx->ws;
     CK(cudaMemsetAsync(ws + P.off_tick, 0, P.Bw * 4, s));
     const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
@@ -540,6 +556,7 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
 // Plan every job, size the workspace for the largest, enqueue all of them, then synchronise
 // when the caller asked for it or host memory is involved (outputs must be readable on return).
 bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStream_t s) {
+    NvtxRange nv_("bzk_prove");
     std::vector<Plan> plans(njobs);
     size_t ws_need = 0, stage_need = 0;
     bool need_sync = false;
@@ -640,6 +657,7 @@ std::vector<MkStage> merkle_stages(uint32_t n) {
 }
 
 bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) {
+    NvtxRange nv_("bzk_merkle");
     if (!m) return fail(ctx, BZK_EINVAL, "batch is NULL");
     if (m->log_blocks > 30) return fail(ctx, BZK_EINVAL, "log_blocks must be <= 30");
     if (m->hash > 1) return fail(ctx, BZK_EINVAL, "hash must be BZK_MERKLE_COMPRESS or BZK_MERKLE_SHA256");
@@ -959,6 +977,7 @@ bzk_status encode_wave(bzk_ctx *ctx, const bzk_encoder *E, fe *C, uint64_t nb, c
 
 bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint64_t batch, uint32_t codes_mem,
                        uint32_t flags, cudaStream_t s) {
+    NvtxRange nv_("bzk_encode");
     if (!E || !codes) return fail(ctx, BZK_EINVAL, "encoder/codes is NULL");
     if (E->device != ctx->device) return fail(ctx, BZK_EINVAL, "encoder belongs to another device");
     if (batch == 0) return fail(ctx, BZK_EINVAL, "batch must be >= 1");
