@@ -950,14 +950,20 @@ bzk_status encoder_create_impl(bzk_ctx *ctx, const bzk_code *c, bzk_encoder **ou
 }
 
 cudaError_t spmv(bzk_ctx *ctx, const SellDev &M, const fe *src, fe *dst, uint64_t stride, uint64_t nb, cudaStream_t s) {
-    enc::SpmvParams p;
-    p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
-    p.slices = M.slices; p.src = src; p.dst = dst; p.stride = stride; p.batch = nb;
     const uint32_t warps = BZK_ENC_TPB / 32;
-    dim3 grid((M.slices + warps - 1) / warps, (uint32_t)((nb + BZK_ENC_K - 1) / BZK_ENC_K));
-    ProfScope ps_(ctx, s, 8);
-    ++ctx->launches;
-    return enc_launch_spmv(grid, warps * 32, s, p);
+    const uint64_t per_launch = 65535ull * BZK_ENC_K;   // gridDim.y limit
+    for (uint64_t c0 = 0; c0 < nb; c0 += per_launch) {
+        const uint64_t n = std::min<uint64_t>(per_launch, nb - c0);
+        enc::SpmvParams p;
+        p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
+        p.slices = M.slices; p.src = src + c0 * stride; p.dst = dst + c0 * stride; p.stride = stride; p.batch = n;
+        dim3 grid((M.slices + warps - 1) / warps, (uint32_t)((n + BZK_ENC_K - 1) / BZK_ENC_K));
+        ProfScope ps_(ctx, s, 8);
+        ++ctx->launches;
+        cudaError_t e = enc_launch_spmv(grid, warps * 32, s, p);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
 }
 
 // encode nb codewords in place: C[b][0..n) = message on entry, C[b][0..2n) = codeword on exit
