@@ -82,8 +82,12 @@ __device__ __forceinline__ fe ld_fe_hint(const fe *p, uint64_t pol) {
 #define BZK_ENC_TPB 128  // threads per CTA (4 warp slices; finer occupancy steps at ~100 registers)
 #endif
 
+#ifndef BZK_ENC_MINB
+#define BZK_ENC_MINB 1   // min resident CTAs per SM for the register allocator (1 = unconstrained)
+#endif
+
 template <int K, int U>
-__global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
+__global__ void __launch_bounds__(BZK_ENC_TPB, BZK_ENC_MINB) k_spmv(SpmvParams p) {
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t slice = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (slice >= p.slices) return;
