@@ -118,3 +118,41 @@ def test_vml_image_shapes(orc):
             for key in KEYS:
                 assert np.array_equal(outs[li][key][b].numpy().view(np.uint64).reshape(ref[key].shape), ref[key])
     p.close()
+
+
+def test_mk20_full_size(orc):
+    """NEXT-3 at bench.py's mk20 call: 256 trees x 2^20 blocks, node arrays on the device (one
+    bzk_merkle call over the whole batch).  Sampled trees recomputed by the oracle (every node);
+    every root checked against the sampled-leaf authentication paths is implied by the node check."""
+    from paper_conf_asplos_lucw0cz25_b200 import inputs
+    B, n = 256, 20
+    blocks = torch.empty((B, 1 << n, 64), dtype=torch.uint8, device="cuda")
+    bzk.bzk_generate_blocks(blocks, B, n, 0)
+    mb = bzk.MerkleBuilder(0)
+    roots, nodes = mb.build(blocks, n, bzk.BZK_MERKLE_COMPRESS)
+    torch.cuda.synchronize()
+    for b in (0, 137, 255):
+        exp_root, exp_nodes = orc.merkle(inputs.gen_blocks(1, n, first_index=b)[0], n, 0)
+        assert bytes(roots[b].cpu().numpy()) == exp_root
+        assert np.array_equal(nodes[b].cpu().numpy(), exp_nodes)
+    mb.close()
+
+
+def test_enc20_full_size(orc):
+    """NEXT-4 at bench.py's enc20 call: 256 codewords of 2^20 elements in one bzk_encode; sampled
+    codewords recomputed by the oracle element by element."""
+    from paper_conf_asplos_lucw0cz25_b200 import inputs
+    B, log_n = 256, 20
+    n = 1 << log_n
+    code = inputs.gen_code(log_n, 6)
+    enc = bzk.Encoder(code, 0)
+    msgs = torch.empty((B, 1, n, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(msgs, B, 1, log_n, 0, "uniform")
+    codes = torch.empty((B, 2 * n, 4), dtype=torch.int64, device="cuda")
+    codes[:, :n].copy_(msgs[:, 0])
+    enc.encode(codes)
+    torch.cuda.synchronize()
+    for b in (0, 255):
+        m = inputs.gen_tables(1, 1, log_n, first_index=b)[0, 0]
+        assert np.array_equal(codes[b].cpu().numpy().view(np.uint64), orc.encode(code, m))
+    enc.close()
