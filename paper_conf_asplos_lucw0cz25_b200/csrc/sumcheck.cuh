@@ -486,6 +486,10 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
     }
 }
 
+#ifndef BZK_PF_DIST
+#define BZK_PF_DIST 1   // prefetch distance in loop iterations (grid strides): 1 beats 2 and 4
+#endif
+
 // L2 bulk prefetch of a contiguous byte range (cp.async.bulk.prefetch, sm_90+; no registers, no smem)
 __device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
@@ -676,7 +680,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
 #pragma unroll
         for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
         for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
-            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
+            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + BZK_PF_DIST * stride);
             fe a[D], sv[D];
             load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
             eval_one<D, DERIVE>(a, sv, uacc);
@@ -687,7 +691,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
         fe ha[D], hs[D];
         bool held = false;
         for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
-            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + 2 * stride);
+            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + BZK_PF_DIST * stride);
             fe a[D], sv[D];
             load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
             if (held) {
