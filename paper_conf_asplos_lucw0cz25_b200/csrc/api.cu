@@ -147,7 +147,7 @@ struct Plan {
 // tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
 // (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round; default: on for d >= 3 only)
 struct Knobs {
-    uint64_t ppt_max = 64, waves = 4;
+    uint64_t ppt_max = 256, waves = 4;   // ppt_max sweep 32..1024: 256 best for c2, c3, m0
     // L2 bulk prefetch: -1 = by degree.  d <= 2: off (the fused rounds then read exactly their bytes;
     // with it 1.5x, -6 % at c2, -2 % at m0); d >= 3: on (IMAD-bound, +2 % at c3).  DESIGN.md sec. 8.
     int prefetch = -1;
