@@ -813,9 +813,21 @@ def main():
                 "step_frac": round(step_gmulmod / int_peak, 4),
                 "hbm_alg_frac": round(alg_bytes / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
                 "hbm_peak_gbs": hbm_peak}
+    # the dominant kernel's bound: the larger of its algorithmic IMAD time and HBM time at the peaks
+    # (d = 1 fused rounds move 192 B per 2 products: HBM-bound; d >= 2 BN254 rounds: IMAD-bound)
+    t_alu = mulmods_per_launch / (int_peak * 1e9)
+    t_hbm = bytes_per_launch / (hbm_peak * 1e9)
+    ach_gbs = bytes_per_launch / avg_launch_s / 1e9
+    roofline["alu_time_at_peak_ms"] = round(t_alu * 1000, 4)
+    roofline["hbm_time_at_peak_ms"] = round(t_hbm * 1000, 4)
+    if not gl and t_hbm > t_alu:
+        roofline.update({"bound": "hbm", "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
+                         "frac": round(ach_gbs / hbm_peak, 4),
+                         "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); this kernel's algorithmic "
+                                        "HBM time exceeds its IMAD time at the roofs",
+                         "alu_gmulmod_s": round(achieved, 2), "alu_frac": round(achieved / int_peak, 4)})
     if gl:
         # Goldilocks (8-byte elements): the dominant kernel streams; its roof is HBM bandwidth
-        ach_gbs = bytes_per_launch / avg_launch_s / 1e9
         roofline.update({"bound": "hbm", "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
                          "frac": round(ach_gbs / hbm_peak, 4),
                          "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); achieved = algorithmic bytes per "
