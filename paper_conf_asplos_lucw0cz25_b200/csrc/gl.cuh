@@ -247,7 +247,7 @@ __device__ __forceinline__ void load_pair(const uint64_t *src, uint64_t *dst, ui
 #define GL_OCC 3
 #endif
 #ifndef GL_SPLIT
-#define GL_SPLIT 1   // fused LSB rounds: issue every raw load of an iteration before the folds
+#define GL_SPLIT 1   // fused rounds (both orders): issue every raw load of an iteration before the folds
 #endif
 #ifndef GL_MLP_FUSED
 #define GL_MLP_FUSED 2   // pairs per iteration of the split fused loop (g2: 2 -> fused 0.86 of HBM, 4 -> 0.83)
@@ -302,6 +302,35 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
                     bb[q][m] = fold(raw[q][m][1].x, raw[q][m][1].y, r);
                     *reinterpret_cast<ulonglong2 *>(dst + (size_t)m * (2 * h) + 2 * (j + q * stride)) =
                         make_ulonglong2(a[q][m], bb[q][m]);
+                }
+#pragma unroll
+            for (int q = 0; q < MF; ++q) eval_pair<D>(a[q], bb[q], GL_ACC);
+        }
+    }
+    if (!FIRST && ORDER == 1) {
+        // MSB (Alg. 1 pairing): fold pairs (x, x + 2h), this round pairs (j, j + h)
+        for (; j + (MF - 1) * stride < h; j += MF * stride) {
+            uint64_t x[MF][D][4];
+#pragma unroll
+            for (int q = 0; q < MF; ++q)
+#pragma unroll
+                for (int m = 0; m < D; ++m) {
+                    const uint64_t *T = src + (size_t)m * (4 * h) + (j + q * stride);
+                    x[q][m][0] = __ldcs(T);
+                    x[q][m][1] = __ldcs(T + 2 * h);
+                    x[q][m][2] = __ldcs(T + h);
+                    x[q][m][3] = __ldcs(T + 3 * h);
+                }
+            uint64_t a[MF][D], bb[MF][D];
+#pragma unroll
+            for (int q = 0; q < MF; ++q)
+#pragma unroll
+                for (int m = 0; m < D; ++m) {
+                    a[q][m] = fold(x[q][m][0], x[q][m][1], r);
+                    bb[q][m] = fold(x[q][m][2], x[q][m][3], r);
+                    uint64_t *U = dst + (size_t)m * (2 * h);
+                    U[j + q * stride] = a[q][m];
+                    U[j + q * stride + h] = bb[q][m];
                 }
 #pragma unroll
             for (int q = 0; q < MF; ++q) eval_pair<D>(a[q], bb[q], GL_ACC);
