@@ -950,17 +950,18 @@ bzk_status encoder_create_impl(bzk_ctx *ctx, const bzk_code *c, bzk_encoder **ou
 }
 
 cudaError_t spmv(bzk_ctx *ctx, const SellDev &M, const fe *src, fe *dst, uint64_t stride, uint64_t nb, cudaStream_t s) {
-    const uint32_t warps = BZK_ENC_TPB / 32;
-    const uint64_t per_launch = 65535ull * BZK_ENC_K;   // gridDim.y limit
+    const uint32_t warps = BZK_ENC_TPB / 32 / BZK_ENC_G;   // slices per CTA
+    const uint64_t per_launch = 65535ull * BZK_ENC_K * BZK_ENC_G;   // gridDim.y limit
     for (uint64_t c0 = 0; c0 < nb; c0 += per_launch) {
         const uint64_t n = std::min<uint64_t>(per_launch, nb - c0);
         enc::SpmvParams p;
         p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
         p.slices = M.slices; p.src = src + c0 * stride; p.dst = dst + c0 * stride; p.stride = stride; p.batch = n;
-        dim3 grid((M.slices + warps - 1) / warps, (uint32_t)((n + BZK_ENC_K - 1) / BZK_ENC_K));
+        dim3 grid((M.slices + warps - 1) / warps,
+                  (uint32_t)((n + BZK_ENC_K * BZK_ENC_G - 1) / (BZK_ENC_K * BZK_ENC_G)));
         ProfScope ps_(ctx, s, 8);
         ++ctx->launches;
-        cudaError_t e = enc_launch_spmv(grid, warps * 32, s, p);
+        cudaError_t e = enc_launch_spmv(grid, BZK_ENC_TPB, s, p);
         if (e != cudaSuccess) return e;
     }
     return cudaSuccess;

@@ -86,12 +86,23 @@ __device__ __forceinline__ fe ld_fe_hint(const fe *p, uint64_t pol) {
 #define BZK_ENC_MINB 1   // min resident CTAs per SM for the register allocator (1 = unconstrained)
 #endif
 
+// BZK_ENC_G codeword groups per CTA (default 1): with G = 2 the CTA's warps pair up on the same slice
+// for two different codeword groups, so the second warp's weight loads can hit L1.  Measured slower
+// (G = 2: 3,167, G = 4: 2,638 vs 3,388 codes/s): the larger live source-vector set costs more L2 hits
+// than the shared weights save.
+#ifndef BZK_ENC_G
+#define BZK_ENC_G 1
+#endif
+
 template <int K, int U>
 __global__ void __launch_bounds__(BZK_ENC_TPB, BZK_ENC_MINB) k_spmv(SpmvParams p) {
     const uint32_t lane = threadIdx.x & 31;
-    const uint32_t slice = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    constexpr uint32_t SPC = BZK_ENC_TPB / 32 / BZK_ENC_G;   // slices per CTA
+    const uint32_t warp = threadIdx.x >> 5;
+    const uint32_t slice = blockIdx.x * SPC + warp % SPC;
     if (slice >= p.slices) return;
-    const uint64_t b0 = (uint64_t)blockIdx.y * K;
+    const uint64_t b0 = ((uint64_t)blockIdx.y * BZK_ENC_G + warp / SPC) * K;
+    if (b0 >= p.batch) return;
     const uint32_t row = p.perm[(size_t)slice * 32 + lane];
     const uint32_t W = p.slice_w[slice];
     const uint64_t off = p.slice_off[slice] + lane;
