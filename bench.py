@@ -707,7 +707,8 @@ def main():
         kk = max(1, (k - 1).bit_length())          # generator tables have 2^kk >= k entries
         g = torch.empty((B, 1, 1 << kk, 4), dtype=torch.int64, device="cuda")
         bzk.bzk_generate(g, B, 1, kk, first, "uniform", data_seed=0x5052470000000000, stream=stream)
-        out["challenges"].copy_(g[:, 0, :k, :])
+        with torch.cuda.stream(stream):          # ordered after the generator on the same stream
+            out["challenges"].copy_(g[:, 0, :k, :])
         stream.synchronize()
     batch = prover.batch(tables, k, d, order, None, first, flags, out)
 

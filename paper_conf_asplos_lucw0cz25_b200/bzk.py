@@ -33,7 +33,8 @@ BZK_MERKLE_COMPRESS, BZK_MERKLE_SHA256 = 0, 1
 EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
            "bzk_strerror", "bzk_last_error", "bzk_generate", "bzk_profile_enable", "bzk_profile_read",
            "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version",
-           "bzk_merkle", "bzk_generate_blocks", "bzk_encoder_create", "bzk_encoder_destroy", "bzk_encode"]
+           "bzk_merkle", "bzk_generate_blocks", "bzk_encoder_create", "bzk_encoder_destroy", "bzk_encode",
+           "bzk_debug_gl"]
 
 
 class BzkError(RuntimeError):
@@ -97,6 +98,7 @@ def lib():
         L.bzk_launch_count.restype = u64
         L.bzk_debug_field.argtypes = [i32, u64, vp, vp, vp, vp]
         L.bzk_debug_sha256.argtypes = [vp, u32, u64, vp, vp]
+        L.bzk_debug_gl.argtypes = [i32, u64, vp, vp, vp, vp]
         L.bzk_debug_bench.argtypes = [i32, u32, ctypes.POINTER(ctypes.c_double), vp]
         L.bzk_version.restype = ctypes.c_char_p
         L.bzk_merkle.argtypes = [vp, ctypes.POINTER(bzk_merkle_batch), vp]
@@ -107,7 +109,7 @@ def lib():
         L.bzk_encode.argtypes = [vp, vp, vp, u64, u32, u32, vp]
         for name in ("bzk_create", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
                      "bzk_generate", "bzk_profile_enable", "bzk_profile_read", "bzk_debug_field",
-                     "bzk_debug_sha256", "bzk_debug_bench", "bzk_merkle", "bzk_generate_blocks",
+                     "bzk_debug_sha256", "bzk_debug_bench", "bzk_debug_gl", "bzk_merkle", "bzk_generate_blocks",
                      "bzk_encoder_create", "bzk_encode"):
             getattr(L, name).restype = i32
         _lib = L
@@ -253,6 +255,10 @@ def bzk_launch_count(ctx, reset: bool = False) -> int:
 
 def bzk_debug_field(op: int, n: int, a, b, out, stream=None) -> None:
     _check(lib().bzk_debug_field(op, n, ptr(a), ptr(b), ptr(out), _stream_handle(stream)))
+
+
+def bzk_debug_gl(op: int, n: int, a, b, out, stream=None) -> None:
+    _check(lib().bzk_debug_gl(op, n, ptr(a), ptr(b), ptr(out), _stream_handle(stream)))
 
 
 def bzk_debug_sha256(msgs, msg_len: int, n: int, out, stream=None) -> None:

@@ -79,6 +79,10 @@ struct bzk_ctx {
     cudaGraphExec_t graph_exec = nullptr;
     std::vector<unsigned char> graph_key;
     uint64_t graph_launches = 0;      // kernel launches inside the cached graph
+    // end of the context's last call: every call first waits on it, so calls issued on different
+    // streams never overlap on the shared workspace (ps, tickets, partials, ping-pong buffers)
+    cudaEvent_t ev_done = nullptr;
+    bool ev_done_recorded = false;
 };
 
 namespace {
@@ -180,6 +184,14 @@ uint32_t ctas_for(uint64_t h, uint64_t nb) {
     return (uint32_t)c;
 }
 
+// CTAs per proof over every global round i < i0 (ctas_for is not monotone in h: ppt is floored).
+// The partials buffer is sized with this maximum; each round indexes it with its own stride.
+uint32_t max_round_ctas(uint32_t k, uint32_t i0, uint64_t nb) {
+    uint32_t c = 1;
+    for (uint32_t i = 1; i < i0; ++i) c = std::max(c, ctas_for(1ull << (k - i), nb));
+    return c;
+}
+
 uint32_t cluster_for(uint32_t ctas) {
     uint32_t c = 1;
     while (c * 2 <= knobs().cluster && ctas % (c * 2) == 0) c *= 2;
@@ -191,7 +203,8 @@ size_t align_up(size_t x) { return (x + 255) & ~(size_t)255; }
 bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
     if (!b) return fail(ctx, BZK_EINVAL, "batch is NULL");
     if (b->num_vars > 30) return fail(ctx, BZK_EINVAL, "num_vars must be <= 30");
-    if (b->degree < 1 || b->degree > 4) return fail(ctx, BZK_EINVAL, "degree must be in 1..4");
+    if (b->degree < 1) return fail(ctx, BZK_EINVAL, "degree must be >= 1");
+    if (b->degree > 4) return fail(ctx, BZK_EUNSUPPORTED, "degree > 4 is not built (kernels exist for d = 1..4)");
     if (b->order > 1) return fail(ctx, BZK_EINVAL, "order must be BZK_ORDER_LSB or BZK_ORDER_MSB");
     if (b->batch == 0) return fail(ctx, BZK_EINVAL, "batch must be >= 1");
     if (!b->seed) return fail(ctx, BZK_EINVAL, "seed is NULL");
@@ -200,7 +213,7 @@ bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
         return fail(ctx, BZK_EINVAL, "round_evals/challenges is NULL");
     if (!b->final_evals) return fail(ctx, BZK_EINVAL, "final_evals is NULL");
     if (b->tables_mem > 1 || b->outputs_mem > 1) return fail(ctx, BZK_EINVAL, "bad *_mem value");
-    if (b->first_index + b->batch > (1ull << 28)) return fail(ctx, BZK_EINVAL, "global index must be < 2^28");
+    if (b->batch - 1 > ~0ull - b->first_index) return fail(ctx, BZK_EINVAL, "first_index + batch exceeds 2^64");
     // BN254 kernels access elements with 256-bit loads/stores: device buffers must be 32-byte aligned
     if (!(b->flags & BZK_F_FIELD_GOLDILOCKS)) {
         auto mis = [](const void *q) { return q && ((uintptr_t)q & 31u); };
@@ -246,7 +259,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
         size_t s = std::max(sizeof(ProofState), sizeof(gl::State)) + 4;
-        uint32_t c = P.k ? ctas_for(1ull << (P.k - 1), bw) : 1;
+        uint32_t c = P.k ? max_round_ctas(P.k, P.i0, bw) : 1;
         s += (size_t)c * (P.D + 1) * P.esz;
         if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * P.esz;
         if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * P.esz;
@@ -265,8 +278,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     uint64_t nw = (P.B + bw - 1) / bw;
     bw = (P.B + nw - 1) / nw;
     P.Bw = bw; P.nwaves = nw;
-    P.cmax = P.k ? std::max(ctas_for(1ull << (P.k - 1), bw),
-                            ctas_for(1ull << (P.k - 1), P.B - (nw - 1) * bw)) : 1;
+    P.cmax = P.k ? std::max(max_round_ctas(P.k, P.i0, bw), max_round_ctas(P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
 
     size_t off = 0;
     P.off_seed = off; off += 256;
@@ -281,9 +293,31 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     return BZK_OK;
 }
 
+// a cached CUDA graph holds raw workspace / staging pointers: drop it whenever they move
+void drop_graph(bzk_ctx *ctx) {
+    if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
+    ctx->graph_exec = nullptr;
+    ctx->graph_key.clear();
+    ctx->graph_launches = 0;
+}
+
+// order this call after the context's previous call (whatever stream it ran on)
+bzk_status call_begin(bzk_ctx *ctx, cudaStream_t s) {
+    if (ctx->ev_done_recorded) CK(cudaStreamWaitEvent(s, ctx->ev_done, 0));
+    return BZK_OK;
+}
+
+bzk_status call_end(bzk_ctx *ctx, cudaStream_t s) {
+    CK(cudaEventRecord(ctx->ev_done, s));
+    ctx->ev_done_recorded = true;
+    return BZK_OK;
+}
+
 bzk_status ensure_ws(bzk_ctx *ctx, size_t bytes) {
     if (ctx->ws_size >= bytes) return BZK_OK;
     ctx->auto_limit = 0;
+    drop_graph(ctx);
+    cudaDeviceSynchronize();   // earlier calls (any stream) may still use the old workspace
     if (ctx->ws) { cudaFree(ctx->ws); ctx->ws = nullptr; ctx->ws_size = 0; }
     cudaError_t e = cudaMalloc(&ctx->ws, bytes);
     if (e != cudaSuccess) {
@@ -298,6 +332,7 @@ bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
     if (bytes == 0 || ctx->stage_size >= bytes) return BZK_OK;
     cudaDeviceSynchronize();   // slots may still be in use by earlier work
     ctx->auto_limit = 0;
+    drop_graph(ctx);
     for (int i = 0; i < 2; ++i) {
         if (ctx->stage[i]) cudaFree(ctx->stage[i]);
         ctx->stage[i] = nullptr;
@@ -589,10 +624,12 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
     if (st) return st;
     st = ensure_stage(ctx, stage_need);
     if (st) return st;
+    st = call_begin(ctx, s);
+    if (st) return st;
     if (graph && ctx->graph_exec && ctx->graph_key == key) {
         CK(cudaGraphLaunch(ctx->graph_exec, s));
         ctx->launches += ctx->graph_launches;
-        return BZK_OK;
+        return call_end(ctx, s);
     }
     if (graph) {
         if (ctx->graph_exec) { cudaGraphExecDestroy(ctx->graph_exec); ctx->graph_exec = nullptr; }
@@ -602,7 +639,8 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
     for (size_t j = 0; j < njobs; ++j) {
         st = enqueue_job(ctx, &jobs[j], plans[j], s);
         if (st) {
-            if (graph) { cudaGraph_t g; cudaStreamEndCapture(s, &g); if (g) cudaGraphDestroy(g); }
+            if (graph) { cudaGraph_t g = nullptr; cudaStreamEndCapture(s, &g); if (g) cudaGraphDestroy(g); }
+            else call_end(ctx, s);
             return st;
         }
     }
@@ -616,6 +654,8 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
         ctx->graph_launches = ctx->launches - l0;
         CK(cudaGraphLaunch(ctx->graph_exec, s));
     }
+    st = call_end(ctx, s);
+    if (st) return st;
     if (need_sync) CK(cudaStreamSynchronize(s));
     return BZK_OK;
 }
@@ -710,6 +750,8 @@ bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) 
     if (st) return st;
     st = ensure_stage(ctx, host_in ? align_up(bw * blk_bytes) : 0);
     if (st) return st;
+    st = call_begin(ctx, s);
+    if (st) return st;
     char *ws = (char *)ctx->ws;
     uint8_t *roots_all = host_out ? (uint8_t *)(ws + off_roots) : m->roots;
 
@@ -797,6 +839,8 @@ bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) 
         CK(cudaMemcpyAsync(m->roots, roots_all, B * 32, cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(ctx->d2h_stream));
     }
+    st = call_end(ctx, s);
+    if (st) return st;
     if (host_in || host_out || (m->flags & BZK_F_SYNC)) CK(cudaStreamSynchronize(s));
     return BZK_OK;
 }
@@ -950,15 +994,15 @@ bzk_status encoder_create_impl(bzk_ctx *ctx, const bzk_code *c, bzk_encoder **ou
 }
 
 cudaError_t spmv(bzk_ctx *ctx, const SellDev &M, const fe *src, fe *dst, uint64_t stride, uint64_t nb, cudaStream_t s) {
-    const uint32_t warps = BZK_ENC_TPB / 32 / BZK_ENC_G;   // slices per CTA
-    const uint64_t per_launch = 65535ull * BZK_ENC_K * BZK_ENC_G;   // gridDim.y limit
+    const uint32_t warps = BZK_ENC_TPB / 32;   // slices per CTA
+    const uint64_t per_launch = 65535ull * BZK_ENC_K;   // gridDim.y limit
     for (uint64_t c0 = 0; c0 < nb; c0 += per_launch) {
         const uint64_t n = std::min<uint64_t>(per_launch, nb - c0);
         enc::SpmvParams p;
         p.perm = M.perm; p.slice_off = M.slice_off; p.slice_w = M.slice_w; p.col = M.col; p.val = M.val;
         p.slices = M.slices; p.src = src + c0 * stride; p.dst = dst + c0 * stride; p.stride = stride; p.batch = n;
         dim3 grid((M.slices + warps - 1) / warps,
-                  (uint32_t)((n + BZK_ENC_K * BZK_ENC_G - 1) / (BZK_ENC_K * BZK_ENC_G)));
+                  (uint32_t)((n + BZK_ENC_K - 1) / BZK_ENC_K));
         ProfScope ps_(ctx, s, 8);
         ++ctx->launches;
         cudaError_t e = enc_launch_spmv(grid, BZK_ENC_TPB, s, p);
@@ -993,7 +1037,11 @@ bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint
     const size_t cw = (size_t)2 * n * 32;   // bytes per codeword
     if (codes_mem == BZK_MEM_DEVICE) {
         if ((uintptr_t)codes & 31u) return fail(ctx, BZK_EINVAL, "device codes must be 32-byte aligned");
-        bzk_status st = encode_wave(ctx, E, (fe *)codes, batch, s);
+        bzk_status st = call_begin(ctx, s);
+        if (st) return st;
+        st = encode_wave(ctx, E, (fe *)codes, batch, s);
+        if (st) return st;
+        st = call_end(ctx, s);
         if (st) return st;
         if (flags & BZK_F_SYNC) CK(cudaStreamSynchronize(s));
         return BZK_OK;
@@ -1014,6 +1062,8 @@ bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint
     const uint64_t nw = (batch + bw - 1) / bw;
     bw = (batch + nw - 1) / nw;
     bzk_status st = ensure_stage(ctx, align_up(bw * cw));
+    if (st) return st;
+    st = call_begin(ctx, s);
     if (st) return st;
     for (uint64_t w = 0; w < nw; ++w) {
         const uint64_t b0 = w * bw, nb = std::min<uint64_t>(bw, batch - b0);
@@ -1041,6 +1091,8 @@ bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint
         ctx->slot_used[slot] = true;
     }
     CK(cudaStreamSynchronize(ctx->d2h_stream));
+    st = call_end(ctx, s);
+    if (st) return st;
     CK(cudaStreamSynchronize(s));
     return BZK_OK;
 }
@@ -1061,6 +1113,78 @@ __global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *
             default: r = fe_reduce_256(x); break;
         }
         st_fe(out + i, r);
+    }
+}
+
+// Lazy hot-path primitives at their stated operand bounds (bzk_debug_field ops 7..16; the results are
+// the RAW lazy values, so the host can check both the congruence and the bound).  64 threads per CTA:
+// fixmul_lz reads its table K from shared memory.
+__global__ void __launch_bounds__(64) k_debug_lazy(int op, uint64_t n, const fe *a, const fe *b, fe *out, uint32_t zero) {
+    __shared__ __align__(16) fe sK[64][8];
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const fe x = ld_fe(a + i), y = ld_fe(b + i);
+        fe r;
+        switch (op) {
+            case 7: r = mont_mul_lz(x, y); break;                                       // x y R^-1 + q p
+            case 8: r = mont_mul2_lz(x, y, ld_fe(a + n - 1 - i), ld_fe(b + n - 1 - i)); break;
+            case 9: case 16: {                                                          // K_j = r 2^(32 j + 64)
+                const fe rr = op == 9 ? y : ld_fe(b + n + i);
+                const fe rm = mont_mul(rr, fe_const(2));                                // r R
+                fe pw = fe_zero();
+                pw.l[0] = 1;
+                for (int e = 0; e < 64; ++e) pw = fe_add(pw, pw);                      // 2^64 mod p
+                for (int j = 0; j < 8; ++j) {
+                    sK[threadIdx.x][j] = mont_mul(rm, pw);
+                    for (int e = 0; e < 32; ++e) pw = fe_add(pw, pw);
+                }
+                __syncwarp();
+                r = op == 9 ? fixmul_lz(x, sK[threadIdx.x], zero) : fold_fx(x, y, sK[threadIdx.x], zero);
+                __syncwarp();
+                break;
+            }
+            case 10: {                                                                  // sum of 64 products
+                acc17 acc = acc17_zero();
+                for (uint64_t j = 0; j < 64; ++j) mul_acc(acc, ld_fe(a + (i + j) % n), ld_fe(b + (i + j) % n));
+                r = acc17_to_fe(acc);
+                break;
+            }
+            case 11: {                                                                  // raw 544-bit value
+                acc17 acc;
+                for (int w = 0; w < 8; ++w) { acc.w[w] = x.l[w]; acc.w[8 + w] = y.l[w]; }
+                acc.w[16] = x.l[7];
+                r = acc17_to_fe(acc);
+                break;
+            }
+            case 12: r = lz_sub(y, x); break;                                           // y + 2p - x
+            case 13: r = lz_red(x); break;                                              // x < 4p -> < 2p
+            case 14: { acc9 c; c.lo = x; c.hi = y.l[0]; r = acc9_to_fe(c); break; }   // lo + hi 2^256
+            default: r = lz_add(x, y); break;                                           // 15: plain add
+        }
+        st_fe(out + i, r);
+    }
+}
+
+// Goldilocks primitives (gl.cuh), bzk_debug_gl
+__global__ void k_debug_gl(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out) {
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t x = a[i], y = b[i];
+        uint64_t r;
+        switch (op) {
+            case 0: r = gl::add(x, y); break;
+            case 1: r = gl::sub(x, y); break;
+            case 2: r = gl::mul(x, y); break;
+            case 3: r = gl::add_lazy(x, y); break;
+            case 4: r = gl::reduce128(x, y); break;                                   // x = hi, y = lo
+            case 5: r = gl::fold(x, y, b[n + i]); break;                                // x + r (y - x)
+            case 6: {                                                                   // 64 products, lazy
+                gl::Wide w{0, 0, 0};
+                for (uint64_t j = 0; j < 64; ++j) gl::wide_mac(w, a[(i + j) % n], b[(i + j) % n]);
+                r = gl::wide_reduce(w);
+                break;
+            }
+            default: r = gl::wide_reduce(gl::Wide{x, y, b[n + i] & 0xffffffffull}); break;   // 7: raw 160-bit
+        }
+        out[i] = r;
     }
 }
 
@@ -1210,6 +1334,34 @@ const char *bzk_strerror(bzk_status s) {
 
 const char *bzk_last_error(const bzk_ctx *ctx) { return ctx ? ctx->last_error.c_str() : ""; }
 
+}  // extern "C"
+
+namespace {
+// frees everything a (possibly partially constructed) context owns
+void ctx_free(bzk_ctx *ctx) {
+    if (ctx->ws) cudaFree(ctx->ws);
+    if (ctx->d_flag) cudaFree(ctx->d_flag);
+    if (ctx->consts) cudaFree(ctx->consts);
+    for (int i = 0; i < 2; ++i)
+        if (ctx->stage[i]) cudaFree(ctx->stage[i]);
+    for (int i = 0; i < 2; ++i) {
+        if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
+        if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
+        if (ctx->ev_nodes_ready[i]) cudaEventDestroy(ctx->ev_nodes_ready[i]);
+        if (ctx->ev_nodes_copied[i]) cudaEventDestroy(ctx->ev_nodes_copied[i]);
+    }
+    if (ctx->ev_done) cudaEventDestroy(ctx->ev_done);
+    if (ctx->d2h_stream) cudaStreamDestroy(ctx->d2h_stream);
+    if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
+    for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+    for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+    if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
+    delete ctx;
+}
+}  // namespace
+
+extern "C" {
+
 bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
     if (!out) return BZK_EINVAL;
     *out = nullptr;
@@ -1223,30 +1375,28 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
     ctx->device = device;
     ctx->workspace_limit = workspace_limit;
     cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device);
-    if (cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaMalloc(&ctx->d_flag, 4) != cudaSuccess ||
-        cudaMalloc(&ctx->consts, sizeof(fe) * kNumConsts) != cudaSuccess) {
-        delete ctx;
-        return BZK_ECUDA;
+    bool ok = cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaStreamCreateWithFlags(&ctx->d2h_stream, cudaStreamNonBlocking) == cudaSuccess &&
+              cudaMalloc(&ctx->d_flag, 4) == cudaSuccess &&
+              cudaMalloc(&ctx->consts, sizeof(fe) * kNumConsts) == cudaSuccess &&
+              cudaEventCreateWithFlags(&ctx->ev_done, cudaEventDisableTiming) == cudaSuccess;
+    for (int i = 0; ok && i < 2; ++i)
+        ok = cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&ctx->ev_consumed[i], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&ctx->ev_nodes_ready[i], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&ctx->ev_nodes_copied[i], cudaEventDisableTiming) == cudaSuccess;
+    if (ok) {
+        set_kernel_attrs<1>();
+        set_kernel_attrs<2>();
+        set_kernel_attrs<3>();
+        set_kernel_attrs<4>();
+        gl_set_attrs();
+        k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
+        ok = cudaStreamSynchronize(ctx->copy_stream) == cudaSuccess;
     }
-    set_kernel_attrs<1>();
-    set_kernel_attrs<2>();
-    set_kernel_attrs<3>();
-    set_kernel_attrs<4>();
-    gl_set_attrs();
-    k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
-    if (cudaStreamSynchronize(ctx->copy_stream) != cudaSuccess) {
-        delete ctx;
-        return BZK_ECUDA;
-    }
-    for (int i = 0; i < 2; ++i) {
-        cudaEventCreateWithFlags(&ctx->ev_copied[i], cudaEventDisableTiming);
-        cudaEventCreateWithFlags(&ctx->ev_consumed[i], cudaEventDisableTiming);
-        cudaEventCreateWithFlags(&ctx->ev_nodes_ready[i], cudaEventDisableTiming);
-        cudaEventCreateWithFlags(&ctx->ev_nodes_copied[i], cudaEventDisableTiming);
-    }
-    if (cudaStreamCreateWithFlags(&ctx->d2h_stream, cudaStreamNonBlocking) != cudaSuccess) {
-        delete ctx;
+    if (!ok) {
+        cudaGetLastError();
+        ctx_free(ctx);
         return BZK_ECUDA;
     }
     *out = ctx;
@@ -1257,23 +1407,7 @@ void bzk_destroy(bzk_ctx *ctx) {
     if (!ctx) return;
     cudaSetDevice(ctx->device);
     cudaDeviceSynchronize();
-    if (ctx->ws) cudaFree(ctx->ws);
-    if (ctx->d_flag) cudaFree(ctx->d_flag);
-    if (ctx->consts) cudaFree(ctx->consts);
-    for (int i = 0; i < 2; ++i)
-        if (ctx->stage[i]) cudaFree(ctx->stage[i]);
-    for (int i = 0; i < 2; ++i) {
-        if (ctx->ev_copied[i]) cudaEventDestroy(ctx->ev_copied[i]);
-        if (ctx->ev_consumed[i]) cudaEventDestroy(ctx->ev_consumed[i]);
-        if (ctx->ev_nodes_ready[i]) cudaEventDestroy(ctx->ev_nodes_ready[i]);
-        if (ctx->ev_nodes_copied[i]) cudaEventDestroy(ctx->ev_nodes_copied[i]);
-    }
-    if (ctx->d2h_stream) cudaStreamDestroy(ctx->d2h_stream);
-    if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
-    for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
-    for (auto e : ctx->ev_pool) cudaEventDestroy(e);
-    if (ctx->copy_stream) cudaStreamDestroy(ctx->copy_stream);
-    delete ctx;
+    ctx_free(ctx);
 }
 
 bzk_status bzk_workspace_size(bzk_ctx *ctx, const bzk_batch *batch, size_t *bytes) {
@@ -1283,7 +1417,7 @@ bzk_status bzk_workspace_size(bzk_ctx *ctx, const bzk_batch *batch, size_t *byte
     Plan P;
     st = make_plan(ctx, batch, P);
     if (st) return st;
-    *bytes = P.total;
+    *bytes = P.total + 2 * P.stage_bytes;   // workspace + the loader's two staging slots (host tables)
     return BZK_OK;
 }
 
@@ -1312,7 +1446,7 @@ bzk_status bzk_sync(bzk_ctx *ctx) {
 
 bzk_status bzk_generate(uint64_t *dst, uint64_t batch, uint32_t d, uint32_t k, uint64_t first_index,
                         uint32_t dist, uint64_t data_seed, void *cuda_stream) {
-    if (!dst || k > 30 || d < 1 || d > 15 || dist > 3 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
+    if (!dst || k > 30 || d < 1 || d > 15 || dist > 5 || first_index + batch > (1ull << 28)) return BZK_EINVAL;
     k_generate<<<kSMs * 16, 256, 0, (cudaStream_t)cuda_stream>>>(dst, batch, d, k, first_index, dist, data_seed);
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }
@@ -1385,9 +1519,20 @@ uint64_t bzk_launch_count(bzk_ctx *ctx, int reset) {
 
 bzk_status bzk_debug_field(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out,
                            void *cuda_stream) {
-    if (op < 0 || op > 6 || !a || !out || (op != 4 && !b)) return BZK_EINVAL;
+    if (op < 0 || op > 16 || !a || !out || (op != 4 && !b)) return BZK_EINVAL;
     if (n == 0) return BZK_OK;
+    if (op >= 7) {
+        k_debug_lazy<<<kSMs * 4, 64, 0, (cudaStream_t)cuda_stream>>>(op, n, (const fe *)a, (const fe *)b, (fe *)out, 0u);
+        return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+    }
     k_debug_field<<<kSMs * 8, 256, 0, (cudaStream_t)cuda_stream>>>(op, n, (const fe *)a, (const fe *)b, (fe *)out);
+    return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
+}
+
+bzk_status bzk_debug_gl(int op, uint64_t n, const uint64_t *a, const uint64_t *b, uint64_t *out, void *cuda_stream) {
+    if (op < 0 || op > 7 || !a || !b || !out) return BZK_EINVAL;
+    if (n == 0) return BZK_OK;
+    k_debug_gl<<<kSMs * 8, 256, 0, (cudaStream_t)cuda_stream>>>(op, n, a, b, out);
     return cudaGetLastError() == cudaSuccess ? BZK_OK : BZK_ECUDA;
 }
 

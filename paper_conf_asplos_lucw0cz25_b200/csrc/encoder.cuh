@@ -46,11 +46,8 @@ struct SpmvParams {
 #define BZK_ENC_U 2      // entries per loop iteration (their gathers are in flight together)
 #endif
 
-// BZK_ENC_L2HINT=1: gathers carry an L2 evict_last policy and the weight stream evict_first, so the
-// streamed weights do not push the live source vectors out of L2.
-#ifndef BZK_ENC_L2HINT
-#define BZK_ENC_L2HINT 1
-#endif
+// Gathers carry an L2 evict_last policy and the weight stream evict_first, so the streamed weights
+// do not push the live source vectors out of L2 (+1-3 % on B200).
 
 __device__ __forceinline__ uint64_t l2_policy_last() {
     uint64_t pol;
@@ -70,45 +67,26 @@ __device__ __forceinline__ fe ld_fe_hint(const fe *p, uint64_t pol) {
         : "l"(p), "l"(pol));
     return r;
 }
-#if BZK_ENC_L2HINT
 #define BZK_ENC_GATHER(x, ptr) (x) = ld_fe_hint((ptr), pol_last)
 #define BZK_ENC_WEIGHT(ptr) ld_fe_hint((ptr), pol_first)
-#else
-#define BZK_ENC_GATHER(x, ptr) BZK_LD8(".nc", x, ptr)
-#define BZK_ENC_WEIGHT(ptr) ld_fe_stream(ptr)
-#endif
 
 #ifndef BZK_ENC_TPB
 #define BZK_ENC_TPB 128  // threads per CTA (4 warp slices; finer occupancy steps at ~100 registers)
 #endif
 
-#ifndef BZK_ENC_MINB
-#define BZK_ENC_MINB 1   // min resident CTAs per SM for the register allocator (1 = unconstrained)
-#endif
-
-// BZK_ENC_G codeword groups per CTA (default 1): with G = 2 the CTA's warps pair up on the same slice
-// for two different codeword groups, so the second warp's weight loads can hit L1.  Measured slower
-// (G = 2: 3,167, G = 4: 2,638 vs 3,388 codes/s): the larger live source-vector set costs more L2 hits
-// than the shared weights save.
-#ifndef BZK_ENC_G
-#define BZK_ENC_G 1
-#endif
-
 template <int K, int U>
-__global__ void __launch_bounds__(BZK_ENC_TPB, BZK_ENC_MINB) k_spmv(SpmvParams p) {
+__global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
     const uint32_t lane = threadIdx.x & 31;
-    constexpr uint32_t SPC = BZK_ENC_TPB / 32 / BZK_ENC_G;   // slices per CTA
+    constexpr uint32_t SPC = BZK_ENC_TPB / 32;   // slices per CTA
     const uint32_t warp = threadIdx.x >> 5;
-    const uint32_t slice = blockIdx.x * SPC + warp % SPC;
+    const uint32_t slice = blockIdx.x * SPC + warp;
     if (slice >= p.slices) return;
-    const uint64_t b0 = ((uint64_t)blockIdx.y * BZK_ENC_G + warp / SPC) * K;
+    const uint64_t b0 = (uint64_t)blockIdx.y * K;
     if (b0 >= p.batch) return;
     const uint32_t row = p.perm[(size_t)slice * 32 + lane];
     const uint32_t W = p.slice_w[slice];
     const uint64_t off = p.slice_off[slice] + lane;
-#if BZK_ENC_L2HINT
     const uint64_t pol_last = l2_policy_last(), pol_first = l2_policy_first();
-#endif
     acc17 acc[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) acc[q] = acc17_zero();
@@ -145,92 +123,6 @@ __global__ void __launch_bounds__(BZK_ENC_TPB, BZK_ENC_MINB) k_spmv(SpmvParams p
             mul_acc(acc[q], w, x);
         }
     }
-    if (row == 0xffffffffu) return;
-#pragma unroll
-    for (int q = 0; q < K; ++q)
-        if (b0 + q < p.batch) st_fe(p.dst + (b0 + q) * p.stride + row, acc17_to_fe(acc[q]));
-}
-
-// BZK_ENC_ASYNC=1: the weight and the K gathers of each entry are staged through a per-thread ring of
-// S shared-memory slots by cp.async (LDGSTS: nothing held in registers while in flight), S entries
-// ahead of use, with the column indices loaded S entries before their gathers are issued -- so
-// 3 S 32-byte loads per thread are in flight instead of the 2 U gathers of k_spmv (ncu: k_spmv
-// stalled on gather latency at 82 % fma-heavy busy).  Chunk-major slots (chunk c of thread t at
-// (slot chunk index * blockDim + t) * 16) keep the shared-memory writes and reads conflict-free.
-// Measured SLOWER on B200 (2,897 vs 3,473 codes/s at S = 4: 122 registers and the LDGSTS/LDS overhead
-// cost more than the extra memory-level parallelism gains); bit-exact, kept as an option.
-#ifndef BZK_ENC_ASYNC
-#define BZK_ENC_ASYNC 0
-#endif
-#ifndef BZK_ENC_S
-#define BZK_ENC_S 4
-#endif
-
-__device__ __forceinline__ void cp_async16_hint(void *smem_dst, const void *gsrc, uint64_t pol) {
-    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(d), "l"(gsrc), "l"(pol)
-                 : "memory");
-}
-
-template <int K, int S>
-__global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv_async(SpmvParams p) {
-    extern __shared__ uint4 ring[];                 // [S][(K + 1) * 2 chunks][blockDim] x 16 B
-    constexpr int CH = (K + 1) * 2;
-    const uint32_t lane = threadIdx.x & 31, tid = threadIdx.x, nt = blockDim.x;
-    const uint32_t slice = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
-    if (slice >= p.slices) return;                  // whole warps leave together (slice is warp-uniform)
-    const uint64_t b0 = (uint64_t)blockIdx.y * K;
-    const uint32_t row = p.perm[(size_t)slice * 32 + lane];
-    const uint32_t W = p.slice_w[slice];
-    const uint64_t off = p.slice_off[slice] + lane;
-    const uint64_t pol_last = l2_policy_last(), pol_first = l2_policy_first();
-    const fe *src[K];
-#pragma unroll
-    for (int q = 0; q < K; ++q) src[q] = p.src + (b0 + q < p.batch ? b0 + q : b0) * p.stride;
-    auto issue = [&](uint32_t t, uint32_t c, int slot) {
-        if (t < W) {
-            const uint4 *wg = reinterpret_cast<const uint4 *>(p.val + off + (uint64_t)t * 32);
-            cp_async16_hint(&ring[(size_t)(slot * CH + 0) * nt + tid], wg, pol_first);
-            cp_async16_hint(&ring[(size_t)(slot * CH + 1) * nt + tid], wg + 1, pol_first);
-#pragma unroll
-            for (int q = 0; q < K; ++q) {
-                const uint4 *xg = reinterpret_cast<const uint4 *>(src[q] + c);
-                cp_async16_hint(&ring[(size_t)(slot * CH + 2 + 2 * q) * nt + tid], xg, pol_last);
-                cp_async16_hint(&ring[(size_t)(slot * CH + 3 + 2 * q) * nt + tid], xg + 1, pol_last);
-            }
-        }
-        cp_async_commit();                          // always commit: uniform group counting
-    };
-    auto ld_col = [&](uint32_t t) -> uint32_t { return t < W ? __ldg(p.col + off + (uint64_t)t * 32) : 0u; };
-    auto lds_fe = [&](int chunk0) -> fe {
-        const uint4 a = ring[(size_t)chunk0 * nt + tid], b = ring[(size_t)(chunk0 + 1) * nt + tid];
-        fe r;
-        r.l[0] = a.x; r.l[1] = a.y; r.l[2] = a.z; r.l[3] = a.w;
-        r.l[4] = b.x; r.l[5] = b.y; r.l[6] = b.z; r.l[7] = b.w;
-        return r;
-    };
-    acc17 acc[K];
-#pragma unroll
-    for (int q = 0; q < K; ++q) acc[q] = acc17_zero();
-    uint32_t cq[S];
-#pragma unroll
-    for (int s_ = 0; s_ < S; ++s_) issue(s_, ld_col(s_), s_);
-#pragma unroll
-    for (int s_ = 0; s_ < S; ++s_) cq[s_] = ld_col(S + s_);
-#pragma unroll 1
-    for (uint32_t t = 0; t < W; t += S) {
-#pragma unroll
-        for (int s_ = 0; s_ < S; ++s_) {
-            if (t + s_ >= W) break;
-            cp_async_wait<S - 1>();
-            const fe w = lds_fe(s_ * CH);
-#pragma unroll
-            for (int q = 0; q < K; ++q) mul_acc(acc[q], w, lds_fe(s_ * CH + 2 + 2 * q));
-            issue(t + s_ + S, cq[s_], s_);          // refill the slot just consumed (data already in acc)
-            cq[s_] = ld_col(t + s_ + 2 * S);
-        }
-    }
-    cp_async_wait<0>();
     if (row == 0xffffffffu) return;
 #pragma unroll
     for (int q = 0; q < K; ++q)

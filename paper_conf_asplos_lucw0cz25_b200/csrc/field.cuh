@@ -281,28 +281,10 @@ __device__ __forceinline__ void row_a(uint32_t A[9], const uint32_t a[8], uint32
         : "r"(a[0]), "r"(a[2]), "r"(a[4]), "r"(a[6]), "r"(bi));
 }
 
-// reduction chains: A += p_even * m (A0 -> 0), B += p_odd * m.
-// BN254 has p0 = 2^32 - 2^28 + 1 and -p^{-1} = -(2^28 + 1) mod 2^32, so the column-0 product
-// needs no multiplier: m = -(A0 + (A0 << 28)) and hi(A0 + m p0) = m - (m >> 4) + carry(A0 + m)
-// (exact: A0 + m p0 = 2^32 (m - (m >> 4)) + (A0 + m - (m << 28) mod 2^32), the last term being
-// 0 or 2^32 exactly as A0 + m carries).  Saves one IMAD and one IMAD.HI per row on the IMAD pipe.
-#ifndef BZK_M_ALU
-#define BZK_M_ALU 0      // 1: m via shift+add on the ALU pipe (fewer IMADs, longer dependency)
-#endif
-#ifndef BZK_P0_TRICK
-#define BZK_P0_TRICK 0   // 1: column-0 reduction product without IMAD.HI
-#endif
-__device__ __forceinline__ uint32_t mont_m(uint32_t a0) {
-#if !BZK_M_ALU
-    return a0 * BZK_NP0;
-#endif
-    uint32_t m;   // -(a0 + (a0 << 28)) on the ALU pipe (shift + add), kept out of the IMAD pipe
-    asm("{\n\t.reg .u32 t;\n\tshl.b32 t, %1, 28;\n\tadd.u32 t, t, %1;\n\tsub.u32 %0, 0, t;\n\t}" : "=r"(m) : "r"(a0));
-    return m;
-}
+// reduction chains: A += p_even * m (A0 -> 0), B += p_odd * m, m = A0 * (-p^{-1}) mod 2^32
+__device__ __forceinline__ uint32_t mont_m(uint32_t a0) { return a0 * BZK_NP0; }
 
 __device__ __forceinline__ void red_a(uint32_t A[9], uint32_t m) {
-#if !BZK_P0_TRICK
     asm("mad.lo.cc.u32  %0, %9, %10, %0;\n\t"
         "madc.hi.cc.u32 %1, %9, %10, %1;\n\t"
         "madc.lo.cc.u32 %2, %9, %11, %2;\n\t"
@@ -315,23 +297,6 @@ __device__ __forceinline__ void red_a(uint32_t A[9], uint32_t m) {
         : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
           "+r"(A[8])
         : "r"(m), "n"(BZK_P0), "n"(BZK_P2), "n"(BZK_P4), "n"(BZK_P6));
-    return;
-#endif
-    const uint32_t h = m - (m >> 4);
-    uint32_t dummy;   // A0 + m == 0 mod 2^32; only its carry is used
-    asm("add.cc.u32     %9, %0, %10;\n\t"
-        "addc.cc.u32    %1, %1, %11;\n\t"
-        "madc.lo.cc.u32 %2, %10, %12, %2;\n\t"
-        "madc.hi.cc.u32 %3, %10, %12, %3;\n\t"
-        "madc.lo.cc.u32 %4, %10, %13, %4;\n\t"
-        "madc.hi.cc.u32 %5, %10, %13, %5;\n\t"
-        "madc.lo.cc.u32 %6, %10, %14, %6;\n\t"
-        "madc.hi.cc.u32 %7, %10, %14, %7;\n\t"
-        "addc.u32       %8, %8, 0;"
-        : "+r"(A[0]), "+r"(A[1]), "+r"(A[2]), "+r"(A[3]), "+r"(A[4]), "+r"(A[5]), "+r"(A[6]), "+r"(A[7]),
-          "+r"(A[8]), "=r"(dummy)
-        : "r"(m), "r"(h), "n"(BZK_P2), "n"(BZK_P4), "n"(BZK_P6));
-    (void)dummy;
 }
 
 __device__ __forceinline__ void red_b(uint32_t B[9], uint32_t m) {
@@ -872,9 +837,6 @@ __device__ __forceinline__ fe ld_fe(const fe *p) {
 // 256-bit global accesses (sm_100: LDG/STG.E.ENL2.256): one instruction per element, and every
 // store writes whole 32-byte sectors (with two 128-bit stores per element the fused rounds read
 // ~60 % of their written bytes back from DRAM: partial-sector write fills, ncu r01g)
-#ifndef BZK_V8
-#define BZK_V8 1
-#endif
 #define BZK_LD8(MOD, r, ptr)                                                                      \
     asm("ld.global" MOD ".v8.u32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"                          \
         : "=r"((r).l[0]), "=r"((r).l[1]), "=r"((r).l[2]), "=r"((r).l[3]), "=r"((r).l[4]), "=r"((r).l[5]), \
@@ -884,14 +846,7 @@ __device__ __forceinline__ fe ld_fe(const fe *p) {
 // streaming load for data read exactly once (evict-first)
 __device__ __forceinline__ fe ld_fe_stream(const fe *p) {
     fe r;
-#if BZK_V8
     BZK_LD8(".cs", r, p);
-#else
-    const uint4 *q = reinterpret_cast<const uint4 *>(p);
-    uint4 x = __ldcs(q), y = __ldcs(q + 1);
-    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
-    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
-#endif
     return r;
 }
 
@@ -906,15 +861,9 @@ __device__ __forceinline__ fe ld_fe_cg(const fe *p) {
 }
 
 __device__ __forceinline__ void st_fe(fe *p, const fe &v) {
-#if BZK_V8
     asm volatile("st.global.v8.u32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(p), "r"(v.l[0]), "r"(v.l[1]),
                  "r"(v.l[2]), "r"(v.l[3]), "r"(v.l[4]), "r"(v.l[5]), "r"(v.l[6]), "r"(v.l[7])
                  : "memory");
-#else
-    uint4 *q = reinterpret_cast<uint4 *>(p);
-    q[0] = make_uint4(v.l[0], v.l[1], v.l[2], v.l[3]);
-    q[1] = make_uint4(v.l[4], v.l[5], v.l[6], v.l[7]);
-#endif
 }
 
 __device__ __forceinline__ void st_fe_cg(fe *p, const fe &v) {

@@ -107,13 +107,10 @@ __device__ __forceinline__ void eval_pair(const uint64_t (&a)[D], const uint64_t
     }
 }
 
-// Lazy evaluation sums (GL_LAZY, default on): the last product of every point is accumulated
+// Lazy evaluation sums: the last product of every point is accumulated
 // unreduced into a 192-bit accumulator (lo, hi, top) and reduced once per thread, instead of a
 // 128 -> 64-bit reduction plus a canonical addition per product (the round kernels were ALU-bound
 // on those, ncu r01).  2^128 = -2^32 (mod p), so top * C128 folds the third word back.
-#ifndef GL_LAZY
-#define GL_LAZY 1
-#endif
 constexpr uint64_t C128 = 0xfffffffe00000001ull;   // 2^128 mod p
 
 struct Wide { uint64_t lo, hi, top; };
@@ -246,9 +243,6 @@ __device__ __forceinline__ void load_pair(const uint64_t *src, uint64_t *dst, ui
 #ifndef GL_OCC
 #define GL_OCC 3
 #endif
-#ifndef GL_SPLIT
-#define GL_SPLIT 1   // fused rounds (both orders): issue every raw load of an iteration before the folds
-#endif
 #ifndef GL_MLP_FUSED
 #define GL_MLP_FUSED 2   // pairs per iteration of the split fused loop (g2: 2 -> fused 0.86 of HBM, 4 -> 0.83)
 #endif
@@ -259,17 +253,10 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
     const uint64_t h = 1ull << P.log_h;
-#if GL_LAZY
     Wide wacc[D + 1];
 #pragma unroll
     for (int t = 0; t <= D; ++t) wacc[t] = Wide{0, 0, 0};
 #define GL_ACC wacc
-#else
-    uint64_t acc[D + 1];
-#pragma unroll
-    for (int t = 0; t <= D; ++t) acc[t] = 0;
-#define GL_ACC acc
-#endif
     const uint64_t *src = P.src + (size_t)b * D * (FIRST ? 2 * h : 4 * h);
     uint64_t *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const uint64_t r = FIRST ? 0 : P.ps[b].r;
@@ -278,8 +265,7 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
     // MLP pairs in flight per iteration (memory-level parallelism: the kernel streams); fewer for
     // d >= 3, whose wider accumulators would otherwise spill
     constexpr int MLP = D <= 2 ? GL_MLP : (GL_MLP > 2 ? 2 : GL_MLP);
-#if GL_SPLIT
-    // all raw loads of the MLP pairs first (LSB fused rounds), then folds + stores, then evaluation:
+    // fused rounds (both orders): all raw loads of the MLP pairs first (LSB fused rounds), then folds + stores, then evaluation:
     // every load is in flight before the first dependent instruction
     constexpr int MF = D <= 2 ? GL_MLP_FUSED : 2;
     if (!FIRST && ORDER == 0) {
@@ -336,7 +322,6 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
             for (int q = 0; q < MF; ++q) eval_pair<D>(a[q], bb[q], GL_ACC);
         }
     }
-#endif
     for (; j + (MLP - 1) * stride < h; j += MLP * stride) {
         uint64_t a[MLP][D], bb[MLP][D];
 #pragma unroll
@@ -350,11 +335,9 @@ __global__ void __launch_bounds__(256, GL_OCC) k_gl_round(RoundParams P) {
         eval_pair<D>(a0, b0, GL_ACC);
     }
 #undef GL_ACC
-#if GL_LAZY
     uint64_t acc[D + 1];
 #pragma unroll
     for (int t = 0; t <= D; ++t) acc[t] = wide_reduce(wacc[t]);
-#endif
     block_reduce<D + 1>(acc, s_red);
     uint64_t *evals = P.round_evals + (size_t)b * P.k * (D + 1);
     uint64_t *chals = P.challenges + (size_t)b * P.k;

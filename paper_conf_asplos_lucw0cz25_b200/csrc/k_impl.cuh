@@ -28,17 +28,12 @@ static cudaError_t launch_round_cl(dim3 grid, uint32_t threads, size_t sm, cudaS
 template <>
 cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
                                 const RoundParams &p) {
-    const size_t sm = first ? round_smem_bytes<BZK_D, true>(threads) : round_smem_bytes<BZK_D, false>(threads);
+    const size_t sm = 0;
     const uint32_t cl = p.cluster;
     if (order == 0) return first ? launch_round_cl<0, true>(grid, threads, sm, s, p, cl)
                                  : launch_round_cl<0, false>(grid, threads, sm, s, p, cl);
     return first ? launch_round_cl<1, true>(grid, threads, sm, s, p, cl)
                  : launch_round_cl<1, false>(grid, threads, sm, s, p, cl);
-}
-
-template <>
-size_t round_smem<BZK_D>(bool first, uint32_t threads) {
-    return first ? round_smem_bytes<BZK_D, true>(threads) : round_smem_bytes<BZK_D, false>(threads);
 }
 
 template <>

@@ -64,27 +64,15 @@ __device__ __forceinline__ void set_iv(uint32_t h[8]) {
     h[4] = 0x510e527fu; h[5] = 0x9b05688cu; h[6] = 0x1f83d9abu; h[7] = 0x5be0cd19u;
 }
 
-// BZK_MK_FMA_ADD=1 (default): every addition is issued as IMAD (x * 1 + y, the 1 opaque to the
-// compiler) on the FMA pipe, leaving the ALU pipe to the rotations and the logic (SHF, LOP3), which
-// only it can execute: 6,366 -> 7,798 trees/s at 256 x 2^20 blocks.
-#ifndef BZK_MK_FMA_ADD
-#define BZK_MK_FMA_ADD 1
-#endif
-// BZK_MK_KSPLIT=1: K[t] + W[t] is also issued as IMAD (else a plain add the compiler places)
-#ifndef BZK_MK_KSPLIT
-#define BZK_MK_KSPLIT 0
-#endif
+// Every addition is issued as IMAD (x * 1 + y, the 1 opaque to the compiler) on the FMA pipe,
+// leaving the ALU pipe to the rotations and the logic (SHF, LOP3), which only it can execute:
+// 6,366 -> 7,798 trees/s at 256 x 2^20 blocks.  K[t] + W[t] stays a plain add.
 static __constant__ uint32_t c_one = 1;
 
 __device__ __forceinline__ uint32_t fadd(uint32_t a, uint32_t b, uint32_t one) {
-#if BZK_MK_FMA_ADD
     uint32_t r;
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(one), "r"(b));
     return r;
-#else
-    (void)one;
-    return a + b;
-#endif
 }
 
 // One round with the working variables named by position (no register moves after unrolling).
@@ -106,47 +94,16 @@ __device__ __forceinline__ uint32_t fadd(uint32_t a, uint32_t b, uint32_t one) {
     BZK_MK_RND(c, d, e, f, g, h, a, b, KW(T + 6));    \
     BZK_MK_RND(b, c, d, e, f, g, h, a, KW(T + 7))
 
-// BZK_MK_ROLLED=1: the 64 rounds run as 4 iterations of a 16-round body (the rolling message-schedule
-// window keeps static register indices; K is read with an indexed constant load): ~8 KB of hot code
-// instead of ~22 KB, but 92 IMAD.MOV per 16 rounds to re-place the working variables.  With ONE
-// hash body in the stage loop the fully unrolled body (default 0) no longer stalls on instruction
-// fetch and is 4 % faster (the first version inlined 8 unrolled bodies and did, ncu r01f).
-#ifndef BZK_MK_ROLLED
-#define BZK_MK_ROLLED 0
-#endif
+// The 64 rounds are fully unrolled (no moves to re-place the working variables).  With ONE hash body
+// in the stage loop this no longer stalls on instruction fetch and beat a rolled 16-round body by 4 %
+// (the first version inlined 8 unrolled bodies and did stall, ncu r01f).
 
 // FIPS 180-4 Sec. 6.2.2: state st <- st + rounds(st, W); w[16] is the big-endian message (clobbered:
 // it holds the rolling 16-word message schedule)
 __device__ __forceinline__ void compress(uint32_t st[8], uint32_t w[16]) {
     const uint32_t one = c_one;
     uint32_t a = st[0], b = st[1], c = st[2], d = st[3], e = st[4], f = st[5], g = st[6], h = st[7];
-#if BZK_MK_ROLLED
-#pragma unroll 1
-    for (int T = 0; T < 64; T += 16) {
-#if BZK_MK_KSPLIT
-#define BZK_MK_KW_MSG(t) fadd(c_K.v[T + (t)], w[(t)], one)
-#else
-#define BZK_MK_KW_MSG(t) (c_K.v[T + (t)] + w[(t)])
-#endif
-        BZK_MK_8ROUNDS(0, BZK_MK_KW_MSG);
-        BZK_MK_8ROUNDS(8, BZK_MK_KW_MSG);
-#undef BZK_MK_KW_MSG
-        if (T < 48) {
-            // next 16 schedule words in place: W[t] = s1(W[t-2]) + W[t-7] + s0(W[t-15]) + W[t-16]
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-                const uint32_t w15 = w[(j + 1) & 15], w2 = w[(j + 14) & 15];
-                w[j] = fadd(fadd(fadd(w[j], (rotr(w15, 7) ^ rotr(w15, 18) ^ (w15 >> 3)), one), w[(j + 9) & 15], one),
-                            (rotr(w2, 17) ^ rotr(w2, 19) ^ (w2 >> 10)), one);
-            }
-        }
-    }
-#else
-#if BZK_MK_KSPLIT
-#define BZK_MK_KW_MSG(t) fadd(c_K.v[(t)], w[(t) & 15], one)
-#else
 #define BZK_MK_KW_MSG(t) (c_K.v[(t)] + w[(t) & 15])
-#endif
 #pragma unroll
     for (int T = 0; T < 64; T += 8) {
         if (T >= 16) {
@@ -162,7 +119,6 @@ __device__ __forceinline__ void compress(uint32_t st[8], uint32_t w[16]) {
         BZK_MK_8ROUNDS(T, BZK_MK_KW_MSG);
     }
 #undef BZK_MK_KW_MSG
-#endif
     st[0] += a; st[1] += b; st[2] += c; st[3] += d; st[4] += e; st[5] += f; st[6] += g; st[7] += h;
 }
 
@@ -170,20 +126,10 @@ __device__ __forceinline__ void compress(uint32_t st[8], uint32_t w[16]) {
 __device__ __forceinline__ void compress_pad64(uint32_t st[8]) {
     const uint32_t one = c_one;
     uint32_t a = st[0], b = st[1], c = st[2], d = st[3], e = st[4], f = st[5], g = st[6], h = st[7];
-#if BZK_MK_ROLLED
-#pragma unroll 1
-    for (int T = 0; T < 64; T += 16) {
-#define BZK_MK_KW_PAD(t) (c_pad_kw.v[T + (t)])
-        BZK_MK_8ROUNDS(0, BZK_MK_KW_PAD);
-        BZK_MK_8ROUNDS(8, BZK_MK_KW_PAD);
-#undef BZK_MK_KW_PAD
-    }
-#else
 #define BZK_MK_KW_PAD(t) (c_pad_kw.v[(t)])
 #pragma unroll
     for (int T = 0; T < 64; T += 8) { BZK_MK_8ROUNDS(T, BZK_MK_KW_PAD); }
 #undef BZK_MK_KW_PAD
-#endif
     st[0] += a; st[1] += b; st[2] += c; st[3] += d; st[4] += e; st[5] += f; st[6] += g; st[7] += h;
 }
 

@@ -15,8 +15,8 @@
 //               folded ones to the other ping-pong buffer (Fig. 5) and evaluates round i
 //               on them in registers (the sums reuse the update's loads).  g_i(1) is not
 //               summed: it is derived exactly as claim_i - g_i(0), claim_i = g_{i-1}(r_{i-1}).
-//       Each thread takes two pairs at a time and sums their products with ONE Montgomery
-//       reduction (mont_mul2).  Partial sums: per thread -> warp shuffle -> shared memory ->
+//       The last product of every summed point goes unreduced into a 544-bit per-thread
+//       accumulator (mul_acc) and is reduced once after the loop.  Partial sums: per thread -> warp shuffle -> shared memory ->
 //       per-CTA partial in global -> last-CTA ticket; the last CTA of each proof reduces the
 //       partials, hashes the transcript and publishes r_i (single pass, no extra launch; the
 //       paper's reduction made repeated global passes).
@@ -115,57 +115,15 @@ __device__ __forceinline__ constexpr int point_t(int idx) {   // -1 = infinity
     return DERIVE ? (idx == 0 ? 0 : idx + 1) : idx;
 }
 
-// Evaluate two pairs at the summed points and accumulate (lazy arithmetic, values < 2p).
-// Inputs per table m: a[m] (= v(0)) and s[m], which is b = v(1) in round 1 and delta = b - a in
-// the fused rounds (whichever the point set needs, to keep registers down).  Products of the two
-// pairs share ONE Montgomery reduction (mont_mul2_lz); sums go to 288-bit accumulators; every sum
-// carries R^{-(D-1)}.
+// d = 1: g(t) is a sum of table values only (no products), so a pair's points t = 0 (a) and, in
+// round 1, t = 1 (b) are summed straight into 288-bit accumulators; the fused rounds derive g(1).
+// Two pairs are added together first (lazy values < 2p each).
 template <int D, bool DERIVE>
 __device__ __forceinline__ void eval_two(const fe (&a)[D], const fe (&s)[D], const fe (&a2)[D], const fe (&s2)[D],
                                          acc9 (&acc)[Pts<D, DERIVE>::NV]) {
-    constexpr int NV = Pts<D, DERIVE>::NV;
-    fe v[D], v2[D], dl[D], dl2[D];
-#pragma unroll
-    for (int idx = 0; idx < NV; ++idx) {
-        const int t = point_t<D, DERIVE>(idx);
-        if ((t < 0 || t == 2) && !DERIVE) {   // round 1: delta = b - a on demand
-#pragma unroll
-            for (int m = 0; m < D; ++m) {
-                dl[m] = lz_sub(s[m], a[m]);
-                dl2[m] = lz_sub(s2[m], a2[m]);
-                if (!(D == 2 && m == 0)) { dl[m] = lz_red(dl[m]); dl2[m] = lz_red(dl2[m]); }   // see load_pair
-            }
-        }
-        const fe *x, *x2;
-        if (t == 0) { x = a; x2 = a2; }
-        else if (t == 1) { x = s; x2 = s2; }                       // FIRST only: s = b
-        else if (t < 0) { x = DERIVE ? s : dl; x2 = DERIVE ? s2 : dl2; }
-        else {
-#pragma unroll
-            for (int m = 0; m < D; ++m) {
-                const fe &d1 = DERIVE ? s[m] : dl[m];
-                const fe &d2 = DERIVE ? s2[m] : dl2[m];
-                if (t == 2) {
-                    // DERIVE: a + 2 delta;  FIRST: b + delta
-                    v[m] = lz_red(lz_add(DERIVE ? a[m] : s[m], d1));
-                    v2[m] = lz_red(lz_add(DERIVE ? a2[m] : s2[m], d2));
-                    if (DERIVE) { v[m] = lz_red(lz_add(v[m], d1)); v2[m] = lz_red(lz_add(v2[m], d2)); }
-                } else {
-                    v[m] = lz_red(lz_add(v[m], d1));
-                    v2[m] = lz_red(lz_add(v2[m], d2));
-                }
-            }
-            x = v; x2 = v2;
-        }
-        if (D == 1) {
-            acc9_add(acc[idx], lz_add(x[0], x2[0]));
-        } else {
-            fe p = x[0], p2 = x2[0];
-#pragma unroll
-            for (int m = 1; m < D - 1; ++m) { p = mont_mul_lz(p, x[m]); p2 = mont_mul_lz(p2, x2[m]); }
-            acc9_add(acc[idx], mont_mul2_lz(p, x[D - 1], p2, x2[D - 1]));
-        }
-    }
+    static_assert(D == 1, "d >= 2 sums go through eval_one / mul_acc");
+    acc9_add(acc[0], lz_add(a[0], a2[0]));
+    if (!DERIVE) acc9_add(acc[1], lz_add(s[0], s2[0]));   // round 1: s = b
 }
 
 // 288-bit accumulator -> canonical field element: hi * 2^256 + lo = hi * (R mod p) + lo (mod p)
@@ -208,12 +166,8 @@ __device__ __forceinline__ fe acc17_to_fe(const acc17 &a) {
     return fe_add(fe_reduce_256(lo), mont_mul(hi, fe_const(2)));
 }
 
-// BZK_UNRED (d >= 2): the last product of every summed point goes into a 544-bit accumulator
-// (mul_acc) and is reduced once per thread, instead of two pairs sharing one reduction (eval_two).
-#ifndef BZK_UNRED
-#define BZK_UNRED 1
-#endif
-template <int D> struct UseUnred { static constexpr bool v = BZK_UNRED && D >= 2; };
+// d >= 2: the last product of every summed point goes into a 544-bit accumulator (mul_acc) and is
+// reduced once per thread (d = 1 has no products: its sums go through eval_two's 288-bit adds).
 
 // one pair at the summed points (same point sets and lazy bounds as eval_two)
 template <int D, bool DERIVE>
@@ -280,24 +234,14 @@ __device__ __forceinline__ fe fold1(const fe &a, const fe &b, const fe &rmont) {
     return fe_add(a, mont_mul(rmont, fe_sub(b, a)));
 }
 
-// lazy fold for the hot loop: a, b < 2p, rmont < p  ->  a + r (b - a) (mod p), result < 2p
-__device__ __forceinline__ fe fold_lz(const fe &a, const fe &b, const fe &rmont) {
-    return lz_red(lz_add(a, mont_mul_lz(rmont, lz_sub(b, a))));
-}
-
-// the same fold through the fixed-multiplier table K of r (field.cuh fixmul_lz; K in shared memory)
+// lazy fold for the hot loop: a, b < 2p -> a + r (b - a) (mod p), result < 2p, through the
+// fixed-multiplier table K of r (field.cuh fixmul_lz; K in shared memory)
 __device__ __forceinline__ fe fold_fx(const fe &a, const fe &b, const fe *K, uint32_t zmask) {
     return lz_red(lz_add(a, fixmul_lz(lz_sub(b, a), K, zmask)));
 }
 
-#ifndef BZK_FIXMUL
-#define BZK_FIXMUL 1   // 1: fused-round folds use the per-(proof, round) table K_i = r 2^(32i+64)
-#endif
-#if BZK_FIXMUL
+// fused-round folds use the per-(proof, round) table K_i = r 2^(32i+64) (fixmul_lz)
 #define BZK_FOLD(a, b) fold_fx(a, b, sK, zmask)
-#else
-#define BZK_FOLD(a, b) fold_lz(a, b, rm)
-#endif
 
 // ---------------------------------------------------------------- per-round finalisation
 
@@ -481,7 +425,7 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
         }
         a[m] = lo;
         // round 1: b; fused rounds: delta (for d = 2 the table-0 delta may stay < 4p: it only
-        // meets mont_mul2_lz(<4p, <2p, <4p, <2p) < 4.02p)
+        // meets mul_acc, a full 512-bit product < 8p^2)
         sv[m] = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
     }
 }
@@ -521,97 +465,6 @@ __device__ __forceinline__ void prefetch_pairs(const fe *src, uint64_t h, uint64
     }
 }
 
-// ---------------------------------------------------------------- cp.async staging of fold groups
-//
-// A "group" is what one fold step of one thread consumes: the E entries (E = 2 in round 1, 4 in a
-// fused round) of ONE table for ONE pair.  Groups stream through a per-thread ring of kStageSlots
-// shared-memory slots filled by cp.async (LDGSTS, no registers held while in flight) kStageDist
-// groups ahead of use, so the IMAD chains of the current group overlap the DRAM latency of the
-// next ones.  Slot layout is transposed (chunk-major across the CTA's threads): the 16-byte chunk c
-// of thread t sits at ((slot * 2E + c) * blockDim + t) * 16, so both the cp.async writes and the
-// LDS.128 reads of a warp are bank-conflict free.
-#ifndef BZK_STAGE
-#define BZK_STAGE 0   // measured slower on B200; kept as an option
-#endif
-constexpr int kStageDist = 2;
-constexpr int kStageSlots = kStageDist + 1;
-
-template <bool FIRST> struct GroupE { static constexpr int E = FIRST ? 2 : 4; };
-
-template <int D, int ORDER, bool FIRST>
-__device__ __forceinline__ const fe *group_entry(const fe *src, uint64_t h, uint64_t jj, int m, int e) {
-    if (FIRST) {
-        const fe *T = src + (size_t)m * (2 * h);
-        return ORDER == 0 ? T + 2 * jj + e : T + jj + (e ? h : 0);
-    }
-    const fe *T = src + (size_t)m * (4 * h);
-    if (ORDER == 0) return T + 4 * jj + e;
-    // MSB fused: the fold pairs are (x, x + 2h); this round pairs (jj, jj + h)
-    const uint64_t off[4] = {0, 2 * h, h, 3 * h};
-    return T + jj + off[e];
-}
-
-__device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc) {
-    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-
-template <int D, int ORDER, bool FIRST>
-__device__ __forceinline__ void issue_group(uint4 *ring, uint32_t slot, const fe *src, uint64_t h, uint64_t jj,
-                                            int m) {
-    constexpr int E = GroupE<FIRST>::E;
-    if (jj < h) {
-#pragma unroll
-        for (int e = 0; e < E; ++e) {
-            const uint4 *g = reinterpret_cast<const uint4 *>(group_entry<D, ORDER, FIRST>(src, h, jj, m, e));
-#pragma unroll
-            for (int c = 0; c < 2; ++c)
-                cp_async16(&ring[((size_t)(slot * 2 * E + 2 * e + c)) * blockDim.x + threadIdx.x], g + c);
-        }
-    }
-    cp_async_commit();   // always commit (possibly empty) so group counting stays uniform
-}
-
-__device__ __forceinline__ fe lds_entry(const uint4 *ring, uint32_t chunk0) {
-    const uint4 x = ring[(size_t)chunk0 * blockDim.x + threadIdx.x];
-    const uint4 y = ring[(size_t)(chunk0 + 1) * blockDim.x + threadIdx.x];
-    fe r;
-    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
-    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
-    return r;
-}
-
-// consume group (q, m) of the current iteration from its ring slot: fold (fused rounds) or pass
-// through (round 1); write the folded entries to dst; return (a, b - a)
-template <int D, int ORDER, bool FIRST>
-__device__ __forceinline__ void consume_group(const uint4 *ring, uint32_t slot, fe *dst, uint64_t h, uint64_t jj,
-                                              int m, const fe &rm, fe &a, fe &sv) {
-    constexpr int E = GroupE<FIRST>::E;
-    const uint32_t c0 = slot * 2 * E;
-    fe lo, hi;
-    if (FIRST) {
-        lo = lds_entry(ring, c0);
-        hi = lds_entry(ring, c0 + 2);
-    } else {
-        lo = fold_lz(lds_entry(ring, c0), lds_entry(ring, c0 + 2), rm);
-        hi = fold_lz(lds_entry(ring, c0 + 4), lds_entry(ring, c0 + 6), rm);
-        fe *U = dst + (size_t)m * (2 * h);
-        if (ORDER == 0) { st_fe(U + 2 * jj, lo); st_fe(U + 2 * jj + 1, hi); }
-        else            { st_fe(U + jj, lo);     st_fe(U + jj + h, hi); }
-    }
-    a = lo;
-    sv = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));   // see load_pair
-}
-
-// dynamic shared memory of k_round (bytes) for a CTA of `threads`
-template <int D, bool FIRST>
-constexpr size_t round_smem_bytes(uint32_t threads) {
-    return BZK_STAGE ? (size_t)kStageSlots * 2 * GroupE<FIRST>::E * 16 * threads : 0;
-}
-
 template <int D, int ORDER, bool FIRST>
 __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
     constexpr bool DERIVE = !FIRST;
@@ -629,53 +482,16 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     fe *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
     const fe rm = FIRST ? fe_zero() : P.ps[b].rmont;
     __shared__ __align__(16) fe sK[8];   // fixed-multiplier table of r_{i-1} (fused rounds)
-    if (!FIRST && BZK_FIXMUL) {
+    if (!FIRST) {
         if (threadIdx.x < 8) sK[threadIdx.x] = mont_mul(rm, P.consts[kConstPow2 + threadIdx.x]);   // r 2^(32t+64)
         __syncthreads();
     }
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     const uint32_t lane = threadIdx.x & 31;
-#ifdef BZK_STAGGER_NS
-    // experiment: de-phase the warps of a CTA so their IMAD-heavy and ALU-heavy stretches interleave
-    if (BZK_STAGGER_NS > 0) __nanosleep((threadIdx.x >> 5) % 4 * BZK_STAGGER_NS);
-#endif
-#if BZK_STAGE
-    extern __shared__ __align__(16) uint4 ring[];
-    {
-        const uint64_t j0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-        // group g -> iteration g / (2D), pair slot q = (g % 2D) / D, table m = g % D
-        auto g_jj = [&](uint64_t g) { return j0 + (g / (2 * D)) * 2 * stride + ((g % (2 * D)) / D) * stride; };
-#pragma unroll
-        for (int g = 0; g < kStageDist; ++g)
-            issue_group<D, ORDER, FIRST>(ring, g % kStageSlots, src, h, g_jj(g), g % D);
-        uint64_t g = 0;
-        for (uint64_t j = j0; j < h; j += 2 * stride) {
-            fe a[2][D], sv[2][D];
-#pragma unroll
-            for (int q = 0; q < 2; ++q)
-#pragma unroll
-                for (int m = 0; m < D; ++m, ++g) {
-                    const uint64_t gn = g + kStageDist;
-                    issue_group<D, ORDER, FIRST>(ring, (uint32_t)(gn % kStageSlots), src, h, g_jj(gn), (int)(gn % D));
-                    cp_async_wait<kStageDist>();
-                    const uint64_t jj = j + q * stride;
-                    if (jj < h) {
-                        consume_group<D, ORDER, FIRST>(ring, (uint32_t)(g % kStageSlots), dst, h, jj, m, rm, a[q][m],
-                                                       sv[q][m]);
-                    } else {
-                        a[q][m] = fe_zero();
-                        sv[q][m] = fe_zero();
-                    }
-                }
-            eval_two<D, DERIVE>(a[0], sv[0], a[1], sv[1], wacc);
-        }
-        cp_async_wait<0>();
-    }
-#else
     // One pair per loop iteration (keeps the loop body -- 2d folds + one two-pair evaluation -- small
     // enough for the instruction cache); every second pair is held in registers and evaluated
     // together with the next one, so the two pairs' products share one Montgomery reduction.
-    if constexpr (UseUnred<D>::v) {
+    if constexpr (D >= 2) {
         acc17 uacc[NV];
 #pragma unroll
         for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
@@ -709,7 +525,6 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
             eval_two<D, DERIVE>(ha, hs, z, z, wacc);
         }
     }
-#endif
 
     fe acc[NV];
 #pragma unroll
@@ -880,7 +695,5 @@ cudaError_t launch_tail(uint32_t order, uint32_t grid, uint32_t threads, size_t 
                         const TailParams &p);
 template <int D>
 cudaError_t set_kernel_attrs();   // once per process, before any launch or graph capture
-template <int D>
-size_t round_smem(bool first, uint32_t threads);
 
 }  // namespace bzk

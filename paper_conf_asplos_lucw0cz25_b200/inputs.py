@@ -1,16 +1,30 @@
 """Seeded synthetic inputs shared by the oracle side and the CUDA side.
 
-This module holds NONE of the method's arithmetic (no field operations, no
-modulus): it only turns a counter into 64-bit words.  The CUDA side implements
-the same counter-based generator in ``csrc/gen.cu`` (``bzk_generate``); the two
-are checked word-for-word by ``tests/test_gpu_generator.py``.
+This module holds NONE of the method's arithmetic (no field operations): it
+only turns a counter into 64-bit words.  The one place a modulus appears is the
+range of the generated values -- they must be canonical field elements, so a
+value drawn from [0, 2^254) that lands in [p, 2^254) is moved down by p once
+(a comparison and a subtraction on raw words, SURVEY.md 8(d) "mask to 254 bits;
+if >= p, subtract p once").  The CUDA side implements the same counter-based
+generator in ``csrc/gen.cuh`` (``bzk_generate``); the two are checked
+word-for-word by ``tests/test_gpu_parity.py::test_generator_matches_host_twin``.
 
 Recipe:
     ctr(I, m, x, w) = (I << 36) | (m << 32) | (x << 2) | w          I < 2^28, m < 16, x < 2^30, w < 4
     word            = splitmix64_mix(data_seed + (ctr + 1) * 0x9E3779B97F4A7C15)
-    uniform  : limbs w = 0..3 are the words, limb 3 masked to 61 bits -> value < 2^253 < p
+    uniform  : limbs w = 0..3 are the words, limb 3 masked to 62 bits (value < 2^254), then one
+               conditional subtraction of p -> uniform-ish over the WHOLE field [0, p)
     smallint : limb 0 = word(w=0) & 0xff, limbs 1..3 = 0 (non-negative 8-bit activations, VML)
     vml      : table m = 0 smallint, tables m >= 1 uniform
+    adversarial : the operands where lazy reduction bounds are tightest.  Each table (I, m) draws a
+               mode from  word'(I, m) mod 5  (word' = splitmix64 with data_seed ^ ADV_TABLE_SALT at
+               ctr = I << 36 | m << 32):
+                 0 near-top   p - 1 - (word(w=0) & 0xffff)      in [p - 2^16, p)
+                 1 all p - 1
+                 2 alternating 0 (x even) / p - 1 (x odd)
+                 3 high band  [2^253, 2^253 + 2^252)  (limb 3 = (word(w=3) & (2^60 - 1)) | 2^61)
+                 4 per-element mix: word''(I, m, x) mod 5 (salt ADV_ELEM_SALT) picks near-top,
+                   p - 1, 0, high band or uniform for each element
 I is the GLOBAL proof index, so a proof's tables do not depend on the batch it
 is generated in, the wave it runs in or the GPU it is sharded to.
 """
@@ -29,9 +43,20 @@ MASK61 = np.uint64((1 << 61) - 1)
 DIST_UNIFORM = 0
 DIST_SMALLINT = 1
 DIST_VML = 2
-DIST_GL = 3          # Goldilocks (NEXT-2): ONE word per element, masked to 63 bits -> < 2^63 < p_gl
-DISTS = {"uniform": DIST_UNIFORM, "smallint": DIST_SMALLINT, "vml": DIST_VML, "gl": DIST_GL}
-MASK63 = np.uint64((1 << 63) - 1)
+DIST_GL = 3          # Goldilocks (NEXT-2): ONE word per element, one conditional subtraction of p_gl
+DIST_ADV = 4         # BN254 adversarial (top of the field, p - 1, 0 / p - 1, [2^253, ...)), see above
+DIST_GL_ADV = 5      # Goldilocks adversarial: the same five modes over p_gl, high band [2^63, p_gl)
+DISTS = {"uniform": DIST_UNIFORM, "smallint": DIST_SMALLINT, "vml": DIST_VML, "gl": DIST_GL,
+         "adversarial": DIST_ADV, "gl_adversarial": DIST_GL_ADV}
+MASK62 = np.uint64((1 << 62) - 1)
+MASK60 = np.uint64((1 << 60) - 1)
+BIT61 = np.uint64(1 << 61)
+
+# range bounds of the generated values (the field moduli, as raw 64-bit words; no arithmetic mod p)
+P_BN254 = [0x43E1F593F0000001, 0x2833E84879B97091, 0xB85045B68181585D, 0x30644E72E131A029]
+P_GL = 0xFFFFFFFF00000001
+ADV_TABLE_SALT = 0x5441424C45414456     # "TABLEADV"
+ADV_ELEM_SALT = 0x454C454D41445653      # "ELEMADVS"
 
 
 def splitmix64(ctr: np.ndarray, data_seed: int = DATA_SEED) -> np.ndarray:
@@ -42,16 +67,101 @@ def splitmix64(ctr: np.ndarray, data_seed: int = DATA_SEED) -> np.ndarray:
         return z ^ (z >> np.uint64(31))
 
 
-def gen_tables_gl(batch: int, d: int, k: int, first_index: int = 0, data_seed: int = DATA_SEED) -> np.ndarray:
-    """Goldilocks tables, uint64 [B][d][2^k]: word(I, m, x, w=0) & (2^63 - 1)."""
+def _geq_p(words: np.ndarray) -> np.ndarray:
+    """words [..., 4] (LE u64) >= p_bn254, lexicographically from the top limb."""
+    ge = np.ones(words.shape[:-1], dtype=bool)          # equal so far -> >= holds on full equality
+    for i in range(4):                                  # from the lowest limb up: top limbs decide last
+        pi = np.uint64(P_BN254[i])
+        ge = (words[..., i] > pi) | ((words[..., i] == pi) & ge)
+    return ge
+
+
+def _sub_p(words: np.ndarray) -> np.ndarray:
+    """words - p_bn254 (words >= p), 4-limb subtraction with borrow."""
+    out = np.empty_like(words)
+    borrow = np.zeros(words.shape[:-1], dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        for i in range(4):
+            pi = np.uint64(P_BN254[i])
+            out[..., i] = words[..., i] - pi - borrow
+            borrow = ((words[..., i] < pi) | ((words[..., i] == pi) & (borrow == 1))).astype(np.uint64)
+    return out
+
+
+def _canonical_254(words: np.ndarray) -> np.ndarray:
+    """mask limb 3 to 62 bits (value < 2^254 < 2p), then subtract p once where value >= p"""
+    words = words.copy()
+    words[..., 3] &= MASK62
+    ge = _geq_p(words)
+    if ge.any():
+        words[ge] = _sub_p(words[ge])
+    return words
+
+
+def _pm1(shape) -> np.ndarray:
+    out = np.empty(tuple(shape) + (4,), dtype=np.uint64)
+    out[...] = np.array(P_BN254, dtype=np.uint64)
+    out[..., 0] -= np.uint64(1)
+    return out
+
+
+def _adv_modes(I: int, m: int, x: np.ndarray, data_seed: int):
+    """(table mode, per-element mode array): table mode 0..3 applies to every element; table mode 4
+    gives each element its own mode 0..4 (0 near-top, 1 p - 1, 2 ZERO, 3 high band, 4 uniform)."""
+    base = (np.uint64(I) << np.uint64(36)) | (np.uint64(m) << np.uint64(32))
+    tmode = int(splitmix64(np.array([base], dtype=np.uint64), data_seed ^ ADV_TABLE_SALT)[0] % np.uint64(5))
+    if tmode < 4:
+        return tmode, np.full(x.shape, tmode, dtype=np.int64)
+    return tmode, (splitmix64(base | (x << np.uint64(2)), data_seed ^ ADV_ELEM_SALT) % np.uint64(5)).astype(np.int64)
+
+
+def _adversarial(I: int, m: int, x: np.ndarray, words: np.ndarray, data_seed: int) -> np.ndarray:
+    """BN254 adversarial table (DIST_ADV), modes as in the module docstring."""
+    tmode, mode = _adv_modes(I, m, x, data_seed)
+    out = _canonical_254(words)                                  # element mode 4: uniform
+    near = _pm1(x.shape)
+    near[..., 0] -= words[..., 0] & np.uint64(0xFFFF)            # p - 1 - s, s < 2^16 (limb 0 of p - 1 >= 2^16)
+    out[mode == 0] = near[mode == 0]
+    out[mode == 1] = _pm1(x.shape)[mode == 1]
+    two = _pm1(x.shape)
+    two[(x & np.uint64(1)) == 0] = 0                             # table mode 2: 0 / p - 1 alternating
+    if tmode == 4:
+        two[:] = 0                                               # element mode 2: zero
+    out[mode == 2] = two[mode == 2]
+    high = words.copy()
+    high[..., 3] = (high[..., 3] & MASK60) | BIT61               # [2^253, 2^253 + 2^252)
+    out[mode == 3] = high[mode == 3]
+    return out
+
+
+def gen_tables_gl(batch: int, d: int, k: int, first_index: int = 0, data_seed: int = DATA_SEED,
+                  dist: str | int = "gl") -> np.ndarray:
+    """Goldilocks tables, uint64 [B][d][2^k]: word(I, m, x, w=0), minus p_gl once if >= p_gl
+    ("gl"), or the adversarial modes over p_gl ("gl_adversarial": high band [2^63, 2^63 + 2^62))."""
+    dist = DISTS[dist] if isinstance(dist, str) else int(dist)
     N = 1 << k
     out = np.empty((batch, d, N), dtype=np.uint64)
     x = np.arange(N, dtype=np.uint64)
+    pgl = np.uint64(P_GL)
     for bi in range(batch):
-        I = np.uint64(first_index + bi)
+        I = first_index + bi
         for m in range(d):
-            ctr = (I << np.uint64(36)) | (np.uint64(m) << np.uint64(32)) | (x << np.uint64(2))
-            out[bi, m] = splitmix64(ctr, data_seed) & MASK63
+            ctr = (np.uint64(I) << np.uint64(36)) | (np.uint64(m) << np.uint64(32)) | (x << np.uint64(2))
+            w = splitmix64(ctr, data_seed)
+            uni = np.where(w >= pgl, w - pgl, w)
+            if dist != DIST_GL_ADV:
+                out[bi, m] = uni
+                continue
+            tmode, mode = _adv_modes(I, m, x, data_seed)
+            v = uni.copy()
+            v[mode == 0] = (pgl - np.uint64(1) - (w & np.uint64(0xFFFF)))[mode == 0]
+            v[mode == 1] = pgl - np.uint64(1)
+            two = np.where((x & np.uint64(1)) == 0, np.uint64(0), pgl - np.uint64(1))
+            if tmode == 4:
+                two[:] = 0
+            v[mode == 2] = two[mode == 2]
+            v[mode == 3] = ((w & np.uint64((1 << 62) - 1)) | np.uint64(1 << 63))[mode == 3]
+            out[bi, m] = v
     return out
 
 
@@ -59,7 +169,7 @@ def gen_tables(batch: int, d: int, k: int, first_index: int = 0, dist: str | int
                data_seed: int = DATA_SEED, indices=None) -> np.ndarray:
     """uint64 [B][d][2^k][4] tables for global proof indices first_index.. (or ``indices``)."""
     dist = DISTS[dist] if isinstance(dist, str) else int(dist)
-    assert 0 <= k <= 30 and 1 <= d <= 15
+    assert 0 <= k <= 30 and 1 <= d <= 15 and dist in (DIST_UNIFORM, DIST_SMALLINT, DIST_VML, DIST_ADV)
     idx = np.arange(first_index, first_index + batch, dtype=np.uint64) if indices is None \
         else np.asarray(indices, dtype=np.uint64)
     N = 1 << k
@@ -75,9 +185,10 @@ def gen_tables(batch: int, d: int, k: int, first_index: int = 0, dist: str | int
             if small:
                 out[bi, m, :, 0] = words[:, 0] & np.uint64(0xFF)
                 out[bi, m, :, 1:] = 0
+            elif dist == DIST_ADV:
+                out[bi, m] = _adversarial(int(I), m, x, words, data_seed)
             else:
-                words[:, 3] &= MASK61
-                out[bi, m] = words
+                out[bi, m] = _canonical_254(words)
     return out
 
 

@@ -229,13 +229,18 @@ def test_validate_flag_rejects_noncanonical(prover, orc):
 
 def test_argument_errors(prover):
     t = dev_tables(1, 2, 4)
-    for kw in [dict(k=31), dict(d=5), dict(d=0), dict(order=2)]:
+    for kw in [dict(k=31), dict(d=0), dict(order=2)]:
         k, d, order = kw.get("k", 4), kw.get("d", 2), kw.get("order", 0)
         out = bzk.Prover.alloc_outputs(1, min(k, 4), max(min(d, 4), 1))
         b = prover.batch(t, k, d, order, None, 0, 0, out)
         with pytest.raises(bzk.BzkError) as e:
             bzk.bzk_prove(prover.ctx, b)
         assert e.value.status == bzk.BZK_EINVAL
+    out = bzk.Prover.alloc_outputs(1, 4, 4)
+    b = prover.batch(t, 4, 5, 0, None, 0, 0, out)           # well defined, not built
+    with pytest.raises(bzk.BzkError) as e:
+        bzk.bzk_prove(prover.ctx, b)
+    assert e.value.status == bzk.BZK_EUNSUPPORTED
     out = bzk.Prover.alloc_outputs(1, 4, 2)
     b = prover.batch(t, 4, 2, 0, None, 0, 0, out, batch=0)
     with pytest.raises(bzk.BzkError):
@@ -261,11 +266,13 @@ def test_cuda_graph_replay_and_recapture(prover):
     t = dev_tables(B, d, k)
     ref = prover.prove(t, k, d, 0, flags=bzk.BZK_F_PRESERVE_INPUT)
     out = bzk.Prover.alloc_outputs(B, k, d)
+    torch.cuda.synchronize()
     s = torch.cuda.Stream()
     b = prover.batch(t, k, d, 0, None, 0, bzk.BZK_F_PRESERVE_INPUT | bzk.BZK_F_GRAPH, out)
     for rep in range(3):                       # capture, then replays
-        for key in out:
-            out[key].zero_()
+        with torch.cuda.stream(s):
+            for key in out:
+                out[key].zero_()
         bzk.bzk_prove(prover.ctx, b, s)
         s.synchronize()
         for key in ref:
