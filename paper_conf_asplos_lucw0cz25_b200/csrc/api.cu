@@ -12,6 +12,7 @@
 #include <string>
 #include <vector>
 
+#include <cudaTypedefs.h>
 #include <nvtx3/nvToolsExt.h>
 
 #include "bzk.h"
@@ -158,7 +159,11 @@ struct Knobs {
     // BZK_CLUSTER=N: CTAs of a proof form thread-block clusters of up to N (2, 4, 8) that combine
     // their partial sums through DSMEM.  Off by default: measured 10 % slower on B200.
     uint32_t cluster = 1;
+    // BZK_TMA=0/1: k_round stages its operands into shared memory with TMA (sumcheck.cuh) instead of
+    // loading them straight to registers
+    uint32_t tma = 0;
     Knobs() {
+        if (const char *e = getenv("BZK_TMA")) tma = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CLUSTER")) cluster = std::max(1, std::min(8, atoi(e)));
         if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_CTA_WAVES")) waves = std::max(1, atoi(e));
@@ -353,14 +358,41 @@ bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
 // ---------------------------------------------------------------- kernel dispatch
 
 cudaError_t dispatch_round(uint32_t D, uint32_t order, bool first, dim3 grid, cudaStream_t s,
-                           const RoundParams &p) {
+                           const RoundParams &p, const CUtensorMap &tm) {
     switch (D) {
-        case 1: return launch_round<1>(order, first, grid, kRoundThreads, s, p);
-        case 2: return launch_round<2>(order, first, grid, kRoundThreads, s, p);
-        case 3: return launch_round<3>(order, first, grid, kRoundThreads, s, p);
-        case 4: return launch_round<4>(order, first, grid, kRoundThreads, s, p);
+        case 1: return launch_round<1>(order, first, grid, kRoundThreads, s, p, tm);
+        case 2: return launch_round<2>(order, first, grid, kRoundThreads, s, p, tm);
+        case 3: return launch_round<3>(order, first, grid, kRoundThreads, s, p, tm);
+        case 4: return launch_round<4>(order, first, grid, kRoundThreads, s, p, tm);
     }
     return cudaErrorInvalidValue;
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no link-time libcuda dependency)
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) != cudaSuccess ||
+            q != cudaDriverEntryPointSuccess)
+            p = nullptr;
+        return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+    }();
+    return fn;
+}
+
+// The wave's source buffer as rows of 128 B (32 x u32) with the 128-byte swizzle; boxes of box_rows
+// rows (sumcheck.cuh TmaGeo).  rows = buffer bytes / 128.
+bool make_row_map(CUtensorMap *tm, const void *base, uint64_t rows, uint32_t box_rows) {
+    PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[2] = {32, rows};
+    cuuint64_t strides[1] = {128};
+    cuuint32_t box[2] = {32, box_rows};
+    cuuint32_t estr[2] = {1, 1};
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, const_cast<void *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 cudaError_t dispatch_tail(uint32_t D, uint32_t order, uint32_t grid, size_t smem, cudaStream_t s,
@@ -482,9 +514,19 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
             rp.src = (i == 2) ? tab : ((i - 1) % 2 == 0 ? bufX : bufY);
             rp.dst = (i % 2 == 0) ? bufX : bufY;
         }
+        CUtensorMap tm;
+        memset(&tm, 0, sizeof tm);
+        rp.tma = knobs().tma;
+        if (rp.tma) {
+            rp.prefetch = 0;
+            const uint64_t E = i == 1 ? 2 : 4;   // raw entries per pair and table
+            const uint32_t box = P.order == 0 ? (uint32_t)(E * 8) : 8u;
+            if (!make_row_map(&tm, rp.src, io.nb * D * E * h / 4, box))
+                return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (TMA staging)");
+        }
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-        cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp);
+        cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
         ++ctx->launches;
         if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
     }

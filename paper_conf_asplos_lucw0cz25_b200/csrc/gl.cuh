@@ -127,7 +127,8 @@ __device__ __forceinline__ uint64_t wide_reduce(const Wide &A) {   // top < 2^32
 }
 
 // x + y reduced only to 64 bits (congruent mod p, not necessarily canonical): a multiplication
-// input needs no more
+// input needs no more.  Requires x < 2^64 and y < p (then x + y - 2^64 + 2^32 - 1 < 2^64); eval_pair
+// only adds a canonical delta to a lazy value.
 __device__ __forceinline__ uint64_t add_lazy(uint64_t x, uint64_t y) {
     const uint64_t s = x + y;
     return s < x ? s + EPS : s;       // x + y - 2^64 + (2^64 mod p) < 2^64

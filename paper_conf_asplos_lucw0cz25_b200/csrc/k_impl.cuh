@@ -3,11 +3,12 @@
 
 namespace bzk {
 
-template <int ORDER, bool FIRST>
-static cudaError_t launch_round_cl(dim3 grid, uint32_t threads, size_t sm, cudaStream_t s, const RoundParams &p,
-                                   uint32_t cluster) {
-    if (cluster <= 1) {
-        k_round<BZK_D, ORDER, FIRST><<<grid, threads, sm, s>>>(p);
+template <int ORDER, bool FIRST, bool TMA>
+static cudaError_t launch_round_v(dim3 grid, uint32_t threads, cudaStream_t s, const RoundParams &p,
+                                  const CUtensorMap &tm) {
+    const size_t sm = TMA ? tma_smem_bytes<BZK_D, FIRST>() : 0;
+    if (p.cluster <= 1) {
+        k_round<BZK_D, ORDER, FIRST, TMA><<<grid, threads, sm, s>>>(p, tm);
         return cudaGetLastError();
     }
     cudaLaunchConfig_t cfg = {};
@@ -17,32 +18,42 @@ static cudaError_t launch_round_cl(dim3 grid, uint32_t threads, size_t sm, cudaS
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = cluster;
+    attr[0].val.clusterDim.x = p.cluster;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_round<BZK_D, ORDER, FIRST>, p);
+    return cudaLaunchKernelEx(&cfg, k_round<BZK_D, ORDER, FIRST, TMA>, p, tm);
+}
+
+template <bool TMA>
+static cudaError_t launch_round_t(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
+                                  const RoundParams &p, const CUtensorMap &tm) {
+    if (order == 0) return first ? launch_round_v<0, true, TMA>(grid, threads, s, p, tm)
+                                 : launch_round_v<0, false, TMA>(grid, threads, s, p, tm);
+    return first ? launch_round_v<1, true, TMA>(grid, threads, s, p, tm)
+                 : launch_round_v<1, false, TMA>(grid, threads, s, p, tm);
 }
 
 template <>
 cudaError_t launch_round<BZK_D>(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
-                                const RoundParams &p) {
-    const size_t sm = 0;
-    const uint32_t cl = p.cluster;
-    if (order == 0) return first ? launch_round_cl<0, true>(grid, threads, sm, s, p, cl)
-                                 : launch_round_cl<0, false>(grid, threads, sm, s, p, cl);
-    return first ? launch_round_cl<1, true>(grid, threads, sm, s, p, cl)
-                 : launch_round_cl<1, false>(grid, threads, sm, s, p, cl);
+                                const RoundParams &p, const CUtensorMap &tm) {
+    return p.tma ? launch_round_t<true>(order, first, grid, threads, s, p, tm)
+                 : launch_round_t<false>(order, first, grid, threads, s, p, tm);
+}
+
+template <int ORDER, bool FIRST>
+static void set_round_attrs() {
+    cudaFuncSetAttribute(k_round<BZK_D, ORDER, FIRST, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)tma_smem_bytes<BZK_D, FIRST>());
 }
 
 template <>
 cudaError_t set_kernel_attrs<BZK_D>() {
-    const int big = 200 * 1024;
-    cudaFuncSetAttribute(k_round<BZK_D, 0, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-    cudaFuncSetAttribute(k_round<BZK_D, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-    cudaFuncSetAttribute(k_round<BZK_D, 0, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
-    cudaFuncSetAttribute(k_round<BZK_D, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, big);
+    set_round_attrs<0, true>();
+    set_round_attrs<0, false>();
+    set_round_attrs<1, true>();
+    set_round_attrs<1, false>();
     cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     return cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
 }

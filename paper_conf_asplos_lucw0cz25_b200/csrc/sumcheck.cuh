@@ -24,6 +24,7 @@
 //       shared memory, including the final fold that yields final_m = f_m(rho).
 #pragma once
 #include <cooperative_groups.h>
+#include <cuda.h>
 #include <stdint.h>
 #include "field.cuh"
 
@@ -70,6 +71,7 @@ struct RoundParams {
     uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
     uint32_t cluster;     // thread-block cluster size along x (1 = none); divides ctas
     uint32_t zero;        // always 0 (opaque to the compiler: orders the fold-table loads, fixmul_lz)
+    uint32_t tma;         // 1: operands staged into shared memory by TMA (k_round<..., TMA = true>)
 };
 
 // ---------------------------------------------------------------- reductions
@@ -393,41 +395,134 @@ static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed3
 
 // ---------------------------------------------------------------- global round kernel
 
+// Raw entries of one table for pair j: E = 2 (round 1: a, b) or 4 (fused round: the two fold
+// pairs whose results are this round's (a, b)), in the order fold_group consumes them.
+template <int ORDER, bool FIRST> struct Geo {
+    static constexpr int E = FIRST ? 2 : 4;
+};
+
+// element offsets (relative to T + j) of the E raw entries of pair j in a table of E h entries
+template <int ORDER, bool FIRST>
+__device__ __forceinline__ uint64_t raw_off(uint64_t h, uint64_t j, int e) {
+    if (ORDER == 0) return (FIRST ? 2 : 4) * j + e;
+    if (FIRST) return j + (e ? h : 0);
+    // MSB fused: previous round paired (x, x + 2h); this round pairs (j, j + h)
+    return j + (e == 0 ? 0 : e == 1 ? 2 * h : e == 2 ? h : 3 * h);
+}
+
+// From the raw entries x[] of table m: round 1 -> (a, b); fused round -> fold both pairs with
+// r_{i-1}, store the folded pair to the other ping-pong buffer (Fig. 5), return (a, b - a).
+template <int D, int ORDER, bool FIRST>
+__device__ __forceinline__ void fold_group(const fe (&x)[Geo<ORDER, FIRST>::E], int m, fe *dst, uint64_t h,
+                                           uint64_t j, const fe *sK, uint32_t zmask, fe &a, fe &sv) {
+    fe lo, hi;
+    if (FIRST) {
+        lo = x[0];
+        hi = x[1];
+    } else {
+        lo = BZK_FOLD(x[0], x[1]);
+        hi = BZK_FOLD(x[2], x[3]);
+        fe *U = dst + (size_t)m * (2 * h);
+        if (ORDER == 0) { st_fe(U + 2 * j, lo); st_fe(U + 2 * j + 1, hi); }
+        else            { st_fe(U + j, lo);     st_fe(U + j + h, hi); }
+    }
+    a = lo;
+    // round 1: b; fused rounds: delta (for d = 2 the table-0 delta may stay < 4p: it only
+    // meets mul_acc, a full 512-bit product < 8p^2)
+    sv = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
+}
+
 template <int D, int ORDER, bool FIRST>
 __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, uint64_t j, const fe &rm,
                                           const fe *sK, uint32_t zmask, fe (&a)[D], fe (&sv)[D]) {
+    constexpr int E = Geo<ORDER, FIRST>::E;
 #pragma unroll
     for (int m = 0; m < D; ++m) {
-        fe lo, hi;
-        if (FIRST) {
-            const fe *T = src + (size_t)m * (2 * h);
-            if (ORDER == 0) { lo = ld_fe_stream(T + 2 * j); hi = ld_fe_stream(T + 2 * j + 1); }
-            else            { lo = ld_fe_stream(T + j);     hi = ld_fe_stream(T + j + h); }
-        } else {
-            const fe *T = src + (size_t)m * (4 * h);
-            fe *U = dst + (size_t)m * (2 * h);
-            if (ORDER == 0) {
-                fe x0 = ld_fe_stream(T + 4 * j), x1 = ld_fe_stream(T + 4 * j + 1);
-                fe x2 = ld_fe_stream(T + 4 * j + 2), x3 = ld_fe_stream(T + 4 * j + 3);
-                lo = BZK_FOLD(x0, x1);
-                hi = BZK_FOLD(x2, x3);
-                st_fe(U + 2 * j, lo);
-                st_fe(U + 2 * j + 1, hi);
-            } else {
-                // previous round paired (x, x + 2h); this round pairs (j, j + h)
-                fe x0 = ld_fe_stream(T + j), x1 = ld_fe_stream(T + j + 2 * h);
-                fe x2 = ld_fe_stream(T + j + h), x3 = ld_fe_stream(T + j + 3 * h);
-                lo = BZK_FOLD(x0, x1);
-                hi = BZK_FOLD(x2, x3);
-                st_fe(U + j, lo);
-                st_fe(U + j + h, hi);
-            }
-        }
-        a[m] = lo;
-        // round 1: b; fused rounds: delta (for d = 2 the table-0 delta may stay < 4p: it only
-        // meets mul_acc, a full 512-bit product < 8p^2)
-        sv[m] = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
+        const fe *T = src + (size_t)m * (E * h);
+        fe x[E];
+#pragma unroll
+        for (int e = 0; e < E; ++e) x[e] = ld_fe_stream(T + raw_off<ORDER, FIRST>(h, j, e));
+        fold_group<D, ORDER, FIRST>(x, m, dst, h, j, sK, zmask, a[m], sv[m]);
     }
+}
+
+// ---------------------------------------------------------------- TMA staging (k_round<..., TMA>)
+//
+// Each warp streams its 32 pairs' raw entries of every table into its own shared-memory slot with
+// one elected lane issuing cp.async.bulk.tensor copies (TMA, no registers held in flight) completing
+// on a per-(warp, table, stage) mbarrier.  The tensor map views the wave's source buffer as rows of
+// 128 B (32 x u32) with the 128-byte swizzle, so the lanes' 32-byte entries (row = the lane's 4
+// entries for LSB fused rounds) are read back with bank-conflict-free LDS.128.
+//   fused rounds: ONE stage per table; the copy of the next grid-stride tile of table m is issued
+//     as soon as table m's entries are folded (all lanes past their last use: __syncwarp), so it
+//     lands while the rest of this iteration and the next tables compute;
+//   round 1: TWO stages (no fold to hide behind), tile n + 2 issued at the end of iteration n.
+// Slot = E KiB per (warp, table, stage): LSB E entries of 32 lanes are one box of E * 8 rows; MSB
+// reads E segments of 8 rows (the pairs' halves are h entries apart).
+template <int ORDER, bool FIRST> struct TmaGeo {
+    static constexpr int E = Geo<ORDER, FIRST>::E;
+    static constexpr int NSTAGE = FIRST ? 2 : 1;
+    static constexpr uint32_t SLOT = E * 1024;
+    static constexpr uint32_t BOX_ROWS = ORDER == 0 ? E * 8 : 8;
+};
+
+template <int D, bool FIRST>
+constexpr size_t tma_smem_bytes() {   // + 1 KiB: the dynamic base is aligned up to 1 KiB in the kernel
+    return (size_t)(BZK_RT / 32) * D * TmaGeo<0, FIRST>::NSTAGE * TmaGeo<0, FIRST>::SLOT + 1024;
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile("{\n\t.reg .pred P1;\n\t"
+                 "BZK_WAIT:\n\t"
+                 "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+                 "@!P1 bra BZK_WAIT;\n\t}" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void tma_load_rows(void *dst, const CUtensorMap *tm, uint64_t row, uint64_t *bar) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                 ::"r"(smem_u32(dst)), "l"(tm), "r"(0), "r"((int)row), "r"(smem_u32(bar)) : "memory");
+}
+
+// lane 0: arm table m's barrier with the slot's bytes and copy the raw entries of pairs j0..j0+31
+template <int ORDER, bool FIRST>
+__device__ __forceinline__ void tma_issue(const CUtensorMap *tm, uint8_t *slot, uint64_t *bar, uint64_t row0,
+                                          uint64_t h, uint64_t j0) {
+    using G = TmaGeo<ORDER, FIRST>;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic reads of the slot before the async writes
+    mbar_expect_tx(bar, G::SLOT);
+    if (ORDER == 0) {
+        tma_load_rows(slot, tm, row0 + j0 * G::E / 4, bar);
+    } else {
+#pragma unroll
+        for (int e = 0; e < G::E; ++e) tma_load_rows(slot + e * 1024, tm, row0 + raw_off<ORDER, FIRST>(h, j0, e) / 4, bar);
+    }
+}
+
+// raw entry e of this lane's pair from a (swizzled) slot
+template <int ORDER, bool FIRST>
+__device__ __forceinline__ fe tma_entry(const uint8_t *slot, uint32_t lane, int e) {
+    uint32_t seg, row, c0;
+    if (ORDER == 0) {
+        seg = 0;
+        if (FIRST) { row = lane >> 1; c0 = 4 * (lane & 1) + 2 * e; }
+        else       { row = lane;      c0 = 2 * e; }
+    } else {
+        seg = e; row = lane >> 2; c0 = 2 * (lane & 3);
+    }
+    const uint8_t *base = slot + seg * 1024 + row * 128;
+    const uint4 x = *reinterpret_cast<const uint4 *>(base + ((c0 ^ (row & 7)) << 4));
+    const uint4 y = *reinterpret_cast<const uint4 *>(base + (((c0 + 1) ^ (row & 7)) << 4));
+    fe r;
+    r.l[0] = x.x; r.l[1] = x.y; r.l[2] = x.z; r.l[3] = x.w;
+    r.l[4] = y.x; r.l[5] = y.y; r.l[6] = y.z; r.l[7] = y.w;
+    return r;
 }
 
 #ifndef BZK_PF_DIST
@@ -465,8 +560,9 @@ __device__ __forceinline__ void prefetch_pairs(const fe *src, uint64_t h, uint64
     }
 }
 
-template <int D, int ORDER, bool FIRST>
-__global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(RoundParams P) {
+template <int D, int ORDER, bool FIRST, bool TMA>
+__global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
+    k_round(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
     constexpr bool DERIVE = !FIRST;
     constexpr int NV = Pts<D, DERIVE>::NV;
     __shared__ fe s_red[32 * NV];
@@ -488,10 +584,76 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1)) k_round(
     }
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
     const uint32_t lane = threadIdx.x & 31;
-    // One pair per loop iteration (keeps the loop body -- 2d folds + one two-pair evaluation -- small
-    // enough for the instruction cache); every second pair is held in registers and evaluated
-    // together with the next one, so the two pairs' products share one Montgomery reduction.
-    if constexpr (D >= 2) {
+    if constexpr (TMA) {
+        using G = TmaGeo<ORDER, FIRST>;
+        extern __shared__ uint8_t tma_raw[];
+        __shared__ __align__(8) uint64_t bars[(BZK_RT / 32) * D * G::NSTAGE];
+        uint8_t *tma_base = tma_raw + ((1024 - (smem_u32(tma_raw) & 1023)) & 1023);
+        const uint32_t warp = threadIdx.x >> 5;
+        uint8_t *wslots = tma_base + (size_t)warp * D * G::NSTAGE * G::SLOT;
+        uint64_t *wbars = bars + warp * D * G::NSTAGE;
+        if (lane == 0) {
+#pragma unroll
+            for (int q = 0; q < D * G::NSTAGE; ++q) mbar_init(&wbars[q]);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncwarp();
+        const uint64_t row0 = (uint64_t)b * D * (G::E * h / 4);   // this proof's first row (table 0)
+        const uint64_t trows = G::E * h / 4;                       // rows per table
+        const uint64_t j0 = (uint64_t)blockIdx.x * blockDim.x + warp * 32;
+        if (lane == 0)
+#pragma unroll
+            for (int s = 0; s < G::NSTAGE; ++s)
+                if (j0 + s * stride < h)
+#pragma unroll
+                    for (int m = 0; m < D; ++m)
+                        tma_issue<ORDER, FIRST>(&tmap, wslots + (s * D + m) * G::SLOT, &wbars[s * D + m],
+                                                row0 + m * trows, h, j0 + s * stride);
+        acc17 uacc[NV];
+#pragma unroll
+        for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
+        uint32_t it = 0;
+        for (uint64_t jw = j0; jw < h; jw += stride, ++it) {
+            const uint32_t s = G::NSTAGE == 1 ? 0 : (it & 1);
+            const uint32_t par = G::NSTAGE == 1 ? (it & 1) : ((it >> 1) & 1);
+            const uint64_t j = jw + lane;
+            fe a[D], sv[D];
+#pragma unroll
+            for (int m = 0; m < D; ++m) {
+                uint8_t *slot = wslots + (s * D + m) * G::SLOT;
+                mbar_wait(&wbars[s * D + m], par);
+                fe x[G::E];
+#pragma unroll
+                for (int e = 0; e < G::E; ++e) x[e] = tma_entry<ORDER, FIRST>(slot, lane, e);
+                fold_group<D, ORDER, FIRST>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
+                if (!FIRST) {
+                    __syncwarp();            // every lane has consumed the slot (the folds used x[])
+                    if (lane == 0 && jw + stride < h)
+                        tma_issue<ORDER, FIRST>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);
+                }
+            }
+            if constexpr (D >= 2) {
+                eval_one<D, DERIVE>(a, sv, uacc);
+            } else {
+                acc9_add(wacc[0], a[0]);
+                if (!DERIVE) acc9_add(wacc[1], sv[0]);
+            }
+            if (FIRST) {
+                __syncwarp();                // the evaluation consumed every lane's entries
+                if (lane == 0 && jw + 2 * stride < h)
+#pragma unroll
+                    for (int m = 0; m < D; ++m)
+                        tma_issue<ORDER, FIRST>(&tmap, wslots + (s * D + m) * G::SLOT, &wbars[s * D + m],
+                                                row0 + m * trows, h, jw + 2 * stride);
+            }
+        }
+        if constexpr (D >= 2) {
+#pragma unroll
+            for (int t = 0; t < NV; ++t) { wacc[t].lo = acc17_to_fe(uacc[t]); wacc[t].hi = 0; }
+        }
+    } else if constexpr (D >= 2) {
+        // One pair per loop iteration; the last product of every point goes unreduced into a
+        // 544-bit accumulator, reduced once after the loop.
         acc17 uacc[NV];
 #pragma unroll
         for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
@@ -689,7 +851,7 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
 // launchers, explicitly instantiated per degree in k_d<D>.cu (parallel compilation)
 template <int D>
 cudaError_t launch_round(uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
-                         const RoundParams &p);
+                         const RoundParams &p, const CUtensorMap &tm);
 template <int D>
 cudaError_t launch_tail(uint32_t order, uint32_t grid, uint32_t threads, size_t smem, cudaStream_t s,
                         const TailParams &p);

@@ -182,7 +182,7 @@ def test_mont_mul_lz_bounds(xb, yb):
     got = run_op(7, a, b)
     for x, y, r in zip(a, b, got):
         assert r % P == x * y * RINV % P
-        assert r < x * y // R + P and r < 1.76 * P, (x, y, r)
+        assert r * R < x * y + P * R and r < 1.76 * P, (x, y, r)     # t = (x y + q p) / R, q < R
 
 
 @pytest.mark.parametrize("xb,yb", [(2 * P, 2 * P), (P, R)])
@@ -298,7 +298,10 @@ def test_gl_lazy_ops():
     rng = np.random.default_rng(9)
     xs = gl_edges(rng, 2**64, 40)
     a, b = pairs(xs, xs)
-    for g, x, y in zip(gl_run(3, a, b), a, b):       # add_lazy: congruent, fits 64 bits
+    # add_lazy: x < 2^64 (a lazy sum), y canonical -- how eval_pair uses it (v + delta)
+    ya = gl_edges(rng, PGL, 40)
+    xa, yb = pairs(xs, ya)
+    for g, x, y in zip(gl_run(3, xa, yb), xa, yb):
         assert g % PGL == (x + y) % PGL and g < 2**64
     assert gl_run(4, a, b) == [((x << 64) + y) % PGL for x, y in zip(a, b)]   # reduce128(hi, lo)
     n = 256
