@@ -21,6 +21,7 @@
 #include "gl.cuh"
 #include "gen.cuh"
 #include "merkle.cuh"
+#include "multiround.cuh"
 #include "encoder.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
@@ -144,6 +145,8 @@ struct Plan {
     uint32_t cmax;
     bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
     uint32_t given;       // BZK_F_GIVEN_CHALLENGES
+    bool multi;           // given challenges, d = 1, BN254: k_multi passes (NEXT-1)
+    uint32_t part_nv;     // field elements per CTA partial (D + 1, or 2^kMultiM column sums)
     bool gl;              // BZK_F_FIELD_GOLDILOCKS (NEXT-2)
     size_t esz;           // bytes per element: 32 (BN254) or 8 (Goldilocks)
     size_t out_bytes_per_proof;
@@ -159,15 +162,27 @@ struct Knobs {
     // BZK_CLUSTER=N: CTAs of a proof form thread-block clusters of up to N (2, 4, 8) that combine
     // their partial sums through DSMEM.  Off by default: measured 10 % slower on B200.
     uint32_t cluster = 1;
-    // BZK_TMA=0/1: k_round stages its operands into shared memory with TMA (sumcheck.cuh) instead of
-    // loading them straight to registers
-    uint32_t tma = 0;
+    // k_round stages its operands into shared memory with TMA (sumcheck.cuh) instead of loading them
+    // straight to registers: by default for the fused rounds of d >= 2 and round 1 of d >= 3 (B200 A/B,
+    // profiles/r02/r02b_*: c2 fused rounds -11 % time, c2 round 1 +7 %, c3 both -3 %, m0 (d = 1) +3 %);
+    // BZK_TMA=0 / 1 forces it off / on everywhere
+    int tma = -1;
+    // BZK_MULTI=0/1: given-challenge d = 1 proofs run k_multi passes (several rounds per read of the
+    // table, multiround.cuh) instead of one k_round launch per round
+    uint32_t multi = 1;
+    uint32_t multi_m = 3;      // BZK_MULTI_M: rounds per k_multi pass (1..3)
     Knobs() {
+        if (const char *e = getenv("BZK_MULTI_M")) multi_m = std::max(1, std::min(3, atoi(e)));
+        if (const char *e = getenv("BZK_MULTI")) multi = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_TMA")) tma = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CLUSTER")) cluster = std::max(1, std::min(8, atoi(e)));
         if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_CTA_WAVES")) waves = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_PREFETCH")) prefetch = atoi(e) ? 1 : 0;
+    }
+    uint32_t tma_for(uint32_t d, bool first) const {
+        if (tma >= 0) return (uint32_t)tma;
+        return first ? (d >= 3 ? 1u : 0u) : (d >= 2 ? 1u : 0u);
     }
     uint32_t prefetch_for(uint32_t d) const {
         return prefetch < 0 ? (d >= 3 ? 1u : 0u) : (uint32_t)prefetch;
@@ -194,6 +209,26 @@ uint32_t ctas_for(uint64_t h, uint64_t nb) {
 uint32_t max_round_ctas(uint32_t k, uint32_t i0, uint64_t nb) {
     uint32_t c = 1;
     for (uint32_t i = 1; i < i0; ++i) c = std::max(c, ctas_for(1ull << (k - i), nb));
+    return c;
+}
+
+// Known-challenge multi-round passes (NEXT-1, d = 1): (K, m) per pass, K = variables left before the
+// pass, m <= 3 rounds per pass, until the on-chip tail's K_t = k - i0 + 1 variables remain.
+constexpr uint32_t kMultiM = 3;   // largest pass (k_multi instantiations; partials hold 2^kMultiM sums)
+std::vector<std::pair<uint32_t, uint32_t>> multi_passes(uint32_t k, uint32_t i0) {
+    std::vector<std::pair<uint32_t, uint32_t>> v;
+    const uint32_t Kt = k - i0 + 1;
+    for (uint32_t K = k; K > Kt;) {
+        const uint32_t m = std::min(knobs().multi_m, K - Kt);
+        v.push_back({K, m});
+        K -= m;
+    }
+    return v;
+}
+
+uint32_t max_multi_ctas(uint32_t k, uint32_t i0, uint64_t nb) {
+    uint32_t c = 1;
+    for (auto &pm : multi_passes(k, i0)) c = std::max(c, ctas_for(1ull << (pm.first - pm.second), nb));
     return c;
 }
 
@@ -243,6 +278,8 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     if (P.k == 0) { P.i0 = 1; P.log_h0 = 0; }
     else if (P.k - 1 <= kTailLog) { P.i0 = 1; P.log_h0 = P.k - 1; }
     else { P.i0 = P.k - kTailLog; P.log_h0 = kTailLog; }
+    P.multi = P.given && P.D == 1 && !P.gl && P.i0 > 1 && knobs().multi;
+    P.part_nv = P.multi ? (1u << kMultiM) : P.D + 1;
     const bool preserve = (b->flags & BZK_F_PRESERVE_INPUT) != 0;
     P.need_bufX = P.i0 > 2;
     P.need_bufY = P.i0 > 3;
@@ -264,8 +301,8 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
         size_t s = std::max(sizeof(ProofState), sizeof(gl::State)) + 4;
-        uint32_t c = P.k ? max_round_ctas(P.k, P.i0, bw) : 1;
-        s += (size_t)c * (P.D + 1) * P.esz;
+        uint32_t c = P.k ? (P.multi ? max_multi_ctas(P.k, P.i0, bw) : max_round_ctas(P.k, P.i0, bw)) : 1;
+        s += (size_t)c * P.part_nv * P.esz;
         if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * P.esz;
         if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * P.esz;
         if (P.host_tables) s += 2 * P.elem_table;
@@ -284,12 +321,13 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     bw = (P.B + nw - 1) / nw;
     P.Bw = bw; P.nwaves = nw;
     P.cmax = P.k ? std::max(max_round_ctas(P.k, P.i0, bw), max_round_ctas(P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
+    if (P.multi) P.cmax = std::max(max_multi_ctas(P.k, P.i0, bw), max_multi_ctas(P.k, P.i0, P.B - (nw - 1) * bw));
 
     size_t off = 0;
     P.off_seed = off; off += 256;
     P.off_ps = off; off = align_up(off + bw * std::max(sizeof(ProofState), sizeof(gl::State)));
     P.off_tick = off; off = align_up(off + bw * 4);
-    P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * (P.D + 1) * P.esz);
+    P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * P.part_nv * P.esz);
     P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * P.esz);
     P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * P.esz);
     P.off_out = off; if (P.host_outputs) off = align_up(off + P.B * P.out_bytes_per_proof);
@@ -496,7 +534,39 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         ++ctx->launches;
         CK(cudaGetLastError());
     }
-    for (uint32_t i = 1; i < P.i0; ++i) {
+    const fe *tail_src = nullptr;       // multi passes: the folded round-i0 table for k_tail
+    uint64_t tail_stride = 0;
+    if (P.multi) {
+        // NEXT-1: m rounds per read of the table (multiround.cuh).  MSB folds in place after the first
+        // pass (each thread owns its column); LSB ping-pongs between the two scratch buffers.
+        const fe *cur = tab;
+        uint64_t cur_stride = P.N;
+        uint32_t round = 1;
+        for (auto &pm : multi_passes(k, P.i0)) {
+            const uint32_t K = pm.first, m = pm.second;
+            MultiParams mp;
+            memset(&mp, 0, sizeof mp);
+            mp.src = cur; mp.src_stride = cur_stride;
+            if (round == 1) { mp.dst = bufX; mp.dst_stride = 1ull << (K - m); }
+            else if (P.order == 1) { mp.dst = const_cast<fe *>(cur); mp.dst_stride = cur_stride; }
+            else { mp.dst = (cur == bufX) ? bufY : bufX; mp.dst_stride = 1ull << (K - m); }
+            mp.logK = K; mp.round0 = round; mp.k = k;
+            mp.ctas = ctas_for(1ull << (K - m), io.nb);
+            mp.partials = part; mp.tickets = tick;
+            mp.challenges = (const fe *)io.challenges; mp.round_evals = (fe *)io.round_evals;
+            mp.claims = (fe *)io.claims;
+            dim3 grid(mp.ctas, (uint32_t)io.nb);
+            ProfScope ps_(ctx, s, 9);
+            cudaError_t e = multi_launch(P.order, m, grid, s, mp);
+            ++ctx->launches;
+            if (e != cudaSuccess) return cuda_fail(ctx, e, "k_multi launch");
+            cur = mp.dst; cur_stride = mp.dst_stride;
+            round += m;
+        }
+        tail_src = cur;
+        tail_stride = cur_stride;
+    }
+    for (uint32_t i = 1; i < (P.multi ? 1u : P.i0); ++i) {
         RoundParams rp;
         memset(&rp, 0, sizeof rp);
         rp.log_h = k - i;
@@ -516,7 +586,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         }
         CUtensorMap tm;
         memset(&tm, 0, sizeof tm);
-        rp.tma = knobs().tma;
+        rp.tma = knobs().tma_for(D, i == 1);
         if (rp.tma) {
             rp.prefetch = 0;
             const uint64_t E = i == 1 ? 2 : 4;   // raw entries per pair and table
@@ -538,7 +608,8 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         tp.final_evals = (fe *)io.final_evals; tp.claims = (fe *)io.claims;
         tp.consts = ctx->consts;
         tp.given = P.given;
-        if (P.i0 <= 2) tp.src = tab;
+        if (tail_src) { tp.src = tail_src; tp.folded = 1; tp.src_stride = tail_stride; }
+        else if (P.i0 <= 2) tp.src = tab;
         else tp.src = ((P.i0 - 1) % 2 == 0) ? bufX : bufY;
         size_t smem = k == 0 ? 0 : (size_t)D * 3 * (1ull << P.log_h0) * 32;
         ProfScope ps_(ctx, s, 2);

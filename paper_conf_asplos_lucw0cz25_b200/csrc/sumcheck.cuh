@@ -758,6 +758,8 @@ struct TailParams {
     fe *round_evals, *challenges, *final_evals, *claims;
     const fe *consts;
     uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
+    uint32_t folded;      // 1: src holds the round-i0 table itself ([D][2h0] per proof, i0 > 1: k_multi)
+    uint64_t src_stride;  // elements per proof in src (0: the default D * 2h0 or D * 4h0)
 };
 
 template <int D, int ORDER>
@@ -789,8 +791,8 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
     }
 
     // stage the round-i0 table (2h0 entries per m) into A
-    if (P.i0 == 1) {
-        const fe *src = P.src + (size_t)b * D * (2 * h0);
+    if (P.i0 == 1 || P.folded) {
+        const fe *src = P.src + (size_t)b * (P.src_stride ? P.src_stride : (size_t)D * (2 * h0));
         for (uint32_t x = threadIdx.x; x < (uint32_t)D * 2 * h0; x += blockDim.x) A[x] = ld_fe(src + x);
     } else {
         const fe *src = P.src + (size_t)b * D * (4 * h0);
