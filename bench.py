@@ -52,6 +52,9 @@ CONFIGS = {
                                        "SHA-256 of the 64-byte block (two compressions), every node level written"),
     "enc20": (256, 0, 20, 0, "code", "NEXT-4 linear-time encoder: 256 messages x 2^20 BN254 Fr elements (P:320 Table 5 "
                                      "shape), Spielman-style rate-1/2 code, left degrees 10/20, base 64 (readings R21-R24)"),
+    "c5": (8192, 2, 20, 0, "uniform", "configs[4]: 8192 proofs x product of 2 multilinears, k=20, BN254 Fr, sharded "
+                                      "by proof across the GPUs (strong scaling), waves of <= 1024 proofs per GPU "
+                                      "regenerated on the device between waves (untimed)"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -192,48 +195,66 @@ def enc_edges(code) -> int:
         int(code["G0"]["row_ptr"][-1])
 
 
-def cpu_baseline(cfg, max_proofs=8):
-    """The oracle as it stands on this box's host cores: a bounded sample of the same workload."""
+def cpu_model() -> str:
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def cpu_baseline(cfg, max_proofs=None):
+    """The oracle as it stands on this box's host cores: a bounded sample of the same workload
+    (default min(B, 4 x cores) proofs -- SURVEY.md 8(d) -- one per thread, all cores busy)."""
     import numpy as np  # noqa: F401
 
     import oracle
     from paper_conf_asplos_lucw0cz25_b200 import inputs
     B, d, k, order, dist, _ = CONFIGS[cfg]
     cores = len(os.sched_getaffinity(0))
-    n = max(1, min(max_proofs, cores, B))
+    n = max(1, min(max_proofs or 4 * cores, B))
+    threads = min(n, cores)
     oracle.build()
     if dist == "code":
         code = inputs.gen_code(k, 6)
         ms = inputs.gen_tables(n, 1, k, 0)[:, 0]
         t0 = time.perf_counter()
-        oracle.encode_batch(code, ms, nthreads=n)
+        oracle.encode_batch(code, ms, nthreads=threads)
         dt = time.perf_counter() - t0
-        return {"value": n / dt, "unit": "codes/s", "cores": n, "kind": "oracle",
-                "sample": f"{n} codewords of {cfg} (2^{k} elements), one per thread, {dt:.1f} s wall "
-                          f"= {n * dt:.0f} CPU-seconds"}
+        return {"value": n / dt, "unit": "codes/s", "cores": threads, "proofs": n, "kind": "oracle", "cpu_model": cpu_model(),
+                "sample": f"{n} codewords of {cfg} (2^{k} elements) on {threads} threads, {dt:.1f} s wall"}
     if dist == "blocks":
         blocks = inputs.gen_blocks(n, k, 0)
         t0 = time.perf_counter()
-        oracle.merkle_batch(blocks, k, d, nodes=True, nthreads=n)
+        oracle.merkle_batch(blocks, k, d, nodes=True, nthreads=threads)
         dt = time.perf_counter() - t0
-        return {"value": n / dt, "unit": "trees/s", "cores": n, "kind": "oracle",
-                "sample": f"{n} trees of {cfg} (2^{k} blocks, hash mode {d}), one per thread, {dt:.1f} s wall "
-                          f"= {n * dt:.0f} CPU-seconds"}
+        return {"value": n / dt, "unit": "trees/s", "cores": threads, "proofs": n, "kind": "oracle", "cpu_model": cpu_model(),
+                "sample": f"{n} trees of {cfg} (2^{k} blocks, hash mode {d}) on {threads} threads, {dt:.1f} s wall"}
     if dist == "gl":
         import concurrent.futures as cf
         tabs = inputs.gen_tables_gl(n, d, k, 0)
         t0 = time.perf_counter()
-        with cf.ThreadPoolExecutor(n) as ex:     # ctypes releases the GIL: one proof per thread
+        with cf.ThreadPoolExecutor(threads) as ex:     # ctypes releases the GIL: one proof per thread
             list(ex.map(lambda b: oracle.gl_prove(tabs[b], k, d, order, inputs.DEFAULT_SEED, b), range(n)))
+        dt = time.perf_counter() - t0
+    elif cfg == "m0lit":
+        import concurrent.futures as cf
+        tabs = inputs.gen_tables(n, d, k, 0, dist)
+        rs = [np.ascontiguousarray(inputs.gen_tables(1, 1, max(1, (k - 1).bit_length()), b, "uniform",
+                                                     data_seed=0x5052470000000000)[0, 0, :k]) for b in range(n)]
+        t0 = time.perf_counter()
+        with cf.ThreadPoolExecutor(threads) as ex:     # the oracle's given-challenge prover (Alg. 1)
+            list(ex.map(lambda b: oracle.prove_given(tabs[b], k, d, order, rs[b]), range(n)))
         dt = time.perf_counter() - t0
     else:
         tabs = inputs.gen_tables(n, d, k, 0, dist)
         t0 = time.perf_counter()
-        oracle.prove_batch(tabs, k, d, order, inputs.DEFAULT_SEED, 0, nthreads=n)
+        oracle.prove_batch(tabs, k, d, order, inputs.DEFAULT_SEED, 0, nthreads=threads)
         dt = time.perf_counter() - t0
-    return {"value": n / dt, "unit": "proofs/s", "cores": n, "kind": "oracle",
-            "sample": f"{n} proofs of {cfg} (d={d}, k={k}), one per thread, {dt:.1f} s wall "
-                      f"= {n * dt:.0f} CPU-seconds"}
+    return {"value": n / dt, "unit": "proofs/s", "cores": threads, "proofs": n, "kind": "oracle", "cpu_model": cpu_model(),
+            "sample": f"{n} proofs of {cfg} (d={d}, k={k}) on {threads} threads, {dt:.1f} s wall"}
 
 
 def run_reference(args, rank, world):
@@ -247,8 +268,8 @@ def run_reference(args, rank, world):
     cb = None
     for _ in range(args.steps):
         cb = cpu_baseline(args.config, max_proofs=args.ref_proofs)
-        times.append(cb["cores"] / cb["value"])
-    nproofs = cb["cores"]
+        times.append(cb["proofs"] / cb["value"])
+    nproofs = cb["proofs"]
     value = nproofs * len(times) / sum(times)
     unit = cb["unit"]
     metric = {"blocks": MERKLE_METRIC, "code": ENC_METRIC}.get(dist, METRIC)
@@ -257,8 +278,8 @@ def run_reference(args, rank, world):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * sum(times) / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
             "data": "synthetic", "config": {"workload": desc, "batch_sampled": nproofs, "d": d, "k": k},
-            "cpu_baseline": {"value": value, "unit": unit, "cores": nproofs, "kind": "oracle",
-                             "sample": cb["sample"]},
+            "cpu_baseline": {"value": value, "unit": unit, "cores": cb["cores"], "kind": "oracle",
+                             "cpu_model": cb.get("cpu_model"), "sample": cb["sample"]},
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -630,6 +651,353 @@ def run_encoder(args, rank, world):
     if dist:
         dist.destroy_process_group()
 
+# ---------------------------------------------------------------- sum-check (configs c1, c2, c3, c5, m0, m0lit, g2)
+
+GOLDEN_DIGESTS = os.path.join(ROOT, "tests", "golden", "c5_proof_digests.txt")
+# IMAD-pipe slots of the kernels' products: a 32 x 32 -> 64-bit limb product is one
+# IMAD.WIDE = 2 fma-heavy slots.  Fixed-multiplier fold (fixmul_lz): 64 + 18 products; unreduced
+# 256 x 256-bit product into a 544-bit accumulator (mul_acc): 64; full Montgomery product: 136.
+SLOT_FIXMUL, SLOT_MULACC, SLOT_MONT = 164, 128, 272
+
+
+def multi_passes(k: int, m_max: int = 3):
+    """api.cu multi_passes: (K, m) of the known-challenge k_multi passes (d = 1, NEXT-1)."""
+    tail_log = 8
+    i0 = 1 if k - 1 <= tail_log else k - tail_log
+    kt, out, K = k - i0 + 1, [], k
+    while K > kt:
+        m = min(m_max, K - kt)
+        out.append((K, m))
+        K -= m
+    return out
+
+
+def imad_slots(d: int, k: int, kind: str) -> int:
+    """fma-heavy slots of the products one proof's launches of `kind` execute (the kernels' arithmetic,
+    DESIGN.md sec. 6): round 1 sums d+1 points per pair, each (d-2) Montgomery products + 1 unreduced
+    product; a fused round folds 2d entries per pair and sums d points (g(1) derived); a k_multi pass
+    does one unreduced product per entry."""
+    tail_log = 8
+    i0 = 1 if k - 1 <= tail_log else k - tail_log
+    point = 0 if d == 1 else (d - 2) * SLOT_MONT + SLOT_MULACC
+    if kind == "round1":
+        return (d + 1) * point * (1 << (k - 1)) if i0 > 1 else 0
+    if kind == "fused":
+        return sum((2 * d * SLOT_FIXMUL + d * point) * (1 << (k - i)) for i in range(2, i0))
+    if kind == "multi":
+        return sum(SLOT_MULACC * (1 << K) for K, _ in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3"))))
+    raise ValueError(kind)
+
+
+def multi_bytes(k: int) -> int:
+    """algorithmic HBM bytes per proof of the k_multi passes: each reads its table once, writes 2^-m"""
+    return sum(32 * ((1 << K) + (1 << (K - m))) for K, m in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3"))))
+
+
+def proof_digests(out: dict) -> list:
+    """per-proof digest (tests/golden/make_golden_c5.py): sha256(round_evals || challenges ||
+    final_evals || claim)[:8], LE u64 limbs as the C ABI lays them out"""
+    import hashlib
+    arrs = [out[k_].cpu().numpy() for k_ in ("round_evals", "challenges", "final_evals", "claims")]
+    res = []
+    for b in range(arrs[0].shape[0]):
+        h = hashlib.sha256()
+        for a in arrs:
+            h.update(a[b].tobytes())
+        res.append(h.hexdigest()[:16])
+    return res
+
+
+def golden_check(digests: list, first: int, cfg: str) -> dict | None:
+    """compare per-proof digests with the oracle-written golden file (d = 2, k = 20, LSB, uniform)"""
+    if cfg not in ("c2", "c5") or not os.path.exists(GOLDEN_DIGESTS):
+        return None
+    gold = {}
+    for ln in open(GOLDEN_DIGESTS):
+        if ln.strip() and not ln.startswith("#"):
+            i, dg = ln.split()
+            gold[int(i)] = dg
+    checked = [(first + n, dg) for n, dg in enumerate(digests) if first + n in gold]
+    bad = [i for i, dg in checked if gold[i] != dg]
+    return {"proofs_checked": len(checked), "proofs_total": len(digests), "mismatches": len(bad),
+            "first_mismatch": bad[0] if bad else None,
+            "source": "tests/golden/c5_proof_digests.txt (per-proof SHA-256 of the CPU oracle's outputs, "
+                      "written by tests/golden/make_golden_c5.py from oracle/ only)"}
+
+
+def run_sumcheck(args, rank, world, local):
+    import torch
+
+    from paper_conf_asplos_lucw0cz25_b200 import bzk
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+
+    B, d, k, order, gen_dist, desc = CONFIGS[args.config]
+    strong = args.config == "c5"
+    if strong:
+        # configs[4]: the GLOBAL batch is fixed; rank r proves the contiguous indices shard_range(B, W, r)
+        # in waves of <= --wave proofs, each wave's tables regenerated on the device (untimed)
+        global_B = args.batch or B
+        first, count = shard.shard_range(global_B, world, rank)
+        wave = max(1, min(count, args.wave))
+        waves = [(first + w0, min(wave, count - w0)) for w0 in range(0, count, wave)]
+    else:
+        if args.batch:
+            B = args.batch
+        first, count = shard.weak_range(B, rank)
+        global_B = B * world
+        wave = count
+        waves = [(first, count)]
+    consume = args.config == "c3" or strong
+    gl = gen_dist == "gl"
+    esz = 8 if gl else 32
+    flags = 0 if consume else bzk.BZK_F_PRESERVE_INPUT
+    if gl:
+        flags |= bzk.BZK_F_FIELD_GOLDILOCKS
+
+    def tshape(n):
+        return (n, d, 1 << k) if gl else (n, d, 1 << k, 4)
+    given = args.config == "m0lit"
+    if given:
+        flags |= bzk.BZK_F_GIVEN_CHALLENGES
+    stream = torch.cuda.Stream()
+    tables = torch.empty(tshape(wave), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(tables, waves[0][1], d, k, waves[0][0], gen_dist, stream=stream)
+    prover = bzk.Prover(local)
+    out = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(count, k, d)
+    if given:
+        # pre-seeded challenges (the paper's PRG output, P:211): canonical values from the generator
+        kk = max(1, (k - 1).bit_length())          # generator tables have 2^kk >= k entries
+        g = torch.empty((count, 1, 1 << kk, 4), dtype=torch.int64, device="cuda")
+        bzk.bzk_generate(g, count, 1, kk, first, "uniform", data_seed=0x5052470000000000, stream=stream)
+        with torch.cuda.stream(stream):          # ordered after the generator on the same stream
+            out["challenges"].copy_(g[:, 0, :k, :])
+        stream.synchronize()
+
+    def wave_out(w0, n):
+        return {key: v[w0 - first:w0 - first + n] for key, v in out.items()}
+    batches = [prover.batch(tables, k, d, order, None, w0, flags, wave_out(w0, n), batch=n) for w0, n in waves]
+    seed_keep = list(prover._seed_bufs)  # noqa: F841 (the job structs point at this seed buffer)
+    # weak scaling (one wave per rank): the whole step is captured once and replayed as a CUDA graph
+    batch_g = None if strong else prover.batch(tables, k, d, order, None, first, flags | bzk.BZK_F_GRAPH, out)
+
+    def regen(w0, n):
+        bzk.bzk_generate(tables, n, d, k, w0, gen_dist, stream=stream)
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        if batch_g is not None:
+            if consume:
+                regen(first, count)
+            bzk.bzk_prove(prover.ctx, batch_g, stream)   # the first call captures the CUDA graph
+        else:
+            for (w0, n), b in zip(waves, batches):
+                regen(w0, n)
+                bzk.bzk_prove(prover.ctx, b, stream)
+    stream.synchronize()
+
+    def timed_region(use_graph, profile):
+        calls = [(w0, n, batch_g if use_graph else b) for (w0, n), b in zip(waves, batches)]
+        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in calls]
+              for _ in range(args.steps)]
+        bzk.bzk_profile_enable(prover.ctx, profile)
+        bzk.bzk_profile_read(prover.ctx, reset=True)
+        bzk.bzk_launch_count(prover.ctx, reset=True)
+        barrier()
+        with ClockSampler(local) as clk:
+            for i in range(args.steps):
+                for c, (w0, n, b) in enumerate(calls):
+                    if consume:
+                        regen(w0, n)                     # untimed: outside the events
+                    ev[i][c][0].record(stream)
+                    bzk.bzk_prove(prover.ctx, b, stream)
+                    ev[i][c][1].record(stream)
+            stream.synchronize()
+            barrier()
+        launches = bzk.bzk_launch_count(prover.ctx, reset=True)
+        prof = bzk.bzk_profile_read(prover.ctx, reset=True)
+        bzk.bzk_profile_enable(prover.ctx, False)
+        return [sum(a.elapsed_time(b_) for a, b_ in row) for row in ev], launches, prof, clk.summary()
+
+    # timed region 1 (the headline value): weak scaling replays the whole step as one CUDA graph; the
+    # strong-scaling waves are launched call by call
+    step_ms, launches, _, clocks = timed_region(batch_g is not None, False)
+    # timed region 2 (roofline): the same steps launched kernel by kernel with CUDA events around
+    # every launch on the launch stream (per-kernel device time)
+    step_ms_prof, _, prof, _ = timed_region(False, True)
+    my_ms = float(sum(step_ms))
+
+    # ---------------- outputs: digests, gather to rank 0, golden check (outside the timed regions)
+    keys = ("round_evals", "challenges", "final_evals", "claims")
+    digest = shard.output_digest([out[key].cpu() for key in keys])
+    max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
+    digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
+    gathered, gold = None, None
+    if dist:
+        # the proofs themselves are gathered to rank 0 over NCCL (NVLink) after the timed region
+        # (north star: "NCCL is used only to gather proofs and timing"); rank 0 digests the global batch
+        torch.cuda.synchronize()
+        g0 = time.perf_counter()
+        allp = shard.gather_outputs({k_: out[k_] for k_ in keys}, dist, dst=0)
+        torch.cuda.synchronize()
+        g_ms = (time.perf_counter() - g0) * 1000.0
+        if rank == 0:
+            gbytes = sum(v.numel() * v.element_size() for v in allp.values())
+            gathered = {"proofs": int(allp["claims"].shape[0]), "bytes": int(gbytes), "ms": round(g_ms, 3),
+                        "backend": dist.get_backend(), "collective": "gather to rank 0",
+                        "global_digest": shard.output_digest([allp[k_].cpu() for k_ in keys])}
+            if not gl and d == 2 and k == 20 and order == 0 and gen_dist == "uniform":
+                gold = golden_check(proof_digests(allp), 0, args.config if strong else "c2")
+    elif not gl and d == 2 and k == 20 and order == 0 and gen_dist == "uniform" and not given:
+        gold = golden_check(proof_digests(out), first, args.config if strong else "c2")
+
+    total_proofs = global_B * args.steps
+    value = total_proofs / (max_ms / 1000.0)
+    ms_per_step = max_ms / args.steps
+
+    # ---------------- roofline of the dominant kernel
+    hbm_peak, sm_max_mhz, peak_src = peaks()
+    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused", "multi_round": "multi"}
+    dom = max(kinds, key=lambda n: prof[n][0])
+    dom_ms, dom_cnt = prof[dom]
+    launches_per_step = max(1, dom_cnt / args.steps)
+    avg_launch_s = dom_ms / max(1, dom_cnt) / 1000.0
+    slot_peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6          # fma-heavy slots / s
+    slots_per_launch = imad_slots(d, k, kinds[dom]) * count / launches_per_step
+    if kinds[dom] == "multi":
+        bytes_per_launch = multi_bytes(k) * count / launches_per_step
+        mulmods_per_launch = sum((1 << K) for K, _ in multi_passes(k)) * count / launches_per_step
+    else:
+        bytes_per_launch = alg_bytes_kind(d, k, kinds[dom], esz) * count / launches_per_step
+        mulmods_per_launch = alg_mulmods(d, k, kinds[dom]) * count / launches_per_step
+    ach_slots = slots_per_launch / avg_launch_s
+    ach_gbs = bytes_per_launch / avg_launch_s / 1e9
+    int_peak = slot_peak / IMAD_PER_MULMOD / 1e9                 # G mulmod/s (r01 unit, 272 slots)
+    mulmod_rate = mulmods_per_launch / avg_launch_s / 1e9
+    t_alu = slots_per_launch / slot_peak
+    t_hbm = bytes_per_launch / (hbm_peak * 1e9)
+    total_alg = alg_mulmods(d, k, "total") * count
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        # DRAM bytes per launch of the dominant kernel from one `ncu --set full` capture of the same
+        # command, if it was taken on this workload and build
+        with open(tpath) as f:
+            tj = json.load(f)
+        for e in (tj if isinstance(tj, list) else [tj]):
+            if e.get("config") == args.config and e.get("kernel_kind") == dom and e.get("batch") == count:
+                traffic = e["dram_bytes_per_launch"]
+    if t_alu >= t_hbm and not gl:
+        roofline = {"bound": "alu", "kernel": dom, "achieved": round(ach_slots / 1e12, 3),
+                    "peak": round(slot_peak / 1e12, 3), "unit": "T IMAD-slot/s",
+                    "frac": round(ach_slots / slot_peak, 4), "traffic": traffic,
+                    "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} fma-heavy slots/clk x "
+                                   f"{sm_max_mhz:.0f} MHz ({peak_src} max clock); achieved = the kernel's product "
+                                   "slots per launch (fixmul fold 164, unreduced 256x256 product 128, Montgomery "
+                                   "product 272; DESIGN.md sec. 6) / CUDA-event launch time"}
+    else:
+        roofline = {"bound": "hbm", "kernel": dom, "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
+                    "frac": round(ach_gbs / hbm_peak, 4), "traffic": traffic,
+                    "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); achieved = algorithmic bytes per "
+                                   "launch / CUDA-event launch time"}
+    roofline.update({"alg_bytes_per_launch": bytes_per_launch, "imad_slots_per_launch": slots_per_launch,
+                     "alu_time_at_peak_ms": round(t_alu * 1000, 4), "hbm_time_at_peak_ms": round(t_hbm * 1000, 4),
+                     "imad_frac": round(ach_slots / slot_peak, 4), "hbm_frac": round(ach_gbs / hbm_peak, 4),
+                     "mulmod_equiv": {"achieved": round(mulmod_rate, 2), "peak": round(int_peak, 2),
+                                      "unit": "Gmulmod/s (272-slot schoolbook unit, r01)",
+                                      "frac": round(mulmod_rate / int_peak, 4)},
+                     "step_mulmod_frac": round(total_alg / (ms_per_step / 1000.0) / 1e9 / int_peak, 4),
+                     "step_hbm_alg_frac": round(d * (1 << k) * esz * count / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
+                     "hbm_peak_gbs": hbm_peak})
+
+    kernel_ms = {n: round(v[0] / args.steps, 3) for n, v in prof.items() if v[1]}
+    line = {"metric": METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+            "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "u64" if gl else "u32",
+            "data": "synthetic",
+            "config": {"workload": desc, "batch_per_gpu": count, "global_batch": global_B, "d": d, "k": k,
+                       "order": "LSB" if order == 0 else "MSB", "field": "Goldilocks" if gl else "BN254 Fr",
+                       "waves_per_gpu": len(waves), "wave_size": wave,
+                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (wave * d * (1 << k) * esz / 2**30)},
+            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
+            "kernel_ms_per_step": kernel_ms, "ms_per_step_kernel_by_kernel": round(sum(step_ms_prof) / args.steps, 3),
+            "roofline": roofline, "clocks": clocks,
+            "digest_rank0": digests[0], "digests_per_rank": len(digests)}
+    if dist:
+        line["dist"] = {"backend": dist.get_backend(), "world_size": dist.get_world_size(),
+                        "nccl_version": ".".join(map(str, torch.cuda.nccl.version())) if dist.get_backend() == "nccl"
+                        else None, "data_path_collectives": 0}
+    if gathered:
+        line["proofs_gathered"] = gathered
+    if gold:
+        line["golden_check"] = gold
+
+    # ---------------- e2e: host (pinned) tables in, host outputs out, through bzk_prove
+    if not args.no_e2e and args.config != "c3":
+        del tables
+        torch.cuda.empty_cache()
+        # pinned host memory is shared by all ranks of the node: cap each rank's e2e batch at 40 % of
+        # the available host memory / world (same metric, proofs/s, on a smaller host-resident batch)
+        try:
+            avail = os.sysconf("SC_AVPHYS_PAGES") * os.sysconf("SC_PAGE_SIZE")
+        except (ValueError, OSError):
+            avail = 1 << 40
+        proof_bytes = d * (1 << k) * esz
+        Be = int(max(1, min(wave, 0.4 * avail / world // proof_bytes)))
+        host_t = torch.empty(tshape(Be), dtype=torch.int64, pin_memory=True)
+        chunk = max(1, Be // 16)
+        tmp = torch.empty(tshape(chunk), dtype=torch.int64, device="cuda")
+        for c0 in range(0, Be, chunk):
+            n = min(chunk, Be - c0)
+            bzk.bzk_generate(tmp, n, d, k, first + c0, gen_dist, stream=stream)
+            stream.synchronize()
+            host_t[c0:c0 + n].copy_(tmp[:n])
+        del tmp
+        torch.cuda.empty_cache()
+        out_h = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(Be, k, d, device="cpu", pin=True)
+        if given:
+            out_h["challenges"].copy_(out["challenges"][:Be])
+        hb = prover.batch(host_t, k, d, order, None, first,
+                          flags & (bzk.BZK_F_GIVEN_CHALLENGES | bzk.BZK_F_FIELD_GOLDILOCKS), out_h)
+        bzk.bzk_prove(prover.ctx, hb, stream)   # warm-up (allocates staging)
+        barrier()
+        t0 = time.perf_counter()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            bzk.bzk_prove(prover.ctx, hb, stream)   # host tables + host outputs: returns after D2H
+        e1.record(stream)
+        stream.synchronize()
+        barrier()
+        wall = time.perf_counter() - t0
+        e2e_ms = shard.max_over_ranks(e0.elapsed_time(e1), dist, device="cuda")
+        out_bytes = sum(v.numel() * 8 for v in out_h.values())
+        same = all(torch.equal(out_h[key], out[key][:Be].cpu()) for key in out_h)
+        line["e2e"] = {"value": round(Be * world * args.e2e_steps / (e2e_ms / 1000.0), 2), "unit": "proofs/s",
+                       "batch_per_gpu": Be,
+                       "h2d_bytes_per_step": int(host_t.numel() * 8), "d2h_bytes_per_step": int(out_bytes),
+                       "steps": args.e2e_steps, "wall_s": round(wall, 3), "matches_device_run": bool(same),
+                       "path": "bzk_prove(tables_mem=HOST pinned, outputs_mem=HOST): side-stream H2D waves "
+                               "overlapping compute"}
+    if rank == 0 and world == 1 and not args.no_cpu:
+        line["cpu_baseline"] = cpu_baseline(args.config, max_proofs=args.ref_proofs)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    prover.close()
+    if dist:
+        dist.destroy_process_group()
+
 
 def main():
     ap = argparse.ArgumentParser()
@@ -643,8 +1011,9 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--ref-proofs", type=int, default=8)
+    ap.add_argument("--ref-proofs", type=int, default=None, help="oracle sample (default min(B, 4 x cores))")
     ap.add_argument("--vml-chunk", type=int, default=0, help="c4: images per job group (0 = all)")
+    ap.add_argument("--wave", type=int, default=1024, help="c5: proofs per wave on each GPU (<= 1024)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
@@ -668,244 +1037,7 @@ def main():
         run_encoder(args, rank, world)
         return
 
-    import numpy as np
-    import torch
-
-    from paper_conf_asplos_lucw0cz25_b200 import bzk
-    torch.cuda.set_device(local)
-    dist = None
-    if world > 1:
-        import torch.distributed as dist
-        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        else:
-            dist.init_process_group(backend)
-
-    B, d, k, order, gen_dist, desc = CONFIGS[args.config]
-    if args.batch:
-        B = args.batch
-    first, _ = shard.weak_range(B, rank)
-    consume = args.config == "c3"
-    gl = gen_dist == "gl"
-    esz = 8 if gl else 32
-    flags = 0 if consume else bzk.BZK_F_PRESERVE_INPUT
-    if gl:
-        flags |= bzk.BZK_F_FIELD_GOLDILOCKS
-
-    def tshape(n):
-        return (n, d, 1 << k) if gl else (n, d, 1 << k, 4)
-    if args.config == "m0lit":
-        flags |= bzk.BZK_F_GIVEN_CHALLENGES
-    stream = torch.cuda.Stream()
-    tables = torch.empty(tshape(B), dtype=torch.int64, device="cuda")
-    bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
-    prover = bzk.Prover(local)
-    out = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(B, k, d)
-    if flags & bzk.BZK_F_GIVEN_CHALLENGES:
-        # pre-seeded challenges (the paper's PRG output): any canonical values < 2^253
-        kk = max(1, (k - 1).bit_length())          # generator tables have 2^kk >= k entries
-        g = torch.empty((B, 1, 1 << kk, 4), dtype=torch.int64, device="cuda")
-        bzk.bzk_generate(g, B, 1, kk, first, "uniform", data_seed=0x5052470000000000, stream=stream)
-        with torch.cuda.stream(stream):          # ordered after the generator on the same stream
-            out["challenges"].copy_(g[:, 0, :k, :])
-        stream.synchronize()
-    batch = prover.batch(tables, k, d, order, None, first, flags, out)
-
-    batch_g = prover.batch(tables, k, d, order, None, first, flags | bzk.BZK_F_GRAPH, out)
-
-    def step(b):
-        if consume:
-            # consume mode destroys the input: regenerate it (untimed) before every step
-            bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
-        bzk.bzk_prove(prover.ctx, b, stream)
-
-    for _ in range(args.warmup):
-        step(batch_g)        # the first call captures the CUDA graph of the whole step
-    stream.synchronize()
-
-    def barrier():
-        if dist:
-            dist.barrier()
-        torch.cuda.synchronize()
-
-    def timed_region(b, profile):
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-        bzk.bzk_profile_enable(prover.ctx, profile)
-        bzk.bzk_profile_read(prover.ctx, reset=True)
-        bzk.bzk_launch_count(prover.ctx, reset=True)
-        barrier()
-        with ClockSampler(local) as clk:
-            for i in range(args.steps):
-                if consume:
-                    bzk.bzk_generate(tables, B, d, k, first, gen_dist, stream=stream)
-                ev[i][0].record(stream)
-                bzk.bzk_prove(prover.ctx, b, stream)
-                ev[i][1].record(stream)
-            stream.synchronize()
-            barrier()
-        launches = bzk.bzk_launch_count(prover.ctx, reset=True)
-        prof = bzk.bzk_profile_read(prover.ctx, reset=True)
-        bzk.bzk_profile_enable(prover.ctx, False)
-        return [a.elapsed_time(b_) for a, b_ in ev], launches, prof, clk.summary()
-
-    # timed region 1 (the headline value): the whole step replayed as one CUDA graph
-    step_ms, launches, _, clocks = timed_region(batch_g, False)
-    # timed region 2 (roofline): the same steps launched kernel by kernel with CUDA events around
-    # every launch on the launch stream (per-kernel device time)
-    step_ms_prof, _, prof, _ = timed_region(batch, True)
-    my_ms = float(sum(step_ms))
-
-    # output digest (for cross-GPU-count comparisons) -- outside the timed region
-    digest = shard.output_digest([out[key].cpu() for key in ("round_evals", "challenges", "final_evals", "claims")])
-
-    max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
-    digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
-    # the proofs themselves are gathered to rank 0 over NCCL (NVLink) after the timed region
-    # (north star: "NCCL is used only to gather proofs and timing"); rank 0 digests the global batch
-    gathered = None
-    if dist:
-        torch.cuda.synchronize()
-        g0 = time.perf_counter()
-        allp = shard.gather_outputs({k_: out[k_] for k_ in ("round_evals", "challenges", "final_evals", "claims")},
-                                    dist, dst=0)
-        torch.cuda.synchronize()
-        g_ms = (time.perf_counter() - g0) * 1000.0
-        if rank == 0:
-            gbytes = sum(v.numel() * v.element_size() for v in allp.values())
-            gathered = {"proofs": B * world, "bytes": int(gbytes), "ms": round(g_ms, 3),
-                        "backend": dist.get_backend(),
-                        "global_digest": shard.output_digest([allp[k_].cpu() for k_ in
-                                                              ("round_evals", "challenges", "final_evals", "claims")])}
-
-    total_proofs = B * world * args.steps
-    value = total_proofs / (max_ms / 1000.0)
-    ms_per_step = max_ms / args.steps
-
-    # ---------------- roofline of the dominant kernel (ALU-bound: integer pipe)
-    hbm_peak, sm_max_mhz, peak_src = peaks()
-    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused"}
-    dom = max(kinds, key=lambda n: prof[n][0])
-    dom_ms, dom_cnt = prof[dom]
-    mulmods_per_launch = alg_mulmods(d, k, kinds[dom]) * B / max(1, dom_cnt / args.steps)
-    avg_launch_s = dom_ms / max(1, dom_cnt) / 1000.0
-    achieved = mulmods_per_launch / avg_launch_s / 1e9
-    int_peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6 / IMAD_PER_MULMOD / 1e9
-    total_alg = alg_mulmods(d, k, "total") * B
-    step_gmulmod = total_alg / (ms_per_step / 1000.0) / 1e9
-    # HBM: algorithmic bytes (read each input once) and the streaming schedule's bytes
-    alg_bytes = d * (1 << k) * esz * B
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tpath):
-        # DRAM bytes per launch of the dominant kernel from one `ncu --set full` capture of the same
-        # command (scripts/ncu_traffic.sh), if it was taken on this workload
-        with open(tpath) as f:
-            tj = json.load(f)
-        for e in (tj if isinstance(tj, list) else [tj]):
-            if e.get("config") == args.config and e.get("kernel_kind") == dom and e.get("batch") == B:
-                traffic = e["dram_bytes_per_launch"]
-    bytes_per_launch = alg_bytes_kind(d, k, kinds[dom], esz) * B / max(1, dom_cnt / args.steps)
-    roofline = {"bound": "alu", "kernel": dom, "achieved": round(achieved, 2), "peak": round(int_peak, 2),
-                "unit": "Gmulmod/s", "frac": round(achieved / int_peak, 4), "traffic": traffic,
-                "alg_bytes_per_launch": bytes_per_launch,
-                "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} MHz "
-                               f"({peak_src} max clock) / {IMAD_PER_MULMOD} IMAD per mulmod",
-                "step_frac": round(step_gmulmod / int_peak, 4),
-                "hbm_alg_frac": round(alg_bytes / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
-                "hbm_peak_gbs": hbm_peak}
-    # the dominant kernel's bound: the larger of its algorithmic IMAD time and HBM time at the peaks
-    # (d = 1 fused rounds move 192 B per 2 products: HBM-bound; d >= 2 BN254 rounds: IMAD-bound)
-    t_alu = mulmods_per_launch / (int_peak * 1e9)
-    t_hbm = bytes_per_launch / (hbm_peak * 1e9)
-    ach_gbs = bytes_per_launch / avg_launch_s / 1e9
-    roofline["alu_time_at_peak_ms"] = round(t_alu * 1000, 4)
-    roofline["hbm_time_at_peak_ms"] = round(t_hbm * 1000, 4)
-    if not gl and t_hbm > t_alu:
-        roofline.update({"bound": "hbm", "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
-                         "frac": round(ach_gbs / hbm_peak, 4),
-                         "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); this kernel's algorithmic "
-                                        "HBM time exceeds its IMAD time at the roofs",
-                         "alu_gmulmod_s": round(achieved, 2), "alu_frac": round(achieved / int_peak, 4)})
-    if gl:
-        # Goldilocks (8-byte elements): the dominant kernel streams; its roof is HBM bandwidth
-        roofline.update({"bound": "hbm", "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
-                         "frac": round(ach_gbs / hbm_peak, 4),
-                         "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_src}); achieved = algorithmic bytes per "
-                                        "launch (reads 4dh + writes 2dh elements per proof for a fused round, 2dh "
-                                        "reads for round 1) / CUDA-event launch time",
-                         "alu_gmulmod_s": round(achieved, 2)})
-
-    kernel_ms = {n: round(v[0] / args.steps, 3) for n, v in prof.items() if v[1]}
-    line = {"metric": METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64" if gl else "u32", "data": "synthetic",
-            "config": {"workload": desc, "batch_per_gpu": B, "global_batch": B * world, "d": d, "k": k,
-                       "order": "LSB" if order == 0 else "MSB", "field": "Goldilocks" if gl else "BN254 Fr",
-                       "l2": "inputs larger than L2 (%.0f GiB vs 126 MB); no flush" % (B * d * (1 << k) * esz / 2**30)},
-            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps,
-            "kernel_ms_per_step": kernel_ms, "ms_per_step_kernel_by_kernel": round(sum(step_ms_prof) / args.steps, 3),
-            "roofline": roofline, "clocks": clocks,
-            "digest_rank0": digests[0], "digests_per_rank": len(digests)}
-    if gathered:
-        line["proofs_gathered"] = gathered
-
-    # ---------------- e2e: host (pinned) tables in, host outputs out, through bzk_prove
-    if not args.no_e2e and not consume:
-        del tables
-        torch.cuda.empty_cache()
-        # pinned host memory is shared by all ranks of the node: cap each rank's e2e batch at 40 % of
-        # the available host memory / world (same metric, proofs/s, on a smaller host-resident batch)
-        try:
-            avail = os.sysconf("SC_AVPHYS_PAGES") * os.sysconf("SC_PAGE_SIZE")
-        except (ValueError, OSError):
-            avail = 1 << 40
-        proof_bytes = d * (1 << k) * esz
-        Be = int(max(1, min(B, 0.4 * avail / world // proof_bytes)))
-        host_t = torch.empty(tshape(Be), dtype=torch.int64, pin_memory=True)
-        chunk = max(1, Be // 16)
-        tmp = torch.empty(tshape(chunk), dtype=torch.int64, device="cuda")
-        for c0 in range(0, Be, chunk):
-            n = min(chunk, Be - c0)
-            bzk.bzk_generate(tmp, n, d, k, first + c0, gen_dist, stream=stream)
-            stream.synchronize()
-            host_t[c0:c0 + n].copy_(tmp[:n])
-        del tmp
-        torch.cuda.empty_cache()
-        out_h = (bzk.Prover.alloc_outputs_gl if gl else bzk.Prover.alloc_outputs)(Be, k, d, device="cpu", pin=True)
-        if flags & bzk.BZK_F_GIVEN_CHALLENGES:
-            out_h["challenges"].copy_(out["challenges"][:Be])
-        hb = prover.batch(host_t, k, d, order, None, first,
-                          flags & (bzk.BZK_F_GIVEN_CHALLENGES | bzk.BZK_F_FIELD_GOLDILOCKS), out_h)
-        bzk.bzk_prove(prover.ctx, hb, stream)   # warm-up (allocates staging)
-        barrier()
-        t0 = time.perf_counter()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(args.e2e_steps):
-            bzk.bzk_prove(prover.ctx, hb, stream)   # host tables + host outputs: returns after D2H
-        e1.record(stream)
-        stream.synchronize()
-        barrier()
-        wall = time.perf_counter() - t0
-        e2e_ms = e0.elapsed_time(e1)
-        e2e_ms = shard.max_over_ranks(e2e_ms, dist, device="cuda")
-        out_bytes = sum(v.numel() * 8 for v in out_h.values())
-        same = all(torch.equal(out_h[key], out[key][:Be].cpu()) for key in out_h)
-        line["e2e"] = {"value": round(Be * world * args.e2e_steps / (e2e_ms / 1000.0), 2), "unit": "proofs/s",
-                       "batch_per_gpu": Be,
-                       "h2d_bytes_per_step": int(host_t.numel() * 8), "d2h_bytes_per_step": int(out_bytes),
-                       "steps": args.e2e_steps, "wall_s": round(wall, 3), "matches_device_run": bool(same),
-                       "path": "bzk_prove(tables_mem=HOST pinned, outputs_mem=HOST): side-stream H2D waves "
-                               "overlapping compute"}
-    if rank == 0 and world == 1 and not args.no_cpu:
-        line["cpu_baseline"] = cpu_baseline(args.config)
-    if rank == 0:
-        print(json.dumps(line), flush=True)
-    prover.close()
-    if dist:
-        dist.destroy_process_group()
-
+    run_sumcheck(args, rank, world, local)
 
 if __name__ == "__main__":
     main()

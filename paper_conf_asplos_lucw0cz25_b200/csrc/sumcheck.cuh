@@ -456,12 +456,13 @@ __device__ __forceinline__ void load_pair(const fe *src, fe *dst, uint64_t h, ui
 //   fused rounds: ONE stage per table; the copy of the next grid-stride tile of table m is issued
 //     as soon as table m's entries are folded (all lanes past their last use: __syncwarp), so it
 //     lands while the rest of this iteration and the next tables compute;
-//   round 1: TWO stages (no fold to hide behind), tile n + 2 issued at the end of iteration n.
+//   round 1: THREE stages (no fold to hide behind and a short iteration): at the top of iteration n
+//     tile n + 2 goes into the stage iteration n - 1 consumed.
 // Slot = E KiB per (warp, table, stage): LSB E entries of 32 lanes are one box of E * 8 rows; MSB
 // reads E segments of 8 rows (the pairs' halves are h entries apart).
 template <int ORDER, bool FIRST> struct TmaGeo {
     static constexpr int E = Geo<ORDER, FIRST>::E;
-    static constexpr int NSTAGE = FIRST ? 2 : 1;
+    static constexpr int NSTAGE = FIRST ? 3 : 1;
     static constexpr uint32_t SLOT = E * 1024;
     static constexpr uint32_t BOX_ROWS = ORDER == 0 ? E * 8 : 8;
 };
@@ -603,7 +604,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
         const uint64_t j0 = (uint64_t)blockIdx.x * blockDim.x + warp * 32;
         if (lane == 0)
 #pragma unroll
-            for (int s = 0; s < G::NSTAGE; ++s)
+            for (int s = 0; s < (FIRST ? G::NSTAGE - 1 : 1); ++s)
                 if (j0 + s * stride < h)
 #pragma unroll
                     for (int m = 0; m < D; ++m)
@@ -614,9 +615,17 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
         for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
         uint32_t it = 0;
         for (uint64_t jw = j0; jw < h; jw += stride, ++it) {
-            const uint32_t s = G::NSTAGE == 1 ? 0 : (it & 1);
-            const uint32_t par = G::NSTAGE == 1 ? (it & 1) : ((it >> 1) & 1);
+            const uint32_t s = G::NSTAGE == 1 ? 0 : it % G::NSTAGE;
+            const uint32_t par = G::NSTAGE == 1 ? (it & 1) : ((it / G::NSTAGE) & 1);
             const uint64_t j = jw + lane;
+            if (FIRST && lane == 0 && jw + (G::NSTAGE - 1) * stride < h) {
+                // the stage of tile it + NSTAGE - 1 was consumed by iteration it - 1 (__syncwarp below)
+                const uint32_t sn = (it + G::NSTAGE - 1) % G::NSTAGE;
+#pragma unroll
+                for (int m = 0; m < D; ++m)
+                    tma_issue<ORDER, FIRST>(&tmap, wslots + (sn * D + m) * G::SLOT, &wbars[sn * D + m],
+                                            row0 + m * trows, h, jw + (G::NSTAGE - 1) * stride);
+            }
             fe a[D], sv[D];
 #pragma unroll
             for (int m = 0; m < D; ++m) {
@@ -638,14 +647,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
                 acc9_add(wacc[0], a[0]);
                 if (!DERIVE) acc9_add(wacc[1], sv[0]);
             }
-            if (FIRST) {
-                __syncwarp();                // the evaluation consumed every lane's entries
-                if (lane == 0 && jw + 2 * stride < h)
-#pragma unroll
-                    for (int m = 0; m < D; ++m)
-                        tma_issue<ORDER, FIRST>(&tmap, wslots + (s * D + m) * G::SLOT, &wbars[s * D + m],
-                                                row0 + m * trows, h, jw + 2 * stride);
-            }
+            if (FIRST) __syncwarp();         // the evaluation consumed every lane's entries of stage s
         }
         if constexpr (D >= 2) {
 #pragma unroll

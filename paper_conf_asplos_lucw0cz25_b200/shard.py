@@ -58,20 +58,29 @@ def gather_bytes(blob: bytes, dist, device=None) -> list[bytes]:
 
 
 def gather_outputs(tensors: dict, dist, dst: int = 0):
-    """Gather each rank's output tensors (equal shapes per rank) to rank ``dst``, concatenated
-    along the proof dimension in rank order.  Returns the dict on ``dst``, None elsewhere."""
+    """Gather each rank's output tensors to rank ``dst`` (torch.distributed.gather: only ``dst``
+    receives), concatenated along the proof dimension in rank order.  Ranks may hold different proof
+    counts (strong scaling with a remainder): every rank pads to the largest count and ``dst`` trims.
+    Returns the dict on ``dst``, None elsewhere."""
     import torch
     if dist is None or not dist.is_initialized() or dist.get_world_size() == 1:
         return tensors
     world, rank = dist.get_world_size(), dist.get_rank()
-    out = {}
     nccl = dist.get_backend() == "nccl"
+    any_t = next(iter(tensors.values()))
+    dev = any_t.device if (nccl and any_t.is_cuda) else torch.device("cpu")
+    cnt = torch.tensor([any_t.shape[0]], dtype=torch.int64, device=dev)
+    counts = [torch.zeros_like(cnt) for _ in range(world)]
+    dist.all_gather(counts, cnt)
+    counts = [int(c.item()) for c in counts]
+    top = max(counts)
+    out = {}
     for key in sorted(tensors):
-        t = tensors[key].contiguous()
-        if not nccl and t.is_cuda:
-            t = t.cpu()                      # gloo: host tensors
-        parts = [torch.empty_like(t) for _ in range(world)]
-        dist.all_gather(parts, t)
+        t = tensors[key].to(dev).contiguous()
+        if t.shape[0] < top:
+            t = torch.cat([t, t.new_zeros((top - t.shape[0],) + tuple(t.shape[1:]))])
+        parts = [torch.empty_like(t) for _ in range(world)] if rank == dst else None
+        dist.gather(t, parts, dst=dst)
         if rank == dst:
-            out[key] = torch.cat(parts, dim=0)
+            out[key] = torch.cat([p[:c] for p, c in zip(parts, counts)], dim=0)
     return out if rank == dst else None
