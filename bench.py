@@ -55,6 +55,9 @@ CONFIGS = {
     "c5": (8192, 2, 20, 0, "uniform", "configs[4]: 8192 proofs x product of 2 multilinears, k=20, BN254 Fr, sharded "
                                       "by proof across the GPUs (strong scaling), waves of <= 1024 proofs per GPU "
                                       "regenerated on the device between waves (untimed)"),
+    "zk20": (64, 2, 20, 0, "chain", "NEXT-4 section-4 chain per proof (P:207-213): a 2^20-element input in S=4 segments "
+                                    "of 2^18, each encoded (rate 1/2) and committed with a Merkle tree, root of roots, "
+                                    "then a d=2, k=20 sum-check seeded with the final root (P:211)"),
     "c4": (64, 2, 16, 0, "vml", "configs[3]: verifiable-ML workload, VGG-16/CIFAR-10-shaped layer sum-checks (2 degree-2 "
                                 "sum-checks per layer, k_l = ceil(log2 max(in_l, out_l))), streamed host->device"),
 }
@@ -999,6 +1002,129 @@ def run_sumcheck(args, rank, world, local):
         dist.destroy_process_group()
 
 
+CHAIN_METRIC = "section-4 chain proofs/s (encode + Merkle commit + root of roots + sum-check, NEXT-4)"
+CHAIN_SEGMENTS, CHAIN_LOG_N = 4, 18
+
+
+def run_chain(args, rank, world, local):
+    """NEXT-4: bzk_commit_prove over a batch -- per proof S segments encoded, each codeword committed
+    (Merkle tree over its 64-byte blocks), the S roots combined by a root-of-roots tree, and a sum-check
+    (d = 2, k = 20) seeded with the final root, all in one stream-ordered library call."""
+    import torch
+
+    from paper_conf_asplos_lucw0cz25_b200 import bzk, inputs
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    B, d, k, order, _, desc = CONFIGS[args.config]
+    if args.batch:
+        B = args.batch
+    S, log_n = CHAIN_SEGMENTS, CHAIN_LOG_N
+    n = 1 << log_n
+    first, _ = shard.weak_range(B, rank)
+    code = inputs.gen_code(log_n, 6)
+    enc = bzk.Encoder(code, local)
+    stream = torch.cuda.Stream()
+    msgs = torch.empty((B * S, 1, n, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(msgs, B * S, 1, log_n, first * S, "uniform", data_seed=0x42415443485A4B53, stream=stream)
+    codes = torch.empty((B, S, 2 * n, 4), dtype=torch.int64, device="cuda")
+    roots = torch.empty((B, S, 32), dtype=torch.uint8, device="cuda")
+    fin = torch.empty((B, 32), dtype=torch.uint8, device="cuda")
+    tables = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(tables, B, d, k, first, "uniform", stream=stream)
+    out = bzk.Prover.alloc_outputs(B, k, d)
+    stream.synchronize()
+    commit = bzk.bzk_commit(S, bzk.BZK_MERKLE_COMPRESS, codes.data_ptr(), roots.data_ptr(), None, fin.data_ptr())
+    sb = bzk.make_batch(k, d, order, bzk.BZK_F_PRESERVE_INPUT, B, first, None, tables, bzk.BZK_MEM_DEVICE,
+                        bzk.BZK_MEM_DEVICE, out["round_evals"], out["challenges"], out["final_evals"], out["claims"])
+
+    def reset():
+        with torch.cuda.stream(stream):       # untimed: every step encodes the same messages
+            codes.view(B * S, 2 * n, 4)[:, :n].copy_(msgs[:, 0])
+
+    def barrier():
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        reset()
+        bzk.bzk_commit_prove(enc.ctx, enc.enc, commit, sb, stream)
+    stream.synchronize()
+
+    def timed(profile):
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+        bzk.bzk_profile_enable(enc.ctx, profile)
+        bzk.bzk_profile_read(enc.ctx, reset=True)
+        bzk.bzk_launch_count(enc.ctx, reset=True)
+        barrier()
+        with ClockSampler(local) as clk:
+            for i in range(args.steps):
+                reset()
+                ev[i][0].record(stream)
+                bzk.bzk_commit_prove(enc.ctx, enc.enc, commit, sb, stream)
+                ev[i][1].record(stream)
+            stream.synchronize()
+            barrier()
+        launches = bzk.bzk_launch_count(enc.ctx, reset=True)
+        prof = bzk.bzk_profile_read(enc.ctx, reset=True)
+        bzk.bzk_profile_enable(enc.ctx, False)
+        return float(sum(a.elapsed_time(b) for a, b in ev)), launches, prof, clk.summary()
+
+    my_ms, launches, _, clocks = timed(False)
+    _, _, prof, _ = timed(True)
+    max_ms = shard.max_over_ranks(my_ms, dist, device="cuda")
+    digest = shard.output_digest([fin.cpu()] + [out[key].cpu() for key in ("round_evals", "challenges", "final_evals",
+                                                                           "claims")])
+    digests = [x.hex() for x in shard.gather_bytes(bytes.fromhex(digest), dist, device="cuda")]
+    ms_per_step = max_ms / args.steps
+    value = B * world * args.steps / (max_ms / 1000.0)
+    kernel_ms = {nm: round(v[0] / args.steps, 3) for nm, v in prof.items() if v[1]}
+    # roofline of the dominant kernel kind (encoder products: IMAD; Merkle stages: ALU; sum-check rounds)
+    hbm_peak, sm_max_mhz, peak_src = peaks()
+    dom = max(kernel_ms, key=kernel_ms.get)
+    edges = enc_edges(code)
+    roof = {"kernel": dom}
+    if dom == "encoder_spmv":
+        ach = B * S * edges / (kernel_ms[dom] / 1000.0) / 1e9
+        peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6 / IMAD_PER_EDGE_PRODUCT / 1e9
+        roof.update({"bound": "alu", "achieved": round(ach, 2), "peak": round(peak, 2), "unit": "Gproduct/s",
+                     "frac": round(ach / peak, 4), "traffic": None,
+                     "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} IMAD/clk x {sm_max_mhz:.0f} MHz "
+                                    f"/ {IMAD_PER_EDGE_PRODUCT} IMAD slots per edge product"})
+    elif dom == "merkle_stage":
+        hashes = B * S * (2 * n - 1) + B * (S - 1)
+        ach = hashes / (kernel_ms[dom] / 1000.0) / 1e9
+        peak = SMS * ALU_PER_CLK_SM * sm_max_mhz * 1e6 / ALU_OPS_PER_COMPRESSION / 1e9
+        roof.update({"bound": "alu", "achieved": round(ach, 3), "peak": round(peak, 3), "unit": "Ghash/s",
+                     "frac": round(ach / peak, 4), "traffic": None})
+    else:
+        slots = (imad_slots(d, k, "round1") + imad_slots(d, k, "fused")) * B
+        t_all = (kernel_ms.get("round1_eval", 0) + kernel_ms.get("fused_fold_eval", 0)) / 1000.0
+        ach = slots / t_all
+        peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6
+        roof.update({"bound": "alu", "achieved": round(ach / 1e12, 3), "peak": round(peak / 1e12, 3),
+                     "unit": "T IMAD-slot/s", "frac": round(ach / peak, 4), "traffic": None})
+    line = {"metric": CHAIN_METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": desc, "proofs_per_gpu": B, "segments": S, "segment_log_n": log_n, "d": d, "k": k,
+                       "edges_per_codeword": edges, "l2": "codewords + tables larger than L2; no flush"},
+            "gpu_launches": launches, "gpu_launches_per_step": launches / args.steps, "kernel_ms_per_step": kernel_ms,
+            "roofline": roof, "clocks": clocks, "digest_rank0": digests[0], "digests_per_rank": len(digests)}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    enc.close()
+    if dist:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -1035,6 +1161,9 @@ def main():
         return
     if CONFIGS[args.config][4] == "code":
         run_encoder(args, rank, world)
+        return
+    if CONFIGS[args.config][4] == "chain":
+        run_chain(args, rank, world, local)
         return
 
     run_sumcheck(args, rank, world, local)

@@ -335,3 +335,26 @@ def encode_batch(code: dict, msgs: np.ndarray, nthreads: int | None = None) -> n
     if s:
         raise ValueError(f"orc_encode_batch failed: {s}")
     return out
+
+
+# ---------------------------------------------------------------- the section-4 chain (NEXT-4)
+
+def commit_prove(code: dict, segments: np.ndarray, tables: np.ndarray, k: int, d: int, order: int, index: int,
+                 mode: int = MERKLE_COMPRESS):
+    """One proof of the chain of PAPER.md:207-213 (Sec. 4, Fig. 7), step by step:
+    1. every message segment is encoded (P:209 "each encoded into an error-correction code");
+    2. every codeword is committed with a Merkle tree over its bytes as 64-byte blocks (P:209);
+    3. "these roots serve as leaf nodes for another Merkle tree module, ultimately yielding a single
+       final root" (P:209): level 1 = H(root_2j || root_2j+1), ..., one root (S = 1: the root itself);
+    4. the sum-check's transcript is seeded with the final root (reading R25).
+    segments: uint64 [S][n][4].  Returns (codewords [S][2n][4], roots [S][32], final root, proof dict)."""
+    S = segments.shape[0]
+    assert S >= 1 and S & (S - 1) == 0
+    codes = np.stack([encode(code, segments[s]) for s in range(S)])
+    roots = np.stack([np.frombuffer(merkle(codes[s].astype("<u8").view(np.uint8).reshape(-1, 64),
+                                           code["log_n"], mode, nodes=False)[0], np.uint8) for s in range(S)])
+    if S == 1:
+        final = roots[0].tobytes()
+    else:
+        final = merkle(roots.reshape(S // 2, 64), (S // 2).bit_length() - 1, mode, nodes=False)[0]
+    return codes, roots, final, prove(tables, k, d, order, final, index)

@@ -25,6 +25,7 @@ BZK_ORDER_LSB, BZK_ORDER_MSB = 0, 1
 BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
 BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
 BZK_F_FIELD_GOLDILOCKS = 32
+BZK_F_SEEDS_DEVICE = 64
 BZK_PROF_KINDS = 10
 PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy",
                    "merkle_stage", "d2h_copy", "encoder_spmv", "multi_round"]
@@ -34,7 +35,7 @@ EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_
            "bzk_strerror", "bzk_last_error", "bzk_generate", "bzk_profile_enable", "bzk_profile_read",
            "bzk_launch_count", "bzk_debug_field", "bzk_debug_sha256", "bzk_debug_bench", "bzk_version",
            "bzk_merkle", "bzk_generate_blocks", "bzk_encoder_create", "bzk_encoder_destroy", "bzk_encode",
-           "bzk_debug_gl"]
+           "bzk_debug_gl", "bzk_commit_prove"]
 
 
 class BzkError(RuntimeError):
@@ -61,6 +62,11 @@ class bzk_merkle_batch(ctypes.Structure):
 class bzk_csr(ctypes.Structure):
     _fields_ = [("rows", ctypes.c_uint32), ("cols", ctypes.c_uint32), ("nnz", ctypes.c_uint64),
                 ("row_ptr", ctypes.c_void_p), ("col", ctypes.c_void_p), ("val", ctypes.c_void_p)]
+
+
+class bzk_commit(ctypes.Structure):
+    _fields_ = [("segments", ctypes.c_uint32), ("hash", ctypes.c_uint32), ("codes", ctypes.c_void_p),
+                ("roots", ctypes.c_void_p), ("nodes", ctypes.c_void_p), ("final_roots", ctypes.c_void_p)]
 
 
 class bzk_code(ctypes.Structure):
@@ -107,10 +113,11 @@ def lib():
         L.bzk_encoder_destroy.argtypes = [vp]
         L.bzk_encoder_destroy.restype = None
         L.bzk_encode.argtypes = [vp, vp, vp, u64, u32, u32, vp]
+        L.bzk_commit_prove.argtypes = [vp, vp, ctypes.POINTER(bzk_commit), ctypes.POINTER(bzk_batch), vp]
         for name in ("bzk_create", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",
                      "bzk_generate", "bzk_profile_enable", "bzk_profile_read", "bzk_debug_field",
                      "bzk_debug_sha256", "bzk_debug_bench", "bzk_debug_gl", "bzk_merkle", "bzk_generate_blocks",
-                     "bzk_encoder_create", "bzk_encode"):
+                     "bzk_encoder_create", "bzk_encode", "bzk_commit_prove"):
             getattr(L, name).restype = i32
         _lib = L
     return _lib
@@ -236,6 +243,10 @@ def bzk_encoder_destroy(enc) -> None:
 
 def bzk_encode(ctx, enc, codes, batch: int, codes_mem: int = BZK_MEM_DEVICE, flags: int = 0, stream=None) -> None:
     _check(lib().bzk_encode(ctx, enc, ptr(codes), batch, codes_mem, flags, _stream_handle(stream)), ctx)
+
+
+def bzk_commit_prove(ctx, enc, commit: bzk_commit, sumcheck: bzk_batch, stream=None) -> None:
+    _check(lib().bzk_commit_prove(ctx, enc, ctypes.byref(commit), ctypes.byref(sumcheck), _stream_handle(stream)), ctx)
 
 
 def bzk_profile_enable(ctx, on: bool) -> None:

@@ -461,6 +461,7 @@ __global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
 
 struct WaveIO {
     Seed32 seed;       // transcript seed, passed to the kernel by value
+    const uint8_t *seeds;   // BZK_F_SEEDS_DEVICE: this wave's per-proof seeds (device [nb][32]), else null
     char *tables;      // device tables of this wave [nb][D][N] x esz
     char *round_evals, *challenges, *final_evals, *claims;   // device outputs of this wave
     uint64_t nb, first_index;
@@ -478,7 +479,7 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
     const uint32_t D = P.D, k = P.k;
     {
         ProfScope ps_(ctx, s, 3);
-        cudaError_t e = gl_launch_init(ps, (uint32_t)io.nb, io.seed.b, io.first_index, k, D, P.order, s);
+        cudaError_t e = gl_launch_init(ps, (uint32_t)io.nb, io.seed.b, io.seeds, io.first_index, k, D, P.order, s);
         ++ctx->launches;
         if (e != cudaSuccess) return cuda_fail(ctx, e, "gl init launch");
     }
@@ -529,7 +530,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
     const uint32_t D = P.D, k = P.k;
     {
         ProfScope ps_(ctx, s, 3);
-        k_transcript_init<<<(uint32_t)((io.nb + 127) / 128), 128, 0, s>>>(ps, (uint32_t)io.nb, io.seed,
+        k_transcript_init<<<(uint32_t)((io.nb + 127) / 128), 128, 0, s>>>(ps, (uint32_t)io.nb, io.seed, io.seeds,
                                                                           io.first_index, k, D, P.order);
         ++ctx->launches;
         CK(cudaGetLastError());
@@ -646,8 +647,14 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     }
     for (uint64_t w = 0; w < P.nwaves; ++w) {
         WaveIO io;
-        memcpy(io.seed.b, b->seed, 32);
         const uint64_t b0 = w * P.Bw;
+        if (b->flags & BZK_F_SEEDS_DEVICE) {
+            memset(io.seed.b, 0, 32);
+            io.seeds = b->seed + b0 * 32;
+        } else {
+            memcpy(io.seed.b, b->seed, 32);
+            io.seeds = nullptr;
+        }
         io.nb = std::min<uint64_t>(P.Bw, P.B - b0);
         io.first_index = b->first_index + b0;
         io.round_evals = o_ev + b0 * ev_pp;
@@ -729,7 +736,9 @@ bzk_status prove_jobs(bzk_ctx *ctx, const bzk_batch *jobs, size_t njobs, cudaStr
         kp += sizeof(s);
         for (size_t j = 0; j < njobs; ++j) {
             memcpy(kp, &jobs[j], sizeof(bzk_batch));
-            memcpy(kp + sizeof(bzk_batch), jobs[j].seed, 32);
+            // host seed: its bytes; device seeds (BZK_F_SEEDS_DEVICE): the pointer in the struct is the key
+            if (jobs[j].flags & BZK_F_SEEDS_DEVICE) memset(kp + sizeof(bzk_batch), 0, 32);
+            else memcpy(kp + sizeof(bzk_batch), jobs[j].seed, 32);
             kp += sizeof(bzk_batch) + 32;
         }
     }
@@ -1210,6 +1219,57 @@ bzk_status encode_impl(bzk_ctx *ctx, const bzk_encoder *E, uint64_t *codes, uint
     return BZK_OK;
 }
 
+// ---------------------------------------------------------------- the section-4 chain (NEXT-4)
+//
+// P:207-213 (Fig. 7): each proof's input is divided into segments, each segment is encoded, every
+// codeword is committed with a Merkle tree, the codeword roots are the leaves of another tree whose
+// root seeds the sum-check's random numbers.  One call runs the chain over a batch of proofs, every
+// step in the library's kernels, stream-ordered (no host round trip between the modules).
+
+bzk_status commit_prove_impl(bzk_ctx *ctx, const bzk_encoder *E, const bzk_commit *c, const bzk_batch *sc,
+                             cudaStream_t s) {
+    NvtxRange nv_("bzk_commit_prove");
+    if (!E || !c || !sc) return fail(ctx, BZK_EINVAL, "encoder/commit/sumcheck is NULL");
+    if (!c->codes || !c->roots || !c->final_roots) return fail(ctx, BZK_EINVAL, "codes/roots/final_roots is NULL");
+    const uint32_t S = c->segments;
+    if (S == 0 || (S & (S - 1)) || S > (1u << 20)) return fail(ctx, BZK_EINVAL, "segments must be a power of two <= 2^20");
+    if (c->hash > 1) return fail(ctx, BZK_EINVAL, "hash must be BZK_MERKLE_COMPRESS or BZK_MERKLE_SHA256");
+    if (sc->flags & (BZK_F_SEEDS_DEVICE | BZK_F_GIVEN_CHALLENGES))
+        return fail(ctx, BZK_EINVAL, "the chain derives the seeds: no BZK_F_SEEDS_DEVICE / BZK_F_GIVEN_CHALLENGES");
+    bzk_batch b2 = *sc;                  // the sum-check, its transcripts seeded with the final roots
+    b2.flags |= BZK_F_SEEDS_DEVICE;
+    b2.seed = c->final_roots;
+    bzk_status st = validate_args(ctx, &b2);   // every argument error before the first launch
+    if (st) return st;
+    const uint64_t B = sc->batch;
+    // 1. encode the B x S segments in place (codeword = message || redundancy, bzk_encode)
+    st = encode_impl(ctx, E, c->codes, B * S, BZK_MEM_DEVICE, 0, s);
+    if (st) return st;
+    // 2. a Merkle tree per codeword: 2n elements = n blocks of 64 bytes (two elements per block)
+    bzk_merkle_batch m1;
+    memset(&m1, 0, sizeof m1);
+    m1.log_blocks = E->log_n; m1.hash = c->hash; m1.blocks_mem = BZK_MEM_DEVICE; m1.batch = B * S;
+    m1.blocks = (const uint8_t *)c->codes; m1.outputs_mem = BZK_MEM_DEVICE; m1.roots = c->roots; m1.nodes = c->nodes;
+    st = merkle_impl(ctx, &m1, s);
+    if (st) return st;
+    // 3. root of roots: the S roots of a proof are the leaves, so level 1 = H(root_2j || root_2j+1) =
+    //    the level 0 of a tree over S / 2 blocks (adjacent root pairs, already contiguous in `roots`)
+    if (S == 1) {
+        CK(cudaMemcpyAsync(c->final_roots, c->roots, B * 32, cudaMemcpyDeviceToDevice, s));
+    } else {
+        uint32_t lg = 0;
+        while ((2u << lg) < S) ++lg;
+        bzk_merkle_batch m2;
+        memset(&m2, 0, sizeof m2);
+        m2.log_blocks = lg; m2.hash = c->hash; m2.blocks_mem = BZK_MEM_DEVICE; m2.batch = B;
+        m2.blocks = c->roots; m2.outputs_mem = BZK_MEM_DEVICE; m2.roots = c->final_roots;
+        st = merkle_impl(ctx, &m2, s);
+        if (st) return st;
+    }
+    // 4. the sum-check of every proof, its transcript seeded with its final root
+    return prove_jobs(ctx, &b2, 1, s);
+}
+
 // ---------------------------------------------------------------- debug kernels
 
 __global__ void k_debug_field(int op, uint64_t n, const fe *a, const fe *b, fe *out) {
@@ -1589,6 +1649,13 @@ bzk_status bzk_encode(bzk_ctx *ctx, const bzk_encoder *enc, uint64_t *codes, uin
     if (!ctx) return BZK_EINVAL;
     cudaSetDevice(ctx->device);
     return encode_impl(ctx, enc, codes, batch, codes_mem, flags, (cudaStream_t)cuda_stream);
+}
+
+bzk_status bzk_commit_prove(bzk_ctx *ctx, const bzk_encoder *enc, const bzk_commit *commit, const bzk_batch *sumcheck,
+                            void *cuda_stream) {
+    if (!ctx) return BZK_EINVAL;
+    cudaSetDevice(ctx->device);
+    return commit_prove_impl(ctx, enc, commit, sumcheck, (cudaStream_t)cuda_stream);
 }
 
 bzk_status bzk_generate_blocks(uint8_t *dst, uint64_t batch, uint32_t n, uint64_t first_index, uint64_t data_seed,

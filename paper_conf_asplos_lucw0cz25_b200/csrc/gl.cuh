@@ -192,12 +192,18 @@ __device__ __forceinline__ void finalize(uint64_t (&g)[D + 1], uint32_t round, S
 
 struct Seed32Gl { uint8_t b[32]; };
 
-static __global__ void k_gl_transcript_init(State *ps, uint32_t nproofs, Seed32Gl seed, uint64_t first_index,
-                                            uint32_t k, uint32_t d, uint32_t order) {
+static __global__ void k_gl_transcript_init(State *ps, uint32_t nproofs, Seed32Gl seed, const uint8_t *seeds,
+                                            uint64_t first_index, uint32_t k, uint32_t d, uint32_t order) {
     uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
     if (b >= nproofs) return;
     uint32_t st[8];
-    transcript_init(st, seed.b, first_index + b, k, d, order, 1u);
+    if (seeds) {
+        Seed32Gl own;
+        for (int i = 0; i < 32; ++i) own.b[i] = seeds[(size_t)b * 32 + i];
+        transcript_init(st, own.b, first_index + b, k, d, order, 1u);
+    } else {
+        transcript_init(st, seed.b, first_index + b, k, d, order, 1u);
+    }
 #pragma unroll
     for (int i = 0; i < 8; ++i) ps[b].st[i] = st[i];
 }
@@ -448,8 +454,8 @@ cudaError_t gl_launch_round(uint32_t D, uint32_t order, bool first, dim3 grid, u
                             const gl::RoundParams &p);
 cudaError_t gl_launch_tail(uint32_t D, uint32_t order, uint32_t grid, uint32_t threads, size_t smem, cudaStream_t s,
                            const gl::TailParams &p);
-cudaError_t gl_launch_init(gl::State *ps, uint32_t nproofs, const uint8_t seed[32], uint64_t first_index, uint32_t k,
-                           uint32_t d, uint32_t order, cudaStream_t s);
+cudaError_t gl_launch_init(gl::State *ps, uint32_t nproofs, const uint8_t seed[32], const uint8_t *seeds_dev,
+                           uint64_t first_index, uint32_t k, uint32_t d, uint32_t order, cudaStream_t s);
 cudaError_t gl_set_attrs();
 
 }  // namespace bzk

@@ -47,11 +47,12 @@ cudaError_t gl_launch_tail(uint32_t D, uint32_t order, uint32_t grid, uint32_t t
     return cudaErrorInvalidValue;
 }
 
-cudaError_t gl_launch_init(gl::State *ps, uint32_t nproofs, const uint8_t seed[32], uint64_t first_index, uint32_t k,
-                           uint32_t d, uint32_t order, cudaStream_t s) {
+cudaError_t gl_launch_init(gl::State *ps, uint32_t nproofs, const uint8_t seed[32], const uint8_t *seeds_dev,
+                           uint64_t first_index, uint32_t k, uint32_t d, uint32_t order, cudaStream_t s) {
     gl::Seed32Gl sd;
-    memcpy(sd.b, seed, 32);
-    gl::k_gl_transcript_init<<<(nproofs + 127) / 128, 128, 0, s>>>(ps, nproofs, sd, first_index, k, d, order);
+    memset(sd.b, 0, 32);
+    if (seed) memcpy(sd.b, seed, 32);
+    gl::k_gl_transcript_init<<<(nproofs + 127) / 128, 128, 0, s>>>(ps, nproofs, sd, seeds_dev, first_index, k, d, order);
     return cudaGetLastError();
 }
 

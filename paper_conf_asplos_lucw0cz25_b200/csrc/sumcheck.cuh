@@ -383,12 +383,19 @@ static __global__ void k_init_consts(fe *c) {
 
 struct Seed32 { uint8_t b[32]; };
 
-static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed32 seed, uint64_t first_index,
-                                         uint32_t k, uint32_t d, uint32_t order) {
+// seeds (device, may be null): per-proof seeds [nproofs][32] (BZK_F_SEEDS_DEVICE), else `seed` for all
+static __global__ void k_transcript_init(ProofState *ps, uint32_t nproofs, Seed32 seed, const uint8_t *seeds,
+                                         uint64_t first_index, uint32_t k, uint32_t d, uint32_t order) {
     uint32_t b = blockIdx.x * blockDim.x + threadIdx.x;
     if (b >= nproofs) return;
     uint32_t st[8];
-    transcript_init(st, seed.b, first_index + b, k, d, order);
+    if (seeds) {
+        Seed32 own;
+        for (int i = 0; i < 32; ++i) own.b[i] = seeds[(size_t)b * 32 + i];
+        transcript_init(st, own.b, first_index + b, k, d, order);
+    } else {
+        transcript_init(st, seed.b, first_index + b, k, d, order);
+    }
 #pragma unroll
     for (int i = 0; i < 8; ++i) ps[b].st[i] = st[i];
 }

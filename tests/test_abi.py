@@ -75,6 +75,10 @@ def test_module_entry_points_reject_bad_arguments_without_gpu(libbzk):
     assert libbzk.bzk_encoder_create(None, None, ctypes.byref(h)) == bzk.BZK_EINVAL
     assert libbzk.bzk_encode(None, None, None, 1, 0, 0, None) == bzk.BZK_EINVAL
     libbzk.bzk_encoder_destroy(None)   # no-op
+    c = bzk.bzk_commit(4, 0, None, None, None, None)
+    sb = bzk.bzk_batch()
+    assert libbzk.bzk_commit_prove(None, None, ctypes.byref(c), ctypes.byref(sb), None) == bzk.BZK_EINVAL
+    assert libbzk.bzk_debug_gl(0, 1, None, None, None, None) == bzk.BZK_EINVAL
 
 
 def test_abi_struct_layouts_match_header():
@@ -84,8 +88,8 @@ def test_abi_struct_layouts_match_header():
     from paper_conf_asplos_lucw0cz25_b200 import bzk
     src = """#include <stdio.h>
 #include "bzk.h"
-int main(void) { printf("%zu %zu %zu %zu\\n", sizeof(bzk_batch), sizeof(bzk_merkle_batch), sizeof(bzk_csr),
-                        sizeof(bzk_code)); return 0; }
+int main(void) { printf("%zu %zu %zu %zu %zu\\n", sizeof(bzk_batch), sizeof(bzk_merkle_batch), sizeof(bzk_csr),
+                        sizeof(bzk_code), sizeof(bzk_commit)); return 0; }
 """
     with tempfile.TemporaryDirectory() as d:
         c = os.path.join(d, "s.c")
@@ -94,7 +98,7 @@ int main(void) { printf("%zu %zu %zu %zu\\n", sizeof(bzk_batch), sizeof(bzk_merk
         subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
         sizes = [int(x) for x in subprocess.check_output([exe]).split()]
     assert sizes == [ctypes.sizeof(bzk.bzk_batch), ctypes.sizeof(bzk.bzk_merkle_batch), ctypes.sizeof(bzk.bzk_csr),
-                     ctypes.sizeof(bzk.bzk_code)]
+                     ctypes.sizeof(bzk.bzk_code), ctypes.sizeof(bzk.bzk_commit)]
 
 
 def test_product_package_does_not_touch_the_oracle():
