@@ -557,8 +557,13 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
             mp.challenges = (const fe *)io.challenges; mp.round_evals = (fe *)io.round_evals;
             mp.claims = (fe *)io.claims;
             dim3 grid(mp.ctas, (uint32_t)io.nb);
+            CUtensorMap tm;
+            memset(&tm, 0, sizeof tm);
+            const bool tma = P.order == 1 && knobs().tma != 0;   // MSB: segment-wise TMA staging
+            if (tma && !make_row_map(&tm, mp.src, io.nb * cur_stride / 4, 8))
+                return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_multi)");
             ProfScope ps_(ctx, s, 9);
-            cudaError_t e = multi_launch(P.order, m, grid, s, mp);
+            cudaError_t e = multi_launch(P.order, m, tma, grid, s, mp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_multi launch");
             cur = mp.dst; cur_stride = mp.dst_stride;
@@ -1564,6 +1569,7 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
         set_kernel_attrs<3>();
         set_kernel_attrs<4>();
         gl_set_attrs();
+        multi_set_attrs();
         k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
         ok = cudaStreamSynchronize(ctx->copy_stream) == cudaSuccess;
     }

@@ -3,19 +3,31 @@
 
 namespace bzk {
 
-template <int ORDER>
-static cudaError_t multi_launch_o(uint32_t m, dim3 grid, cudaStream_t s, const MultiParams &p) {
+template <int M>
+constexpr size_t multi_tma_smem() { return (size_t)8 * (1u << M) * 1024 + 1024; }   // 8 warps x 2^M KiB + align
+
+template <int ORDER, bool TMA>
+static cudaError_t multi_launch_o(uint32_t m, dim3 grid, cudaStream_t s, const MultiParams &p, const CUtensorMap &tm) {
     switch (m) {
-        case 1: k_multi<ORDER, 1><<<grid, 256, 0, s>>>(p); break;
-        case 2: k_multi<ORDER, 2><<<grid, 256, 0, s>>>(p); break;
-        case 3: k_multi<ORDER, 3><<<grid, 256, 0, s>>>(p); break;
+        case 1: k_multi<ORDER, 1, TMA><<<grid, 256, TMA ? multi_tma_smem<1>() : 0, s>>>(p, tm); break;
+        case 2: k_multi<ORDER, 2, TMA><<<grid, 256, TMA ? multi_tma_smem<2>() : 0, s>>>(p, tm); break;
+        case 3: k_multi<ORDER, 3, TMA><<<grid, 256, TMA ? multi_tma_smem<3>() : 0, s>>>(p, tm); break;
         default: return cudaErrorInvalidValue;
     }
     return cudaGetLastError();
 }
 
-cudaError_t multi_launch(uint32_t order, uint32_t m, dim3 grid, cudaStream_t s, const MultiParams &p) {
-    return order == 0 ? multi_launch_o<0>(m, grid, s, p) : multi_launch_o<1>(m, grid, s, p);
+cudaError_t multi_launch(uint32_t order, uint32_t m, bool tma, dim3 grid, cudaStream_t s, const MultiParams &p,
+                         const CUtensorMap &tm) {
+    if (order == 0) return multi_launch_o<0, false>(m, grid, s, p, tm);
+    return tma ? multi_launch_o<1, true>(m, grid, s, p, tm) : multi_launch_o<1, false>(m, grid, s, p, tm);
+}
+
+cudaError_t multi_set_attrs() {
+    cudaFuncSetAttribute(k_multi<1, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<1>());
+    cudaFuncSetAttribute(k_multi<1, 2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<2>());
+    return cudaFuncSetAttribute(k_multi<1, 3, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)multi_tma_smem<3>());
 }
 
 }  // namespace bzk

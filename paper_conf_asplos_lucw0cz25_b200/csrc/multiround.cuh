@@ -43,10 +43,14 @@ struct MultiParams {
     fe *claims;           // [Bw] (may be null)
 };
 
-template <int ORDER, int M>
-__global__ void __launch_bounds__(256, 2) k_multi(MultiParams P) {
+// TMA = true (MSB only): the warp's 32 columns are streamed into shared memory segment by segment --
+// segment z holds entry z of the 32 columns, the 1 KiB A[y0 + z 2^(K-M) .. + 31] -- and each segment's
+// copy for the next grid-stride block is issued as soon as every lane has consumed it (sumcheck.cuh
+// TMA helpers; 128-byte swizzle, conflict-free LDS), so one entry at a time is live in registers.
+template <int ORDER, int M, bool TMA>
+__global__ void __launch_bounds__(256, 2) k_multi(MultiParams P, const __grid_constant__ CUtensorMap tmap) {
     constexpr int Z = 1 << M;
-    __shared__ fe s_w[Z];              // w(z) R (Montgomery form)
+    __shared__ fe s_w[Z];              // w(z) 2^288 (acc17_to_fe_288 divides the row sums by 2^288)
     __shared__ fe s_r[M][2];           // r_i R, (1 - r_i) R
     __shared__ fe s_red[32 * Z];
     __shared__ int s_last;
@@ -67,7 +71,9 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P) {
             const int bit = ORDER == 1 ? (threadIdx.x >> (M - i)) & 1 : (threadIdx.x >> (i - 1)) & 1;
             w = mont_mul(w, s_r[i - 1][bit]);
         }
-        s_w[threadIdx.x] = w;
+        fe c288 = fe_const(1);                                                    // 2^256 mod p
+        for (int e = 0; e < 32; ++e) c288 = fe_add(c288, c288);                 // 2^288 mod p
+        s_w[threadIdx.x] = mont_mul(w, mont_mul(c288, fe_const(2)));             // w R * 2^288 R / R
     }
     __syncthreads();
 
@@ -75,9 +81,54 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P) {
     const fe *src = P.src + (size_t)b * P.src_stride;
     fe *dst = P.dst + (size_t)b * P.dst_stride;
     const uint64_t stride = (uint64_t)P.ctas * blockDim.x;
-    acc9 col[Z];
+    fe col[Z];                                         // column sums, lazy: < 2p
 #pragma unroll
-    for (int z = 0; z < Z; ++z) col[z] = acc9_zero();
+    for (int z = 0; z < Z; ++z) col[z] = fe_zero();
+    if constexpr (TMA) {
+        static_assert(ORDER == 1, "TMA staging of k_multi is built for the MSB (Alg. 1) layout");
+        extern __shared__ uint8_t tma_raw[];
+        __shared__ __align__(8) uint64_t bars[8 * Z];
+        uint8_t *tma_base = tma_raw + ((1024 - (smem_u32(tma_raw) & 1023)) & 1023);
+        const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+        uint8_t *seg = tma_base + (size_t)warp * Z * 1024;
+        uint64_t *wb = bars + warp * Z;
+        if (lane == 0) {
+#pragma unroll
+            for (int z = 0; z < Z; ++z) mbar_init(&wb[z]);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncwarp();
+        const uint64_t row0 = (uint64_t)b * P.src_stride / 4;     // 4 entries of 32 B per 128-byte row
+        const uint64_t y0 = (uint64_t)blockIdx.x * blockDim.x + warp * 32;
+        auto issue = [&](int z, uint64_t yb) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&wb[z], 1024);
+            tma_load_rows(seg + z * 1024, &tmap, row0 + (yb + (uint64_t)z * Ny) / 4, &wb[z]);
+        };
+        if (lane == 0 && y0 < Ny)
+#pragma unroll
+            for (int z = 0; z < Z; ++z) issue(z, y0);
+        uint32_t it = 0;
+        for (uint64_t yw = y0; yw < Ny; yw += stride, ++it) {
+            acc17 acc = acc17_zero();
+#pragma unroll
+            for (int z = 0; z < Z; ++z) {
+                mbar_wait(&wb[z], it & 1);
+                const uint32_t row = lane >> 2, c0 = 2 * (lane & 3);
+                const uint8_t *base = seg + z * 1024 + row * 128;
+                const uint4 lo = *reinterpret_cast<const uint4 *>(base + ((c0 ^ (row & 7)) << 4));
+                const uint4 hi = *reinterpret_cast<const uint4 *>(base + (((c0 + 1) ^ (row & 7)) << 4));
+                fe x;
+                x.l[0] = lo.x; x.l[1] = lo.y; x.l[2] = lo.z; x.l[3] = lo.w;
+                x.l[4] = hi.x; x.l[5] = hi.y; x.l[6] = hi.z; x.l[7] = hi.w;
+                col[z] = lz_red(lz_add(col[z], x));
+                mul_acc(acc, s_w[z], x);
+                __syncwarp();                          // every lane has used segment z
+                if (lane == 0 && yw + stride < Ny) issue(z, yw + stride);
+            }
+            st_fe(dst + yw + lane, acc17_to_fe_288(acc));
+        }
+    } else
     for (uint64_t y = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; y < Ny; y += stride) {
         fe x[Z];
 #pragma unroll
@@ -85,16 +136,16 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P) {
         acc17 acc = acc17_zero();
 #pragma unroll
         for (int z = 0; z < Z; ++z) {
-            acc9_add(col[z], x[z]);
+            col[z] = lz_red(lz_add(col[z], x[z]));    // < 2p + p, minus 2p when >= 2p
             mul_acc(acc, s_w[z], x[z]);
         }
-        st_fe(dst + y, acc17_to_fe(acc));              // canonical: A'[y] = sum_z w(z) A[y, z]
+        st_fe(dst + y, acc17_to_fe_288(acc));          // canonical: A'[y] = sum_z w(z) A[y, z]
     }
 
     // column sums of the proof: thread -> block -> per-CTA partial -> last-CTA ticket
     fe cs[Z];
 #pragma unroll
-    for (int z = 0; z < Z; ++z) cs[z] = acc9_to_fe(col[z]);
+    for (int z = 0; z < Z; ++z) cs[z] = fe_reduce_once(col[z]);
     block_reduce<Z>(cs, s_red);
     fe *part = P.partials + (size_t)b * P.ctas * Z;
     if (P.ctas > 1) {
@@ -137,6 +188,8 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P) {
 }
 
 // k_multi.cu
-cudaError_t multi_launch(uint32_t order, uint32_t m, dim3 grid, cudaStream_t s, const MultiParams &p);
+cudaError_t multi_launch(uint32_t order, uint32_t m, bool tma, dim3 grid, cudaStream_t s, const MultiParams &p,
+                         const CUtensorMap &tm);
+cudaError_t multi_set_attrs();
 
 }  // namespace bzk

@@ -135,6 +135,44 @@ __device__ __forceinline__ fe acc9_to_fe(const acc9 &a) {
     return fe_add(fe_reduce_256(a.lo), mont_mul(h, fe_const(2)));   // hi * R^2 * R^-1 = hi * R
 }
 
+// 544-bit accumulator -> S * 2^-288 mod p, canonical: NINE Montgomery word steps, so the quotient
+// W = (S + q p) / 2^288 < 2^256 + p needs one conditional subtraction and no extra product (the
+// 8-step form below leaves a 2^256 "hi" part that costs a full Montgomery product).  Callers fold
+// the extra 2^-32 into a constant (k_multi: weights w 2^288 mod p).
+__device__ __forceinline__ fe acc17_to_fe_288(const acc17 &a) {
+    const uint32_t P[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
+    uint32_t t[18];
+#pragma unroll
+    for (int i = 0; i < 17; ++i) t[i] = a.w[i];
+    t[17] = 0;
+#pragma unroll
+    for (int i = 0; i < 9; ++i) {
+        const uint32_t m = t[i] * BZK_NP0;
+        uint64_t c = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const uint64_t x = (uint64_t)m * P[j] + t[i + j] + c;
+            t[i + j] = (uint32_t)x;
+            c = x >> 32;
+        }
+#pragma unroll
+        for (int j = i + 8; j < 18; ++j) {
+            const uint64_t x = (uint64_t)t[j] + c;
+            t[j] = (uint32_t)x;
+            c = x >> 32;
+        }
+    }
+    fe w;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) w.l[i] = t[9 + i];
+    if (t[17]) {   // W >= 2^256: W - p < 2^256 (W < 2^256 + p); the borrow out of the top word cancels t[17]
+        fe r;
+        sub_p(r, w);
+        w = r;
+    }
+    return fe_reduce_256(w);
+}
+
 // 544-bit accumulator -> S * R^{-1} mod p, canonical (once per thread after the loop; plain code)
 __device__ __forceinline__ fe acc17_to_fe(const acc17 &a) {
     const uint32_t P[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
