@@ -73,7 +73,7 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P, const __grid_co
         }
         fe c288 = fe_const(1);                                                    // 2^256 mod p
         for (int e = 0; e < 32; ++e) c288 = fe_add(c288, c288);                 // 2^288 mod p
-        s_w[threadIdx.x] = mont_mul(w, mont_mul(c288, fe_const(2)));             // w R * 2^288 R / R
+        s_w[threadIdx.x] = mont_mul(w, c288);                                     // (w R) 2^288 / R = w 2^288
     }
     __syncthreads();
 

@@ -115,6 +115,35 @@ __device__ __forceinline__ void transcript_init(uint32_t state[8], const uint8_t
     sh.finish(state);
 }
 
+// state_i = SHA-256(state_{i-1} || LE256 g(0..D)) with the message laid out at compile time: the
+// 8 + 8 (D + 1) words, the 0x80 marker, zeros and the 64-bit length sit in a static word array, so
+// every block is compressed straight from registers (no streaming buffer in local memory).  This is
+// the serial part of every round (one thread per proof), so its latency is what counts.
+template <int D>
+__device__ __forceinline__ fe transcript_round_t(uint32_t state[8], const fe (&g)[D + 1]) {
+    constexpr int N = 8 + 8 * (D + 1);                  // message words
+    constexpr int NB = (N + 1 + 2 + 15) / 16;           // blocks incl. the marker and the length
+    uint32_t m[NB * 16];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) m[i] = state[i];
+#pragma unroll
+    for (int t = 0; t <= D; ++t)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) m[8 + 8 * t + i] = bswap32(g[t].l[i]);
+    m[N] = 0x80000000u;
+#pragma unroll
+    for (int i = N + 1; i < NB * 16 - 2; ++i) m[i] = 0;
+    m[NB * 16 - 2] = 0;
+    m[NB * 16 - 1] = (uint32_t)N * 32;
+    uint32_t h[8];
+    sha256_init_state(h);
+#pragma unroll
+    for (int b = 0; b < NB; ++b) sha256_compress(h, m + 16 * b);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) state[i] = h[i];
+    return fe_reduce_256(digest_to_fe_raw(state));
+}
+
 // state_i = SHA-256(state_{i-1} || LE256 g(0..d)); returns r_i canonical (standard form)
 __device__ __forceinline__ fe transcript_round(uint32_t state[8], const fe *g, int d) {
     sha256_words sh;

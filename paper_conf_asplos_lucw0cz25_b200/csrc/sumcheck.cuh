@@ -285,21 +285,6 @@ __device__ __forceinline__ fe fold_fx(const fe &a, const fe &b, const fe *K, uin
 
 // ---------------------------------------------------------------- per-round finalisation
 
-// g(r) from g(0..D) by Lagrange interpolation on the nodes 0..D (all standard form; rm = r R).
-template <int D>
-__device__ __forceinline__ fe lagrange_at(const fe (&g)[D + 1], const fe &rm, const fe *consts) {
-    fe acc = fe_zero();
-#pragma unroll 1
-    for (int j = 0; j <= D; ++j) {
-        fe term = mont_mul(g[j], consts[kConstInvW + 5 * D + j]);          // g_j / w_j
-#pragma unroll 1
-        for (int l = 0; l <= D; ++l)
-            if (l != j) term = mont_mul(term, fe_sub(rm, consts[kConstLR + l]));   // * (r - l)
-        acc = fe_add(acc, term);
-    }
-    return acc;
-}
-
 // x * c for a small non-negative integer c (finalisation only)
 __device__ __forceinline__ fe fe_mul_small(const fe &x, int c) {
     fe r = fe_zero(), y = x;
@@ -326,18 +311,26 @@ __device__ __forceinline__ fe extrapolate_top(const fe (&g)[D + 1], const fe &ci
 
 // Fix the R^{-(D-1)} scale of the round sums, rebuild g(0..D), absorb g into the transcript,
 // derive r_i, write the round's outputs and the next claim.  ONE thread per proof.
-//   MODE 0: S holds g(0..D) directly (on-chip tail)
+//   MODE 0: S holds g(0..D) directly, already in standard form (on-chip tail: its tables 1..D-1 are
+//           held in Montgomery form, so the products carry no R^{-(D-1)})
 //   MODE 1: S holds the FIRST point set, MODE 2 the DERIVE point set (see Pts / point_t)
+// The next claim g_i(r_i) (global rounds) is NOT computed here: the caller's warp does the Lagrange
+// sum with one lane per node (lagrange_warp), from g_out and the returned r R.
 template <int D, int MODE>
 __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], uint32_t round, ProofState &ps,
-                                               fe *round_evals, fe *challenges, fe *claims, const fe *consts,
-                                               fe *rmont_out, bool given) {
+                                               fe *round_evals, fe *challenges, fe *claims, fe *rmont_out,
+                                               fe *g_out, bool given) {
     constexpr int NS = MODE == 2 ? D : D + 1;
     fe g[D + 1];
-    const fe RD = fe_R_pow(D);
     fe fixd[NS];
+    if (MODE == 0) {
 #pragma unroll
-    for (int i = 0; i < NS; ++i) fixd[i] = mont_mul(S[i], RD);
+        for (int i = 0; i < NS; ++i) fixd[i] = S[i];
+    } else {
+        const fe RD = fe_R_pow(D);
+#pragma unroll
+        for (int i = 0; i < NS; ++i) fixd[i] = mont_mul(S[i], RD);
+    }
     if (MODE == 0) {
 #pragma unroll
         for (int t = 0; t <= D; ++t) g[t] = fixd[t];
@@ -359,7 +352,7 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
         uint32_t st[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) st[i] = ps.st[i];
-        r = transcript_round(st, g, D);
+        r = transcript_round_t<D>(st, g);
 #pragma unroll
         for (int i = 0; i < 8; ++i) ps.st[i] = st[i];
         st_fe(&challenges[round - 1], r);
@@ -369,10 +362,28 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
     if (round == 1 && claims) st_fe(claims, fe_add(g[0], g[1]));
     fe rm = mont_mul(r, fe_const(2));
     ps.rmont = rm;
-    // the next claim feeds g(1) = claim - g(0) of a fused global round; the on-chip tail (MODE 0)
-    // sums every point directly, so it skips the interpolation (9-16 serial products per round)
-    if (MODE != 0) ps.claim = lagrange_at<D>(g, rm, consts);
     if (rmont_out) *rmont_out = rm;
+    if (g_out)
+#pragma unroll
+        for (int t = 0; t <= D; ++t) g_out[t] = g[t];
+}
+
+// next claim g_i(r_i) = sum_j g_j / w_j * prod_{l != j} (r - l)  (Lagrange on the nodes 0..D): lane j
+// of the calling warp computes term j (D + 1 serial products instead of (D + 1)^2), then a shuffle sum.
+// Every lane of the warp calls it; g and rm in shared memory (written by lane 0 before a __syncwarp).
+template <int D>
+__device__ __forceinline__ fe lagrange_warp(const fe *g, const fe &rm, const fe *consts) {
+    const int lane = threadIdx.x & 31;
+    fe term = fe_zero();
+    if (lane <= D) {
+        term = mont_mul(g[lane], consts[kConstInvW + 5 * D + lane]);          // g_j / w_j
+#pragma unroll 1
+        for (int l = 0; l <= D; ++l)
+            if (l != lane) term = mont_mul(term, fe_sub(rm, consts[kConstLR + l]));   // * (r - l)
+    }
+#pragma unroll
+    for (int off = 4; off > 0; off >>= 1) term = fe_add(term, shfl_down_fe(term, off));   // lanes 0..7 >= D + 1
+    return term;
 }
 
 // ---------------------------------------------------------------- constants, transcript init
@@ -742,9 +753,16 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
     fe *evals = P.round_evals + (size_t)b * P.k * (D + 1);
     fe *chals = P.challenges + (size_t)b * P.k;
     fe *claim = P.claims ? P.claims + b : nullptr;
+    __shared__ fe s_g[D + 1];
+    __shared__ fe s_rm;
     if (P.ctas == 1) {
-        if (threadIdx.x == 0)
-            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr, P.given);
+        if (threadIdx.x < 32) {
+            if (threadIdx.x == 0)
+                finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
+            __syncwarp();
+            const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
+            if (threadIdx.x == 0) P.ps[b].claim = c;
+        }
         return;
     }
     // Thread-block cluster (launched with cluster dims (cs, 1, 1), cs <= 8, all CTAs of one proof):
@@ -788,9 +806,14 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
 #pragma unroll
         for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], ld_fe_cg(&part[(size_t)c * NV + t]));
     block_reduce<NV>(acc, s_red);
-    if (threadIdx.x == 0) {
-        P.tickets[b] = 0;
-        finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, P.consts, nullptr, P.given);
+    if (threadIdx.x < 32) {
+        if (threadIdx.x == 0) {
+            P.tickets[b] = 0;
+            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
+        }
+        __syncwarp();
+        const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
+        if (threadIdx.x == 0) P.ps[b].claim = c;
     }
 }
 
@@ -837,10 +860,17 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
         return;
     }
 
-    // stage the round-i0 table (2h0 entries per m) into A
+    // stage the round-i0 table (2h0 entries per m) into A.  Tables 1..D-1 are held in Montgomery
+    // form (x R): a product v_0 v_1 ... v_{D-1} through D-1 Montgomery products then comes out in
+    // standard form (no per-round R^{-(D-1)} fix on the serial path); folds are linear, so the form is
+    // kept; the final evaluations are converted back.
+    const fe R2 = fe_const(2);
     if (P.i0 == 1 || P.folded) {
         const fe *src = P.src + (size_t)b * (P.src_stride ? P.src_stride : (size_t)D * (2 * h0));
-        for (uint32_t x = threadIdx.x; x < (uint32_t)D * 2 * h0; x += blockDim.x) A[x] = ld_fe(src + x);
+        for (uint32_t x = threadIdx.x; x < (uint32_t)D * 2 * h0; x += blockDim.x) {
+            const fe v = ld_fe(src + x);
+            A[x] = x < 2 * h0 ? v : mont_mul(v, R2);
+        }
     } else {
         const fe *src = P.src + (size_t)b * D * (4 * h0);
         const fe rm = P.ps[b].rmont;
@@ -851,7 +881,8 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
             if (ORDER == 0) { lo = ld_fe(T + 2 * y); hi = ld_fe(T + 2 * y + 1); }
             else            { lo = ld_fe(T + y);     hi = ld_fe(T + y + 2 * h0); }
             // entries written by a fused round are lazily reduced (< 2p): canonicalise first
-            A[x] = fold1(fe_reduce_once(lo), fe_reduce_once(hi), rm);
+            const fe v = fold1(fe_reduce_once(lo), fe_reduce_once(hi), rm);
+            A[x] = m == 0 ? v : mont_mul(v, R2);
         }
     }
     __syncthreads();
@@ -875,7 +906,7 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
         block_reduce<D + 1>(acc, s_red);
         if (threadIdx.x == 0) {
             fe rm;
-            finalize_round<D, 0>(acc, i, P.ps[b], evals, chals, claim, P.consts, &rm, P.given);
+            finalize_round<D, 0>(acc, i, P.ps[b], evals, chals, claim, &rm, nullptr, P.given);
             s_r = rm;
         }
         __syncthreads();
@@ -893,8 +924,13 @@ __global__ void __launch_bounds__(256) k_tail(TailParams P) {
         fe *tmp = cur; cur = oth; oth = tmp;
         h >>= 1;
     }
-    // after round k the tables have one entry: final_m = f_m(rho)
-    if (threadIdx.x < D) st_fe(&P.final_evals[(size_t)b * D + threadIdx.x], cur[threadIdx.x]);
+    // after round k the tables have one entry: final_m = f_m(rho) (tables 1..D-1 back from Montgomery form)
+    if (threadIdx.x < D) {
+        fe one = fe_zero();
+        one.l[0] = 1;
+        const fe v = cur[threadIdx.x];
+        st_fe(&P.final_evals[(size_t)b * D + threadIdx.x], threadIdx.x == 0 ? v : mont_mul(v, one));
+    }
 }
 
 // launchers, explicitly instantiated per degree in k_d<D>.cu (parallel compilation)
