@@ -22,6 +22,7 @@
 #include "gen.cuh"
 #include "merkle.cuh"
 #include "multiround.cuh"
+#include "small.cuh"
 #include "encoder.cuh"
 #include "sha256.cuh"
 #include "sumcheck.cuh"
@@ -171,7 +172,11 @@ struct Knobs {
     // table, multiround.cuh) instead of one k_round launch per round
     uint32_t multi = 1;
     uint32_t multi_m = 3;      // BZK_MULTI_M: rounds per k_multi pass (1..3)
+    // BZK_SMALL=0/1: proofs whose tables fit a cluster's shared memory run in k_small (one launch,
+    // all rounds, cluster/DSMEM reduction; small.cuh)
+    uint32_t small = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_M")) multi_m = std::max(1, std::min(3, atoi(e)));
         if (const char *e = getenv("BZK_MULTI")) multi = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_TMA")) tma = atoi(e) ? 1 : 0;
@@ -518,8 +523,51 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
     return BZK_OK;
 }
 
+// cluster size (log2) of k_small for this shape, or -1: the smallest cluster whose CTAs hold their share
+// of the tables in <= kSmallSmem bytes, widened (up to 8 CTAs) while the batch leaves SMs idle
+constexpr size_t kSmallSmem = 200 * 1024;
+int small_cs_log(uint32_t D, uint32_t k, uint64_t nb) {
+    if (k == 0 || !knobs().small) return -1;
+    int c = -1;
+    for (int cl = 0; cl <= 3 && cl <= (int)k; ++cl)
+        if ((size_t)D * (((size_t)1 << k) >> cl) * 3 / 2 * sizeof(fe) <= kSmallSmem) { c = cl; break; }
+    if (c < 0) return -1;
+    while (c < 3 && c < (int)k && nb * (2ull << c) <= (uint64_t)2 * kSMs) ++c;   // latency: spread small batches
+    return c;
+}
+
+bzk_status run_wave_small(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s, int cs_log) {
+    SmallParams sp;
+    memset(&sp, 0, sizeof sp);
+    sp.src = (const fe *)io.tables; sp.k = P.k; sp.cs_log = (uint32_t)cs_log; sp.order = P.order; sp.given = P.given;
+    sp.first_index = io.first_index; sp.seed = io.seed; sp.seeds = io.seeds;
+    sp.ps = (ProofState *)((char *)ctx->ws + P.off_ps);
+    sp.round_evals = (fe *)io.round_evals; sp.challenges = (fe *)io.challenges; sp.final_evals = (fe *)io.final_evals;
+    sp.claims = (fe *)io.claims;
+    const uint32_t cs = 1u << cs_log;
+    const size_t smem = (size_t)P.D * ((P.N >> cs_log)) * 3 / 2 * sizeof(fe);
+    dim3 grid(cs, (uint32_t)io.nb);
+    cudaError_t e = cudaSuccess;
+    {
+        ProfScope ps_(ctx, s, 10);
+        switch (P.D) {
+            case 1: e = launch_small<1>(P.order, grid, cs, smem, s, sp); break;
+            case 2: e = launch_small<2>(P.order, grid, cs, smem, s, sp); break;
+            case 3: e = launch_small<3>(P.order, grid, cs, smem, s, sp); break;
+            case 4: e = launch_small<4>(P.order, grid, cs, smem, s, sp); break;
+        }
+    }
+    ++ctx->launches;
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "k_small launch");
+    return BZK_OK;
+}
+
 bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
     NvtxRange nv_("bzk wave");
+    {
+        const int cs_log = small_cs_log(P.D, P.k, io.nb);
+        if (cs_log >= 0) return run_wave_small(ctx, P, io, s, cs_log);
+    }
     char *ws = (char *)ctx->ws;
     ProofState *ps = (ProofState *)(ws + P.off_ps);
     uint32_t *tick = (uint32_t *)(ws + P.off_tick);

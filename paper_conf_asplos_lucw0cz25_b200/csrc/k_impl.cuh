@@ -1,5 +1,6 @@
 // k_impl.cuh -- per-degree kernel instantiation; included by k_d1.cu .. k_d4.cu with BZK_D set.
 #include "sumcheck.cuh"
+#include "small.cuh"
 
 namespace bzk {
 
@@ -54,8 +55,28 @@ cudaError_t set_kernel_attrs<BZK_D>() {
     set_round_attrs<0, false>();
     set_round_attrs<1, true>();
     set_round_attrs<1, false>();
+    cudaFuncSetAttribute(k_small<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(k_small<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     cudaFuncSetAttribute(k_tail<BZK_D, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     return cudaFuncSetAttribute(k_tail<BZK_D, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+}
+
+template <>
+cudaError_t launch_small<BZK_D>(uint32_t order, dim3 grid, uint32_t cs, size_t smem, cudaStream_t s,
+                                const SmallParams &p) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(256, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = cs;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return order == 0 ? cudaLaunchKernelEx(&cfg, k_small<BZK_D, 0>, p) : cudaLaunchKernelEx(&cfg, k_small<BZK_D, 1>, p);
 }
 
 template <>

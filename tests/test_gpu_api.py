@@ -199,3 +199,40 @@ def test_cluster_dsmem_reduction(cluster):
     r = subprocess.run([sys.executable, "-c", CLUSTER_SCRIPT.format(root=ROOT)], env=env, capture_output=True,
                        text=True, timeout=600)
     assert r.returncode == 0 and "cluster ok" in r.stdout, r.stdout + r.stderr
+
+
+PERROUND_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import oracle
+from paper_conf_asplos_lucw0cz25_b200 import bzk, inputs
+oracle.build()
+p = bzk.Prover(0)
+n = 0
+for d in (1, 2, 3, 4):
+    for k in (1, 2, 5, 9, 10, 11, 13):
+        for order in (0, 1):
+            B = 3
+            t = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+            bzk.bzk_generate(t, B, d, k, 50 + k, "adversarial")
+            out = p.prove(t, k, d, order, first_index=50 + k, flags=bzk.BZK_F_PRESERVE_INPUT)
+            torch.cuda.synchronize()
+            host = t.cpu().numpy().view(np.uint64)
+            for b in range(B):
+                ref = oracle.prove(host[b], k, d, order, inputs.DEFAULT_SEED, 50 + k + b)
+                for key in ref:
+                    got = out[key][b].cpu().numpy().view(np.uint64).reshape(ref[key].shape)
+                    assert np.array_equal(got, ref[key]), (key, d, k, order, b)
+                n += 1
+p.close()
+print("per-round ok", n)
+"""
+
+
+def test_per_round_path_at_small_k():
+    """With BZK_SMALL=0 the shapes k_small would take run through the per-round kernels + on-chip
+    tail (round 1, fused rounds, tail-only and first-tail-round-2 cases) -- both paths stay tested."""
+    env = dict(os.environ, BZK_SMALL="0")
+    r = subprocess.run([sys.executable, "-c", PERROUND_SCRIPT.format(root=ROOT)], env=env, capture_output=True,
+                       text=True, timeout=900)
+    assert r.returncode == 0 and "per-round ok" in r.stdout, r.stdout + r.stderr
