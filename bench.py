@@ -689,6 +689,10 @@ def imad_slots(d: int, k: int, kind: str) -> int:
         return sum((2 * d * SLOT_FIXMUL + d * point) * (1 << (k - i)) for i in range(2, i0))
     if kind == "multi":
         return sum(SLOT_MULACC * (1 << K) for K, _ in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3"))))
+    if kind == "small":
+        # k_small: every round sums all d+1 points with (d-1) canonical Montgomery products each and
+        # folds d entries per pair with one Montgomery product
+        return sum(((d + 1) * (d - 1) + d) * SLOT_MONT * (1 << (k - i)) for i in range(1, k + 1))
     raise ValueError(kind)
 
 
@@ -871,7 +875,7 @@ def run_sumcheck(args, rank, world, local):
 
     # ---------------- roofline of the dominant kernel
     hbm_peak, sm_max_mhz, peak_src = peaks()
-    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused", "multi_round": "multi"}
+    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused", "multi_round": "multi", "small_cluster": "small"}
     dom = max(kinds, key=lambda n: prof[n][0])
     dom_ms, dom_cnt = prof[dom]
     launches_per_step = max(1, dom_cnt / args.steps)
@@ -881,6 +885,9 @@ def run_sumcheck(args, rank, world, local):
     if kinds[dom] == "multi":
         bytes_per_launch = multi_bytes(k) * count / launches_per_step
         mulmods_per_launch = sum((1 << K) for K, _ in multi_passes(k)) * count / launches_per_step
+    elif kinds[dom] == "small":
+        bytes_per_launch = d * (1 << k) * esz * count / launches_per_step
+        mulmods_per_launch = alg_mulmods(d, k, "total") * count / launches_per_step
     else:
         bytes_per_launch = alg_bytes_kind(d, k, kinds[dom], esz) * count / launches_per_step
         mulmods_per_launch = alg_mulmods(d, k, kinds[dom]) * count / launches_per_step

@@ -524,14 +524,17 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
 }
 
 // cluster size (log2) of k_small for this shape, or -1: the smallest cluster whose CTAs hold their share
-// of the tables in <= kSmallSmem bytes, widened (up to 8 CTAs) while the batch leaves SMs idle
+// of the tables in <= kSmallSmem bytes, widened (up to 8 CTAs) while the batch leaves SMs idle.  Only
+// for batches that do not fill the GPU (fewer clusters than SMs): k_small is the LATENCY path -- a
+// cluster idles while its leader hashes, which lockstep per-round kernels amortise over many proofs
+// (B200 A/B, profiles/r02/r02h_*: c1 0.207 -> see DESIGN sec. 8; c4's jobs 2.2x slower in k_small)
 constexpr size_t kSmallSmem = 200 * 1024;
 int small_cs_log(uint32_t D, uint32_t k, uint64_t nb) {
     if (k == 0 || !knobs().small) return -1;
     int c = -1;
     for (int cl = 0; cl <= 3 && cl <= (int)k; ++cl)
         if ((size_t)D * (((size_t)1 << k) >> cl) * 3 / 2 * sizeof(fe) <= kSmallSmem) { c = cl; break; }
-    if (c < 0) return -1;
+    if (c < 0 || nb * (1ull << c) > kSMs) return -1;
     while (c < 3 && c < (int)k && nb * (2ull << c) <= (uint64_t)2 * kSMs) ++c;   // latency: spread small batches
     return c;
 }
