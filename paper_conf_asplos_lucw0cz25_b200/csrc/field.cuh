@@ -384,6 +384,10 @@ __device__ __forceinline__ fe mont_mul_lz(const fe &a, const fe &b) {
 // Montgomery product a*b*R^{-1} mod p; a, b canonical -> canonical.
 __device__ __forceinline__ fe mont_mul(const fe &a, const fe &b) { return fe_reduce_once(mont_mul_lz(a, b)); }
 
+// The same product, NOT inlined: for the one-thread-per-proof serial work of a round (finalisation,
+// Lagrange), where one shared copy of the code stays in the instruction cache across call sites.
+static __device__ __noinline__ fe mont_mul_serial(const fe a, const fe b) { return mont_mul(a, b); }
+
 // (x*y + u*v) * R^{-1} (+ q p) with ONE Montgomery reduction (lazy sum of two products).
 // Each row adds x*y_i and u*v_i before the reduction row.  Result < (x*y + u*v)/R + p: with
 // x, y, u, v < 2p it is < 2.52p (< 2^256 since 4p < 2^256); with x, u < p, y, v < 2^256 it is < 3p.

@@ -59,6 +59,40 @@ __device__ __forceinline__ void sha256_compress(uint32_t h[8], const uint32_t wi
     h[0] += a; h[1] += b; h[2] += c; h[3] += d; h[4] += e; h[5] += f; h[6] += g; h[7] += hh;
 }
 
+// The same compression for the SERIAL per-round transcript (one thread per proof, on the critical path
+// of every round): 16 unrolled rounds inside a 4-iteration loop, not inlined, so the per-round hash is
+// ~600 instructions of hot code instead of three inlined copies of a fully unrolled compression
+// (which thrashed the instruction cache: k_small was 22K SASS instructions, ncu no_instruction stalls).
+static __device__ __noinline__ void sha256_compress_serial(uint32_t h[8], const uint32_t win[16]) {
+    uint32_t w[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) w[i] = win[i];
+    uint32_t a = h[0], b = h[1], c = h[2], d = h[3], e = h[4], f = h[5], g = h[6], hh = h[7];
+#pragma unroll 1
+    for (int T = 0; T < 64; T += 16) {
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+            uint32_t wt;
+            if (T == 0) {
+                wt = w[j];
+            } else {
+                const uint32_t w15 = w[(j + 1) & 15], w2 = w[(j + 14) & 15];
+                const uint32_t s0 = rotr32(w15, 7) ^ rotr32(w15, 18) ^ (w15 >> 3);
+                const uint32_t s1 = rotr32(w2, 17) ^ rotr32(w2, 19) ^ (w2 >> 10);
+                wt = w[j] + s0 + w[(j + 9) & 15] + s1;
+                w[j] = wt;
+            }
+            const uint32_t S1 = rotr32(e, 6) ^ rotr32(e, 11) ^ rotr32(e, 25);
+            const uint32_t ch = (e & f) ^ (~e & g);
+            const uint32_t T1 = hh + S1 + ch + c_K256[T + j] + wt;
+            const uint32_t S0 = rotr32(a, 2) ^ rotr32(a, 13) ^ rotr32(a, 22);
+            const uint32_t maj = (a & b) ^ (a & c) ^ (b & c);
+            hh = g; g = f; f = e; e = d + T1; d = c; c = b; b = a; a = T1 + S0 + maj;
+        }
+    }
+    h[0] += a; h[1] += b; h[2] += c; h[3] += d; h[4] += e; h[5] += f; h[6] += g; h[7] += hh;
+}
+
 // Streaming absorber over 32-bit big-endian words (messages here are multiples of 4 bytes).
 struct sha256_words {
     uint32_t h[8];
@@ -137,8 +171,8 @@ __device__ __forceinline__ fe transcript_round_t(uint32_t state[8], const fe (&g
     m[NB * 16 - 1] = (uint32_t)N * 32;
     uint32_t h[8];
     sha256_init_state(h);
-#pragma unroll
-    for (int b = 0; b < NB; ++b) sha256_compress(h, m + 16 * b);
+#pragma unroll 1
+    for (int b = 0; b < NB; ++b) sha256_compress_serial(h, m + 16 * b);
 #pragma unroll
     for (int i = 0; i < 8; ++i) state[i] = h[i];
     return fe_reduce_256(digest_to_fe_raw(state));

@@ -329,7 +329,7 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
     } else {
         const fe RD = fe_R_pow(D);
 #pragma unroll
-        for (int i = 0; i < NS; ++i) fixd[i] = mont_mul(S[i], RD);
+        for (int i = 0; i < NS; ++i) fixd[i] = mont_mul_serial(S[i], RD);
     }
     if (MODE == 0) {
 #pragma unroll
@@ -360,7 +360,7 @@ __device__ __forceinline__ void finalize_round(fe (&S)[MODE == 2 ? D : D + 1], u
 #pragma unroll
     for (int t = 0; t <= D; ++t) st_fe(&round_evals[(size_t)(round - 1) * (D + 1) + t], g[t]);
     if (round == 1 && claims) st_fe(claims, fe_add(g[0], g[1]));
-    fe rm = mont_mul(r, fe_const(2));
+    fe rm = mont_mul_serial(r, fe_const(2));
     ps.rmont = rm;
     if (rmont_out) *rmont_out = rm;
     if (g_out)
@@ -376,10 +376,10 @@ __device__ __forceinline__ fe lagrange_warp(const fe *g, const fe &rm, const fe 
     const int lane = threadIdx.x & 31;
     fe term = fe_zero();
     if (lane <= D) {
-        term = mont_mul(g[lane], consts[kConstInvW + 5 * D + lane]);          // g_j / w_j
+        term = mont_mul_serial(g[lane], consts[kConstInvW + 5 * D + lane]);          // g_j / w_j
 #pragma unroll 1
         for (int l = 0; l <= D; ++l)
-            if (l != lane) term = mont_mul(term, fe_sub(rm, consts[kConstLR + l]));   // * (r - l)
+            if (l != lane) term = mont_mul_serial(term, fe_sub(rm, consts[kConstLR + l]));   // * (r - l)
     }
 #pragma unroll
     for (int off = 4; off > 0; off >>= 1) term = fe_add(term, shfl_down_fe(term, off));   // lanes 0..7 >= D + 1
