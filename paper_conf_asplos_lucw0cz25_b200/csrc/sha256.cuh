@@ -60,15 +60,15 @@ __device__ __forceinline__ void sha256_compress(uint32_t h[8], const uint32_t wi
 }
 
 // The same compression for the SERIAL per-round transcript (one thread per proof, on the critical path
-// of every round): 16 unrolled rounds inside a 4-iteration loop, not inlined, so the per-round hash is
-// ~600 instructions of hot code instead of three inlined copies of a fully unrolled compression
-// (which thrashed the instruction cache: k_small was 22K SASS instructions, ncu no_instruction stalls).
+// of every round): one NON-inlined, fully unrolled copy (K as immediates, no loop overhead) shared by
+// every call site, instead of three inlined copies per transcript (which thrashed the instruction
+// cache: k_small was 22K SASS instructions, ncu no_instruction stalls).
 static __device__ __noinline__ void sha256_compress_serial(uint32_t h[8], const uint32_t win[16]) {
     uint32_t w[16];
 #pragma unroll
     for (int i = 0; i < 16; ++i) w[i] = win[i];
     uint32_t a = h[0], b = h[1], c = h[2], d = h[3], e = h[4], f = h[5], g = h[6], hh = h[7];
-#pragma unroll 1
+#pragma unroll
     for (int T = 0; T < 64; T += 16) {
 #pragma unroll
         for (int j = 0; j < 16; ++j) {

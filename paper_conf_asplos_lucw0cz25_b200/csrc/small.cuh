@@ -9,7 +9,7 @@
 // Folding keeps both layouts CTA-local (LSB: 2j, 2j+1 -> j stays in the slice; MSB: h is a multiple
 // of CS, so j and j + h share the residue), so a round is: local evaluation (all points t = 0..d) ->
 // block reduction -> partial in shared memory -> cluster barrier -> the leader CTA sums the CS
-// partials over DSMEM, hashes the transcript (SHA-256) and publishes r_i R in its shared
+// per-warp partials over DSMEM, hashes the transcript (SHA-256) and publishes r_i R in its shared
 // memory -> cluster barrier -> every CTA reads r_i over DSMEM and folds locally (P:111 line 5).  The
 // last c rounds run in the leader on the CS remaining entries per table it gathers over DSMEM.
 // Tables 1..d-1 are held in Montgomery form (products come out in standard form, no per-round scale
@@ -43,8 +43,7 @@ __global__ void __launch_bounds__(256) k_small(SmallParams P) {
     namespace cg = cooperative_groups;
     cg::cluster_group cl = cg::this_cluster();
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ fe s_red[32 * (D + 1)];
-    __shared__ fe s_part[D + 1];          // this CTA's round partial (the leader reads it over DSMEM)
+    __shared__ fe s_wpart[8][D + 1];      // this CTA's per-warp round partials (the leader reads them)
     __shared__ fe s_rm;                   // leader: r_i R for every CTA of the cluster
     __shared__ fe s_g[2][D][8];           // leader: the last c rounds on the gathered entries
     const uint32_t CS = 1u << P.cs_log, q = cl.block_rank();
@@ -81,46 +80,81 @@ __global__ void __launch_bounds__(256) k_small(SmallParams P) {
     }
     __syncthreads();
 
-    uint32_t round = 1;
-    for (; nl >= 2; ++round) {
-        const uint32_t h = nl / 2;
-        fe acc[D + 1];
-#pragma unroll
-        for (int t = 0; t <= D; ++t) acc[t] = fe_zero();
+    // round 1's evaluation on the loaded table; afterwards every pass folds with r_i AND evaluates
+    // round i + 1 on the folded entries (4 reads, 2 writes per next-round pair, as the global fused
+    // kernel), so a round is one pass over shared memory
+    auto eval_round = [&](fe (&acc)[D + 1], uint32_t n) {
+        const uint32_t h = n / 2;
         for (uint32_t j = threadIdx.x; j < h; j += blockDim.x) {
             fe a[D], bb[D];
 #pragma unroll
             for (int m = 0; m < D; ++m) {
-                const fe *T = cur + (size_t)m * nl;
+                const fe *T = cur + (size_t)m * n;
                 if (ORDER == 0) { a[m] = T[2 * j]; bb[m] = T[2 * j + 1]; }
                 else            { a[m] = T[j];     bb[m] = T[j + h]; }
             }
             eval_pair<D>(a, bb, acc);
         }
-        block_reduce<D + 1>(acc, s_red);
-        if (threadIdx.x == 0)
+    };
+    fe acc[D + 1];
 #pragma unroll
-            for (int t = 0; t <= D; ++t) s_part[t] = acc[t];
+    for (int t = 0; t <= D; ++t) acc[t] = fe_zero();
+    if (nl >= 2) eval_round(acc, nl);
+    uint32_t round = 1;
+    for (; nl >= 2; ++round) {
+        // warp sums -> shared memory; after the cluster barrier the leader warp sums the 8 CS warp
+        // partials of the whole cluster (one remote load per lane, shuffle tree)
+        warp_reduce<D + 1>(acc);
+        if ((threadIdx.x & 31) == 0)
+#pragma unroll
+            for (int t = 0; t <= D; ++t) s_wpart[threadIdx.x >> 5][t] = acc[t];
         cl.sync();                                    // partials visible cluster-wide
-        if (q == 0 && threadIdx.x == 0) {
-            for (uint32_t r = 1; r < CS; ++r) {
-                const fe *rp = cl.map_shared_rank(s_part, r);
+        if (q == 0 && threadIdx.x < 32) {
+            const uint32_t lane = threadIdx.x;
+#pragma unroll
+            for (int t = 0; t <= D; ++t) acc[t] = fe_zero();
+            for (uint32_t s2 = lane; s2 < CS * 8; s2 += 32) {
+                const fe *rp = cl.map_shared_rank(&s_wpart[s2 & 7][0], s2 >> 3);
 #pragma unroll
                 for (int t = 0; t <= D; ++t) acc[t] = fe_add(acc[t], rp[t]);
             }
+            warp_reduce<D + 1>(acc);
+        }
+        if (q == 0 && threadIdx.x == 0) {
             fe rm;
             finalize_round<D, 0>(acc, round, ps, evals, chals, claim, &rm, nullptr, P.given);
             s_rm = rm;
         }
         cl.sync();                                    // r_i published; partials consumed
         const fe rm = *cl.map_shared_rank(&s_rm, 0);
-        for (uint32_t x = threadIdx.x; x < (uint32_t)D * h; x += blockDim.x) {
-            const uint32_t m = x / h, j = x % h;
-            const fe *T = cur + (size_t)m * nl;
-            fe lo, hi;
-            if (ORDER == 0) { lo = T[2 * j]; hi = T[2 * j + 1]; }
-            else            { lo = T[j];     hi = T[j + h]; }
-            oth[(size_t)m * h + j] = fold1(lo, hi, rm);
+#pragma unroll
+        for (int t = 0; t <= D; ++t) acc[t] = fe_zero();
+        const uint32_t h = nl / 2;
+        if (nl >= 4) {
+            const uint32_t h2 = nl / 4;               // pairs of round i + 1
+            for (uint32_t j = threadIdx.x; j < h2; j += blockDim.x) {
+                fe a[D], bb[D];
+#pragma unroll
+                for (int m = 0; m < D; ++m) {
+                    const fe *T = cur + (size_t)m * nl;
+                    fe *U = oth + (size_t)m * h;
+                    if (ORDER == 0) {
+                        a[m] = fold1(T[4 * j], T[4 * j + 1], rm);
+                        bb[m] = fold1(T[4 * j + 2], T[4 * j + 3], rm);
+                        U[2 * j] = a[m];
+                        U[2 * j + 1] = bb[m];
+                    } else {
+                        a[m] = fold1(T[j], T[j + 2 * h2], rm);
+                        bb[m] = fold1(T[j + h2], T[j + 3 * h2], rm);
+                        U[j] = a[m];
+                        U[j + h2] = bb[m];
+                    }
+                }
+                eval_pair<D>(a, bb, acc);
+            }
+        } else if (threadIdx.x < D) {                 // nl == 2: the last local fold
+            const fe *T = cur + (size_t)threadIdx.x * 2;
+            oth[threadIdx.x] = fold1(T[0], T[1], rm);
         }
         __syncthreads();
         fe *tmp = cur; cur = oth; oth = tmp;

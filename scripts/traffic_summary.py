@@ -5,13 +5,18 @@ import json
 import sys
 from collections import defaultdict
 
-BATCH = {"c2": 1024, "c3": 256, "g2": 1024, "m0": 1024, "enc20": 256}   # bench.py default batches
+BATCH = {"c2": 1024, "c3": 256, "g2": 1024, "m0": 1024, "m0lit": 1024, "enc20": 256}   # bench.py default batches
 
 
 def kind_of(name):
     if "k_spmv" in name:
         return "encoder_spmv"
-    first = name.split("(")[0].rstrip(">").split(",")[-1].strip()   # FIRST template flag
+    if "k_multi" in name:
+        return "multi_round"
+    if "k_small" in name:
+        return "small_cluster"
+    args = name.split("<", 1)[1].split(">")[0].split(",")      # k_round<D, ORDER, FIRST, TMA>, k_gl_round<D, ORDER, FIRST>
+    first = args[2].strip()
     return "round1_eval" if first in ("1", "true") else "fused_fold_eval"
 
 
