@@ -86,6 +86,10 @@ struct bzk_ctx {
     // streams never overlap on the shared workspace (ps, tickets, partials, ping-pong buffers)
     cudaEvent_t ev_done = nullptr;
     bool ev_done_recorded = false;
+    // bzk_commit_prove's module pipeline: Merkle and sum-check side streams, Merkle stage scratch
+    cudaStream_t chain_mk = nullptr, chain_sc = nullptr;
+    void *chain_ws = nullptr;
+    size_t chain_ws_size = 0;
 };
 
 namespace {
@@ -175,7 +179,9 @@ struct Knobs {
     // BZK_SMALL=0/1: proofs whose tables fit a cluster's shared memory run in k_small (one launch,
     // all rounds, cluster/DSMEM reduction; small.cuh)
     uint32_t small = 1;
+    uint32_t chain_chunks = 4;   // BZK_CHAIN_CHUNKS: proof chunks of bzk_commit_prove's module pipeline
     Knobs() {
+        if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_M")) multi_m = std::max(1, std::min(3, atoi(e)));
         if (const char *e = getenv("BZK_MULTI")) multi = atoi(e) ? 1 : 0;
@@ -874,6 +880,50 @@ std::vector<MkStage> merkle_stages(uint32_t n) {
     return v;
 }
 
+// The stage chain of one wave of nb trees (device buffers): blocks [nb] x blk_stride bytes, node arrays
+// (may be null) [nb] x nodes_stride, roots [nb][32]; scr[0..1]: inter-stage digests when nodes is null
+// (nb x scratch_pt bytes each).
+bzk_status merkle_chain(bzk_ctx *ctx, uint32_t hash, uint32_t n, const std::vector<MkStage> &stages,
+                        const uint8_t *blocks, uint64_t blk_stride, uint8_t *nodes, uint64_t nodes_bytes,
+                        uint8_t *roots, uint8_t *const scr[2], size_t scratch_pt, uint64_t nb, cudaStream_t s) {
+    const bool dev_nodes = nodes != nullptr;
+    const uint8_t *in = blocks;
+    uint64_t in_stride = blk_stride;
+    for (size_t si = 0; si < stages.size(); ++si) {
+        const MkStage &g = stages[si];
+        const bool last = si + 1 == stages.size();
+        mk::StageParams p;
+        p.in = in; p.in_stride = in_stride;
+        p.nodes = nodes; p.nodes_stride = nodes_bytes;
+        p.n = n; p.lvl0 = g.lvl0; p.lg_tpt = g.lg_tpt;
+        p.threads = nb << g.lg_tpt;
+        const uint32_t top = g.lvl0 + g.lt;      // level of the thread roots
+        if (last) { p.out = roots; p.out_stride = 32; }
+        else if (dev_nodes) { p.out = nullptr; p.out_stride = 0; }
+        else { p.out = scr[si & 1]; p.out_stride = (uint64_t)32 << g.lg_tpt; }
+        const uint32_t tpb = 256;
+        const uint64_t grid = (p.threads + tpb - 1) / tpb;
+        if (grid > 0x7fffffffull) return fail(ctx, BZK_EINVAL, "too many CTAs in one stage launch");
+        {
+            ProfScope ps_(ctx, s, 6);
+            cudaError_t e = merkle_launch_stage(hash, g.lt, (uint32_t)grid, tpb, s, p);
+            ++ctx->launches;
+            if (e != cudaSuccess) return cuda_fail(ctx, e, "k_merkle_stage");
+        }
+        if (!last) {
+            if (dev_nodes) {
+                in = nodes + (((2ull << n) - (2ull << (n - top))) * 32);
+                in_stride = nodes_bytes;
+            } else {
+                in = p.out;
+                in_stride = p.out_stride;
+            }
+        }
+    }
+    (void)scratch_pt;
+    return BZK_OK;
+}
+
 bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) {
     NvtxRange nv_("bzk_merkle");
     if (!m) return fail(ctx, BZK_EINVAL, "batch is NULL");
@@ -964,39 +1014,9 @@ bzk_status merkle_impl(bzk_ctx *ctx, const bzk_merkle_batch *m, cudaStream_t s) 
             }
         }
         uint8_t *scr[2] = {(uint8_t *)(ws + off_scr), (uint8_t *)(ws + off_scr) + bw * scratch_pt};
-        const uint8_t *in = blocks;
-        uint64_t in_stride = blk_bytes;
-        for (size_t si = 0; si < stages.size(); ++si) {
-            const MkStage &g = stages[si];
-            const bool last = si + 1 == stages.size();
-            mk::StageParams p;
-            p.in = in; p.in_stride = in_stride;
-            p.nodes = nodes; p.nodes_stride = nodes_bytes;
-            p.n = n; p.lvl0 = g.lvl0; p.lg_tpt = g.lg_tpt;
-            p.threads = nb << g.lg_tpt;
-            const uint32_t top = g.lvl0 + g.lt;      // level of the thread roots
-            if (last) { p.out = roots_all + b0 * 32; p.out_stride = 32; }
-            else if (dev_nodes) { p.out = nullptr; p.out_stride = 0; }
-            else { p.out = scr[si & 1]; p.out_stride = (uint64_t)32 << g.lg_tpt; }
-            const uint32_t tpb = 256;
-            const uint64_t grid = (p.threads + tpb - 1) / tpb;
-            if (grid > 0x7fffffffull) return fail(ctx, BZK_EINVAL, "too many CTAs in one stage launch");
-            {
-                ProfScope ps_(ctx, s, 6);
-                cudaError_t e = merkle_launch_stage(m->hash, g.lt, (uint32_t)grid, tpb, s, p);
-                ++ctx->launches;
-                if (e != cudaSuccess) return cuda_fail(ctx, e, "k_merkle_stage");
-            }
-            if (!last) {
-                if (dev_nodes) {
-                    in = nodes + (((2ull << n) - (2ull << (n - top))) * 32);
-                    in_stride = nodes_bytes;
-                } else {
-                    in = p.out;
-                    in_stride = p.out_stride;
-                }
-            }
-        }
+        st = merkle_chain(ctx, m->hash, n, stages, blocks, blk_bytes, nodes, nodes_bytes, roots_all + b0 * 32, scr,
+                          scratch_pt, nb, s);
+        if (st) return st;
         if (slot >= 0) {
             CK(cudaEventRecord(ctx->ev_consumed[slot], s));
             ctx->slot_used[slot] = true;
@@ -1290,40 +1310,110 @@ bzk_status commit_prove_impl(bzk_ctx *ctx, const bzk_encoder *E, const bzk_commi
     const uint32_t S = c->segments;
     if (S == 0 || (S & (S - 1)) || S > (1u << 20)) return fail(ctx, BZK_EINVAL, "segments must be a power of two <= 2^20");
     if (c->hash > 1) return fail(ctx, BZK_EINVAL, "hash must be BZK_MERKLE_COMPRESS or BZK_MERKLE_SHA256");
-    if (sc->flags & (BZK_F_SEEDS_DEVICE | BZK_F_GIVEN_CHALLENGES))
-        return fail(ctx, BZK_EINVAL, "the chain derives the seeds: no BZK_F_SEEDS_DEVICE / BZK_F_GIVEN_CHALLENGES");
+    if (sc->flags & (BZK_F_SEEDS_DEVICE | BZK_F_GIVEN_CHALLENGES | BZK_F_FIELD_GOLDILOCKS))
+        return fail(ctx, BZK_EINVAL, "the chain derives the seeds: no SEEDS_DEVICE / GIVEN_CHALLENGES / GOLDILOCKS");
+    if (sc->tables_mem != BZK_MEM_DEVICE || sc->outputs_mem != BZK_MEM_DEVICE)
+        return fail(ctx, BZK_EINVAL, "bzk_commit_prove takes device buffers");
+    auto mis = [](const void *q) { return q && ((uintptr_t)q & 31u); };
+    if (mis(c->codes) || mis(c->roots) || mis(c->nodes) || mis(c->final_roots))
+        return fail(ctx, BZK_EINVAL, "device buffers must be 32-byte aligned");
+    if (E->device != ctx->device) return fail(ctx, BZK_EINVAL, "encoder belongs to another device");
     bzk_batch b2 = *sc;                  // the sum-check, its transcripts seeded with the final roots
     b2.flags |= BZK_F_SEEDS_DEVICE;
     b2.seed = c->final_roots;
     bzk_status st = validate_args(ctx, &b2);   // every argument error before the first launch
     if (st) return st;
-    const uint64_t B = sc->batch;
-    // 1. encode the B x S segments in place (codeword = message || redundancy, bzk_encode)
-    st = encode_impl(ctx, E, c->codes, B * S, BZK_MEM_DEVICE, 0, s);
+    const uint64_t B = sc->batch, n = 1ull << E->log_n;
+    const uint32_t lg = [&] { uint32_t l = 0; while ((2u << l) < S) ++l; return l; }();   // top tree: S/2 blocks
+    // Module pipeline over proof chunks (P:207-213 run as stages, "all pipelined modules are fully
+    // engaged ... concurrently"): chunk j is encoded on the caller's stream while chunk j-1 is committed
+    // on a Merkle stream (ALU-pipe work beside the encoder's IMAD work) and chunk j-2 is proved on a
+    // sum-check stream; events order each chunk's three steps.
+    const uint64_t nc = std::min<uint64_t>(B, knobs().chain_chunks), Bc = (B + nc - 1) / nc;
+    const std::vector<MkStage> st1 = merkle_stages(E->log_n);
+    const std::vector<MkStage> st2 = merkle_stages(lg);
+    const size_t spt1 = c->nodes ? 0 : (size_t)32 << st1[0].lg_tpt, spt2 = (size_t)32 << st2[0].lg_tpt;
+    const size_t scr1 = align_up(Bc * S * spt1), scr2 = align_up(Bc * spt2);
+    const size_t chain_bytes = 2 * scr1 + 2 * scr2 + 256;
+    std::vector<Plan> plans(nc);
+    size_t ws_need = 0;
+    for (uint64_t j = 0; j < nc; ++j) {
+        bzk_batch bj = b2;
+        bj.batch = std::min<uint64_t>(Bc, B - j * Bc);
+        st = make_plan(ctx, &bj, plans[j]);
+        if (st) return st;
+        ws_need = std::max(ws_need, plans[j].total);
+    }
+    st = ensure_ws(ctx, ws_need);
     if (st) return st;
-    // 2. a Merkle tree per codeword: 2n elements = n blocks of 64 bytes (two elements per block)
-    bzk_merkle_batch m1;
-    memset(&m1, 0, sizeof m1);
-    m1.log_blocks = E->log_n; m1.hash = c->hash; m1.blocks_mem = BZK_MEM_DEVICE; m1.batch = B * S;
-    m1.blocks = (const uint8_t *)c->codes; m1.outputs_mem = BZK_MEM_DEVICE; m1.roots = c->roots; m1.nodes = c->nodes;
-    st = merkle_impl(ctx, &m1, s);
+    if (ctx->chain_ws_size < chain_bytes) {
+        cudaDeviceSynchronize();
+        if (ctx->chain_ws) cudaFree(ctx->chain_ws);
+        ctx->chain_ws = nullptr;
+        ctx->chain_ws_size = 0;
+        if (cudaMalloc(&ctx->chain_ws, chain_bytes) != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ctx, BZK_ENOMEM, "cudaMalloc chain scratch");
+        }
+        ctx->chain_ws_size = chain_bytes;
+    }
+    if (!ctx->chain_mk) CK(cudaStreamCreateWithFlags(&ctx->chain_mk, cudaStreamNonBlocking));
+    if (!ctx->chain_sc) CK(cudaStreamCreateWithFlags(&ctx->chain_sc, cudaStreamNonBlocking));
+    cudaStream_t smk = ctx->chain_mk, ssc = ctx->chain_sc;
+    st = call_begin(ctx, s);
     if (st) return st;
-    // 3. root of roots: the S roots of a proof are the leaves, so level 1 = H(root_2j || root_2j+1) =
-    //    the level 0 of a tree over S / 2 blocks (adjacent root pairs, already contiguous in `roots`)
-    if (S == 1) {
-        CK(cudaMemcpyAsync(c->final_roots, c->roots, B * 32, cudaMemcpyDeviceToDevice, s));
-    } else {
-        uint32_t lg = 0;
-        while ((2u << lg) < S) ++lg;
-        bzk_merkle_batch m2;
-        memset(&m2, 0, sizeof m2);
-        m2.log_blocks = lg; m2.hash = c->hash; m2.blocks_mem = BZK_MEM_DEVICE; m2.batch = B;
-        m2.blocks = c->roots; m2.outputs_mem = BZK_MEM_DEVICE; m2.roots = c->final_roots;
-        st = merkle_impl(ctx, &m2, s);
+    std::vector<cudaEvent_t> evs;
+    auto ev = [&]() { cudaEvent_t e = pool_event(ctx); evs.push_back(e); return e; };
+    auto join = [&](cudaStream_t from, cudaStream_t to) -> bzk_status {
+        cudaEvent_t e = ev();
+        CK(cudaEventRecord(e, from));
+        CK(cudaStreamWaitEvent(to, e, 0));
+        return BZK_OK;
+    };
+    if ((st = join(s, smk)) || (st = join(s, ssc))) return st;
+    char *cw = (char *)ctx->chain_ws;
+    uint8_t *const scrA[2] = {(uint8_t *)cw, (uint8_t *)cw + scr1};
+    uint8_t *const scrB[2] = {(uint8_t *)cw + 2 * scr1, (uint8_t *)cw + 2 * scr1 + scr2};
+    const size_t cw_elems = 2 * n, nodes_bytes = (size_t)(2 * n - 1) * 32;
+    const size_t tbl_words = (size_t)sc->degree * ((size_t)1 << sc->num_vars) * 4;
+    for (uint64_t j = 0; j < nc; ++j) {
+        const uint64_t b0 = j * Bc, bc = std::min<uint64_t>(Bc, B - b0);
+        fe *codes_j = (fe *)c->codes + b0 * S * cw_elems;
+        uint8_t *roots_j = c->roots + b0 * S * 32, *fin_j = c->final_roots + b0 * 32;
+        // 1. encode (caller's stream)
+        st = encode_wave(ctx, E, codes_j, bc * S, s);
+        if (st) return st;
+        if ((st = join(s, smk))) return st;
+        // 2. codeword trees + root of roots (Merkle stream)
+        st = merkle_chain(ctx, c->hash, E->log_n, st1, (const uint8_t *)codes_j, cw_elems * 32,
+                          c->nodes ? c->nodes + b0 * S * nodes_bytes : nullptr, nodes_bytes, roots_j, scrA, spt1,
+                          bc * S, smk);
+        if (st) return st;
+        if (S == 1) CK(cudaMemcpyAsync(fin_j, roots_j, bc * 32, cudaMemcpyDeviceToDevice, smk));
+        else {
+            st = merkle_chain(ctx, c->hash, lg, st2, roots_j, (uint64_t)S * 32, nullptr, 0, fin_j, scrB, spt2, bc, smk);
+            if (st) return st;
+        }
+        if ((st = join(smk, ssc))) return st;
+        // 3. the chunk's sum-checks, seeded with their final roots (sum-check stream)
+        bzk_batch bj = b2;
+        bj.batch = bc;
+        bj.first_index = b2.first_index + b0;
+        bj.seed = fin_j;
+        bj.tables = b2.tables + b0 * tbl_words;
+        bj.round_evals = b2.round_evals + b0 * (size_t)sc->num_vars * (sc->degree + 1) * 4;
+        bj.challenges = b2.challenges + b0 * (size_t)sc->num_vars * 4;
+        bj.final_evals = b2.final_evals + b0 * (size_t)sc->degree * 4;
+        bj.claims = b2.claims ? b2.claims + b0 * 4 : nullptr;
+        st = enqueue_job(ctx, &bj, plans[j], ssc);
         if (st) return st;
     }
-    // 4. the sum-check of every proof, its transcript seeded with its final root
-    return prove_jobs(ctx, &b2, 1, s);
+    if ((st = join(smk, s)) || (st = join(ssc, s))) return st;
+    for (auto e : evs) ctx->ev_pool.push_back(e);
+    st = call_end(ctx, s);
+    if (st) return st;
+    if (sc->flags & BZK_F_SYNC) CK(cudaStreamSynchronize(s));
+    return BZK_OK;
 }
 
 // ---------------------------------------------------------------- debug kernels
@@ -1580,6 +1670,9 @@ void ctx_free(bzk_ctx *ctx) {
         if (ctx->ev_nodes_copied[i]) cudaEventDestroy(ctx->ev_nodes_copied[i]);
     }
     if (ctx->ev_done) cudaEventDestroy(ctx->ev_done);
+    if (ctx->chain_mk) cudaStreamDestroy(ctx->chain_mk);
+    if (ctx->chain_sc) cudaStreamDestroy(ctx->chain_sc);
+    if (ctx->chain_ws) cudaFree(ctx->chain_ws);
     if (ctx->d2h_stream) cudaStreamDestroy(ctx->d2h_stream);
     if (ctx->graph_exec) cudaGraphExecDestroy(ctx->graph_exec);
     for (auto &r : ctx->recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }

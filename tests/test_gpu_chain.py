@@ -40,9 +40,11 @@ def run_chain(enc, log_n, S, B, d, k, order, mode, I0, dist="uniform", nodes=Fal
     return msgs.reshape(B, S, n, 4), codes, roots, fin, nd, t, out
 
 
-@pytest.mark.parametrize("S,mode,order,d", [(1, 0, 0, 2), (2, 0, 1, 1), (4, 1, 0, 3), (8, 0, 0, 2)])
-def test_chain_vs_oracle(orc, S, mode, order, d):
-    log_n, B, k = 8, 3, 11
+@pytest.mark.parametrize("S,mode,order,d,B", [(1, 0, 0, 2, 3), (2, 0, 1, 1, 2), (4, 1, 0, 3, 3), (8, 0, 0, 2, 3),
+                                              (2, 0, 0, 2, 1), (2, 1, 1, 2, 5)])
+def test_chain_vs_oracle(orc, S, mode, order, d, B):
+    """B = 1 (one chunk), 2-3 (one proof per chunk), 5 (chunks of 2, 2, 1) of the module pipeline."""
+    log_n, k = 8, 11
     code = inputs.gen_code(log_n, 6)
     enc = bzk.Encoder(code, 0)
     msgs, codes, roots, fin, _, t, out = run_chain(enc, log_n, S, B, d, k, order, mode, 40 + S)
