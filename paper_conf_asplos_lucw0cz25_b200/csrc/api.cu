@@ -179,7 +179,11 @@ struct Knobs {
     // BZK_SMALL=0/1: proofs whose tables fit a cluster's shared memory run in k_small (one launch,
     // all rounds, cluster/DSMEM reduction; small.cuh)
     uint32_t small = 1;
-    uint32_t chain_chunks = 4;   // BZK_CHAIN_CHUNKS: proof chunks of bzk_commit_prove's module pipeline
+    // BZK_CHAIN_CHUNKS: proof chunks of bzk_commit_prove's module pipeline.  Default 1 (modules in
+    // sequence): on B200 the modules do not overlap usefully -- each already fills the GPU, and the
+    // co-running Merkle/sum-check streams evict the encoder's L2-resident source vectors (zk20: 32.1 ms
+    // per step at 1 chunk, 32.6 / 33.7 / 36.0 ms at 2 / 4 / 8, profiles/r02/bench_zk20_ch*_r02m.json)
+    uint32_t chain_chunks = 1;
     Knobs() {
         if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
@@ -1329,7 +1333,8 @@ bzk_status commit_prove_impl(bzk_ctx *ctx, const bzk_encoder *E, const bzk_commi
     // engaged ... concurrently"): chunk j is encoded on the caller's stream while chunk j-1 is committed
     // on a Merkle stream (ALU-pipe work beside the encoder's IMAD work) and chunk j-2 is proved on a
     // sum-check stream; events order each chunk's three steps.
-    const uint64_t nc = std::min<uint64_t>(B, knobs().chain_chunks), Bc = (B + nc - 1) / nc;
+    const uint64_t Bc = (B + std::min<uint64_t>(B, knobs().chain_chunks) - 1) / std::min<uint64_t>(B, knobs().chain_chunks);
+    const uint64_t nc = (B + Bc - 1) / Bc;   // chunks actually used (B = 5 in chunks of 2: 3 chunks)
     const std::vector<MkStage> st1 = merkle_stages(E->log_n);
     const std::vector<MkStage> st2 = merkle_stages(lg);
     const size_t spt1 = c->nodes ? 0 : (size_t)32 << st1[0].lg_tpt, spt2 = (size_t)32 << st2[0].lg_tpt;

@@ -91,3 +91,41 @@ def test_chain_argument_errors():
             bzk.bzk_commit_prove(enc.ctx, enc.enc, c, sb)
         assert e.value.status == bzk.BZK_EINVAL
     enc.close()
+
+
+PIPE_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+sys.path.insert(0, {root!r} + "/tests")
+import oracle
+from paper_conf_asplos_lucw0cz25_b200 import bzk, inputs
+from test_gpu_chain import run_chain, np64, KEYS
+oracle.build()
+log_n, S, B, d, k = 8, 2, 5, 2, 11
+code = inputs.gen_code(log_n, 6)
+enc = bzk.Encoder(code, 0)
+msgs, codes, roots, fin, _, t, out = run_chain(enc, log_n, S, B, d, k, 1, 0, 90)
+host_t = np64(t)
+for b in range(B):
+    c_ref, r_ref, f_ref, p_ref = oracle.commit_prove(code, msgs[b], host_t[b], k, d, 1, 90 + b)
+    assert np.array_equal(np64(codes[b]).reshape(c_ref.shape), c_ref), b
+    assert bytes(fin[b].cpu().numpy()) == f_ref, b
+    for key in KEYS:
+        assert np.array_equal(np64(out[key][b]).reshape(p_ref[key].shape), p_ref[key]), (key, b)
+enc.close()
+print("pipeline ok")
+"""
+
+
+@pytest.mark.parametrize("chunks", [2, 4])
+def test_chain_module_pipeline(chunks):
+    """BZK_CHAIN_CHUNKS > 1: chunks of proofs flow through encode / Merkle / sum-check on three streams
+    (B = 5: chunks of 3 + 2 and 2 + 2 + 1); every output bit-exact."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, BZK_CHAIN_CHUNKS=str(chunks))
+    r = subprocess.run([sys.executable, "-c", PIPE_SCRIPT.format(root=root)], env=env, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "pipeline ok" in r.stdout, r.stdout + r.stderr
