@@ -442,3 +442,19 @@ def test_goldilocks_oracle_pins(orc, d, order):
     giv = orc.gl_prove(t, k, d, order, SEED, 3, given=out["challenges"])
     for key in out:
         assert np.array_equal(giv[key], out[key])
+
+
+def test_c5_golden_digests_file(orc):
+    """tests/golden/c5_proof_digests.txt (written by make_golden_c5.py from oracle/ only) covers the
+    8192 proofs of configs[1]/[4]; two of them recomputed here by the oracle."""
+    import hashlib
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "c5_proof_digests.txt")
+    rows = [ln.split() for ln in open(path) if ln.strip() and not ln.startswith("#")]
+    assert [int(i) for i, _ in rows] == list(range(8192))
+    gold = {int(i): d for i, d in rows}
+    for i in (0, 8191):
+        out = orc.prove(inputs.gen_tables(1, 2, 20, first_index=i)[0], 20, 2, 0, SEED, i)
+        h = hashlib.sha256()
+        for key in ("round_evals", "challenges", "final_evals", "claims"):
+            h.update(out[key].astype("<u8").tobytes())
+        assert h.hexdigest()[:16] == gold[i], i
