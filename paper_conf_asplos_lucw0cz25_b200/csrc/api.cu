@@ -88,6 +88,7 @@ struct bzk_ctx {
     bool ev_done_recorded = false;
     // bzk_commit_prove's module pipeline: Merkle and sum-check side streams, Merkle stage scratch
     cudaStream_t chain_mk = nullptr, chain_sc = nullptr;
+    cudaStream_t dual_stream = nullptr;
     void *chain_ws = nullptr;
     size_t chain_ws_size = 0;
 };
@@ -151,6 +152,8 @@ struct Plan {
     bool host_tables, host_outputs, need_bufX, need_bufY, bufY_alias_input;
     uint32_t given;       // BZK_F_GIVEN_CHALLENGES
     bool multi;           // given challenges, d = 1, BN254: k_multi passes (NEXT-1)
+    bool dual;            // two half-batch waves on two streams, offset by one round (see enqueue_job)
+    size_t wave_bytes;    // bytes of one wave's workspace region [off_ps, off_bufY end) (dual: two copies)
     uint32_t part_nv;     // field elements per CTA partial (D + 1, or 2^kMultiM column sums)
     bool gl;              // BZK_F_FIELD_GOLDILOCKS (NEXT-2)
     size_t esz;           // bytes per element: 32 (BN254) or 8 (Goldilocks)
@@ -184,7 +187,11 @@ struct Knobs {
     // co-running Merkle/sum-check streams evict the encoder's L2-resident source vectors (zk20: 32.1 ms
     // per step at 1 chunk, 32.6 / 33.7 / 36.0 ms at 2 / 4 / 8, profiles/r02/bench_zk20_ch*_r02m.json)
     uint32_t chain_chunks = 1;
+    // BZK_DUAL=0/1: a one-wave device batch runs as two half-batch waves on two streams, the second
+    // one round behind, so one wave's round-1 evaluation (IMAD-heavy) overlaps the other's fused rounds
+    uint32_t dual = 0;
     Knobs() {
+        if (const char *e = getenv("BZK_DUAL")) dual = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_M")) multi_m = std::max(1, std::min(3, atoi(e)));
@@ -281,6 +288,8 @@ bzk_status validate_args(bzk_ctx *ctx, const bzk_batch *b) {
     return BZK_OK;
 }
 
+int small_cs_log(uint32_t D, uint32_t k, uint64_t nb);   // k_small eligibility (run_wave)
+
 bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.k = b->num_vars; P.D = b->degree; P.order = b->order; P.B = b->batch;
     P.N = 1ull << P.k;
@@ -334,6 +343,9 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     // balance the waves
     uint64_t nw = (P.B + bw - 1) / bw;
     bw = (P.B + nw - 1) / nw;
+    P.dual = knobs().dual && nw == 1 && P.B >= 2 && !P.host_tables && !P.gl && !P.multi && P.i0 > 2 &&
+             small_cs_log(P.D, P.k, P.B) < 0;
+    if (P.dual) { nw = 2; bw = (P.B + 1) / 2; }   // two waves of B/2: the same scratch as one wave of B
     P.Bw = bw; P.nwaves = nw;
     P.cmax = P.k ? std::max(max_round_ctas(P.k, P.i0, bw), max_round_ctas(P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
     if (P.multi) P.cmax = std::max(max_multi_ctas(P.k, P.i0, bw), max_multi_ctas(P.k, P.i0, P.B - (nw - 1) * bw));
@@ -345,6 +357,8 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     P.off_part = off; off = align_up(off + (size_t)bw * P.cmax * P.part_nv * P.esz);
     P.off_bufX = off; if (P.need_bufX) off = align_up(off + (size_t)bw * P.D * (P.N / 2) * P.esz);
     P.off_bufY = off; if (P.need_bufY && !P.bufY_alias_input) off = align_up(off + (size_t)bw * P.D * (P.N / 4) * P.esz);
+    P.wave_bytes = off - P.off_ps;
+    if (P.dual) off += P.wave_bytes;              // the second wave's copy of [ps .. bufY]
     P.off_out = off; if (P.host_outputs) off = align_up(off + P.B * P.out_bytes_per_proof);
     P.total = off;
     P.stage_bytes = P.host_tables ? align_up(bw * P.elem_table) : 0;
@@ -475,6 +489,8 @@ __global__ void k_validate(const fe *t, uint64_t n, uint32_t *flag) {
 // ---------------------------------------------------------------- one wave
 
 struct WaveIO {
+    char *ws;          // this wave's workspace base (ctx->ws, or + wave_bytes for the second dual wave)
+    cudaEvent_t ev_r1; // if set: recorded on the wave's stream right after its round-1 launch (dual)
     Seed32 seed;       // transcript seed, passed to the kernel by value
     const uint8_t *seeds;   // BZK_F_SEEDS_DEVICE: this wave's per-proof seeds (device [nb][32]), else null
     char *tables;      // device tables of this wave [nb][D][N] x esz
@@ -484,7 +500,7 @@ struct WaveIO {
 
 // Goldilocks wave (gl.cuh): same schedule as run_wave, 8-byte elements
 bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t s) {
-    char *ws = (char *)ctx->ws;
+    char *ws = io.ws;
     gl::State *ps = (gl::State *)(ws + P.off_ps);
     uint32_t *tick = (uint32_t *)(ws + P.off_tick);
     uint64_t *part = (uint64_t *)(ws + P.off_part);
@@ -554,7 +570,7 @@ bzk_status run_wave_small(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStr
     memset(&sp, 0, sizeof sp);
     sp.src = (const fe *)io.tables; sp.k = P.k; sp.cs_log = (uint32_t)cs_log; sp.order = P.order; sp.given = P.given;
     sp.first_index = io.first_index; sp.seed = io.seed; sp.seeds = io.seeds;
-    sp.ps = (ProofState *)((char *)ctx->ws + P.off_ps);
+    sp.ps = (ProofState *)(io.ws + P.off_ps);
     sp.round_evals = (fe *)io.round_evals; sp.challenges = (fe *)io.challenges; sp.final_evals = (fe *)io.final_evals;
     sp.claims = (fe *)io.claims;
     const uint32_t cs = 1u << cs_log;
@@ -581,7 +597,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         const int cs_log = small_cs_log(P.D, P.k, io.nb);
         if (cs_log >= 0) return run_wave_small(ctx, P, io, s, cs_log);
     }
-    char *ws = (char *)ctx->ws;
+    char *ws = io.ws;
     ProofState *ps = (ProofState *)(ws + P.off_ps);
     uint32_t *tick = (uint32_t *)(ws + P.off_tick);
     fe *part = (fe *)(ws + P.off_part);
@@ -662,10 +678,13 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
                 return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (TMA staging)");
         }
         dim3 grid(rp.ctas, (uint32_t)io.nb);
-        ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-        cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
-        ++ctx->launches;
-        if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
+        {
+            ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
+            cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
+            ++ctx->launches;
+            if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
+        }
+        if (i == 1 && io.ev_r1) CK(cudaEventRecord(io.ev_r1, s));
     }
     {
         TailParams tp;
@@ -696,6 +715,20 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     NvtxRange nv_("bzk job");
     char *ws = (char *)ctx->ws;
     CK(cudaMemsetAsync(ws + P.off_tick, 0, P.Bw * 4, s));
+    // dual: wave 1 runs on the context's second stream, one round behind wave 0 (its first launch waits
+    // for wave 0's round-1 kernel), in its own copy of the wave workspace
+    cudaStream_t s2 = s;
+    cudaEvent_t ev_r1 = nullptr;
+    if (P.dual) {
+        if (!ctx->dual_stream) CK(cudaStreamCreateWithFlags(&ctx->dual_stream, cudaStreamNonBlocking));
+        s2 = ctx->dual_stream;
+        CK(cudaMemsetAsync(ws + P.wave_bytes + P.off_tick, 0, P.Bw * 4, s));
+        cudaEvent_t e0 = pool_event(ctx);
+        CK(cudaEventRecord(e0, s));
+        CK(cudaStreamWaitEvent(s2, e0, 0));
+        ctx->ev_pool.push_back(e0);
+        ev_r1 = pool_event(ctx);
+    }
     const bool validate = (b->flags & BZK_F_VALIDATE) != 0;
     if (validate) CK(cudaMemsetAsync(ctx->d_flag, 0, 4, s));
 
@@ -714,6 +747,13 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
     for (uint64_t w = 0; w < P.nwaves; ++w) {
         WaveIO io;
         const uint64_t b0 = w * P.Bw;
+        io.ws = ws + (P.dual && w == 1 ? P.wave_bytes : 0);
+        io.ev_r1 = (P.dual && w == 0) ? ev_r1 : nullptr;
+        cudaStream_t sw = s;
+        if (P.dual && w == 1) {
+            CK(cudaStreamWaitEvent(s2, ev_r1, 0));
+            sw = s2;
+        }
         if (b->flags & BZK_F_SEEDS_DEVICE) {
             memset(io.seed.b, 0, 32);
             io.seeds = b->seed + b0 * 32;
@@ -744,18 +784,25 @@ bzk_status enqueue_job(bzk_ctx *ctx, const bzk_batch *b, const Plan &P, cudaStre
             io.tables = (char *)b->tables + b0 * P.elem_table;
         }
         if (validate) {
-            ProfScope ps_(ctx, s, 4);
-            if (P.gl) k_validate_gl<<<kSMs * 8, 256, 0, s>>>((const uint64_t *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
-            else      k_validate<<<kSMs * 8, 256, 0, s>>>((const fe *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
+            ProfScope ps_(ctx, sw, 4);
+            if (P.gl) k_validate_gl<<<kSMs * 8, 256, 0, sw>>>((const uint64_t *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
+            else      k_validate<<<kSMs * 8, 256, 0, sw>>>((const fe *)io.tables, io.nb * P.D * P.N, ctx->d_flag);
             ++ctx->launches;
             CK(cudaGetLastError());
         }
-        bzk_status st = P.gl ? run_wave_gl(ctx, P, io, s) : run_wave(ctx, P, io, s);
+        bzk_status st = P.gl ? run_wave_gl(ctx, P, io, sw) : run_wave(ctx, P, io, sw);
         if (st) return st;
         if (slot >= 0) {
             CK(cudaEventRecord(ctx->ev_consumed[slot], s));
             ctx->slot_used[slot] = true;
         }
+    }
+    if (P.dual) {                                  // the caller's stream waits for the second wave
+        cudaEvent_t e1 = pool_event(ctx);
+        CK(cudaEventRecord(e1, s2));
+        CK(cudaStreamWaitEvent(s, e1, 0));
+        ctx->ev_pool.push_back(e1);
+        ctx->ev_pool.push_back(ev_r1);
     }
     if (P.host_outputs) {
         if (P.k) {
@@ -1676,6 +1723,7 @@ void ctx_free(bzk_ctx *ctx) {
     }
     if (ctx->ev_done) cudaEventDestroy(ctx->ev_done);
     if (ctx->chain_mk) cudaStreamDestroy(ctx->chain_mk);
+    if (ctx->dual_stream) cudaStreamDestroy(ctx->dual_stream);
     if (ctx->chain_sc) cudaStreamDestroy(ctx->chain_sc);
     if (ctx->chain_ws) cudaFree(ctx->chain_ws);
     if (ctx->d2h_stream) cudaStreamDestroy(ctx->d2h_stream);
