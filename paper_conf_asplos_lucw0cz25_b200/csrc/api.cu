@@ -189,6 +189,9 @@ struct Knobs {
     uint32_t chain_chunks = 1;
     // BZK_DUAL=0/1: a one-wave device batch runs as two half-batch waves on two streams, the second
     // one round behind, so one wave's round-1 evaluation (IMAD-heavy) overlaps the other's fused rounds
+    // (the paper's "different proofs in different rounds").  Off: every round kernel already
+    // fills the 148 SMs, so the overlap measured +0.2 % (c2), +0.4 % (c3), +0.9 % (m0) -- within noise
+    // (profiles/r02/bench_*_dual*_r02p.json)
     uint32_t dual = 0;
     Knobs() {
         if (const char *e = getenv("BZK_DUAL")) dual = atoi(e) ? 1 : 0;

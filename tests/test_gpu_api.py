@@ -236,3 +236,36 @@ def test_per_round_path_at_small_k():
     r = subprocess.run([sys.executable, "-c", PERROUND_SCRIPT.format(root=ROOT)], env=env, capture_output=True,
                        text=True, timeout=900)
     assert r.returncode == 0 and "per-round ok" in r.stdout, r.stdout + r.stderr
+
+
+DUAL_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r})
+import oracle
+from paper_conf_asplos_lucw0cz25_b200 import bzk, inputs
+oracle.build()
+p = bzk.Prover(0)
+for (B, d, k, order, flags) in [(6, 2, 14, 0, bzk.BZK_F_PRESERVE_INPUT), (5, 3, 13, 1, 0), (4, 1, 15, 1, 0),
+                                (3, 4, 12, 0, bzk.BZK_F_PRESERVE_INPUT), (2, 2, 16, 1, 0)]:
+    t = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(t, B, d, k, 21, "adversarial")
+    host = t.cpu().numpy().view(np.uint64).copy()
+    out = p.prove(t, k, d, order, first_index=21, flags=flags)
+    torch.cuda.synchronize()
+    for b in range(B):
+        ref = oracle.prove(host[b], k, d, order, inputs.DEFAULT_SEED, 21 + b)
+        for key in ref:
+            got = out[key][b].cpu().numpy().view(np.uint64).reshape(ref[key].shape)
+            assert np.array_equal(got, ref[key]), (key, B, d, k, order, b)
+p.close()
+print("dual ok")
+"""
+
+
+def test_dual_stream_waves():
+    """BZK_DUAL=1: a one-wave batch runs as two half waves on two streams, the second one round behind
+    (measured no faster on B200 -- profiles/r02/bench_*_dual*_r02p.json -- so off by default)."""
+    env = dict(os.environ, BZK_DUAL="1")
+    r = subprocess.run([sys.executable, "-c", DUAL_SCRIPT.format(root=ROOT)], env=env, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "dual ok" in r.stdout, r.stdout + r.stderr
