@@ -161,12 +161,10 @@ struct Plan {
 };
 
 // tuning knobs (environment, read once): BZK_PPT_MAX (max pairs per thread), BZK_CTA_WAVES
-// (target CTA waves per launch), BZK_PREFETCH (L2 bulk prefetch in k_round; default: on for d >= 3 only)
+// (target CTA waves per launch).  (Round 1's L2 bulk prefetch option was removed in round 2: the TMA
+// staging replaced it for d >= 3, the only degree it had helped.)
 struct Knobs {
     uint64_t ppt_max = 256, waves = 4;   // ppt_max sweep 32..1024: 256 best for c2, c3, m0
-    // L2 bulk prefetch: -1 = by degree.  d <= 2: off (the fused rounds then read exactly their bytes;
-    // with it 1.5x, -6 % at c2, -2 % at m0); d >= 3: on (IMAD-bound, +2 % at c3).  DESIGN.md sec. 8.
-    int prefetch = -1;
     // BZK_CLUSTER=N: CTAs of a proof form thread-block clusters of up to N (2, 4, 8) that combine
     // their partial sums through DSMEM.  Off by default: measured 10 % slower on B200.
     uint32_t cluster = 1;
@@ -175,9 +173,6 @@ struct Knobs {
     // profiles/r02/r02b_*: c2 fused rounds -11 % time, c2 round 1 +7 %, c3 both -3 %, m0 (d = 1) +3 %);
     // BZK_TMA=0 / 1 forces it off / on everywhere
     int tma = -1;
-    // BZK_MULTI=0/1: given-challenge d = 1 proofs run k_multi passes (several rounds per read of the
-    // table, multiround.cuh) instead of one k_round launch per round
-    uint32_t multi = 1;
     uint32_t multi_m = 3;      // BZK_MULTI_M: rounds per k_multi pass (1..3)
     // BZK_SMALL=0/1: proofs whose tables fit a cluster's shared memory run in k_small (one launch,
     // all rounds, cluster/DSMEM reduction; small.cuh)
@@ -198,19 +193,14 @@ struct Knobs {
         if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_M")) multi_m = std::max(1, std::min(3, atoi(e)));
-        if (const char *e = getenv("BZK_MULTI")) multi = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_TMA")) tma = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CLUSTER")) cluster = std::max(1, std::min(8, atoi(e)));
         if (const char *e = getenv("BZK_PPT_MAX")) ppt_max = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_CTA_WAVES")) waves = std::max(1, atoi(e));
-        if (const char *e = getenv("BZK_PREFETCH")) prefetch = atoi(e) ? 1 : 0;
     }
     uint32_t tma_for(uint32_t d, bool first) const {
         if (tma >= 0) return (uint32_t)tma;
         return first ? (d >= 3 ? 1u : 0u) : (d >= 2 ? 1u : 0u);
-    }
-    uint32_t prefetch_for(uint32_t d) const {
-        return prefetch < 0 ? (d >= 3 ? 1u : 0u) : (uint32_t)prefetch;
     }
 };
 const Knobs &knobs() { static Knobs k; return k; }
@@ -305,7 +295,8 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     if (P.k == 0) { P.i0 = 1; P.log_h0 = 0; }
     else if (P.k - 1 <= kTailLog) { P.i0 = 1; P.log_h0 = P.k - 1; }
     else { P.i0 = P.k - kTailLog; P.log_h0 = kTailLog; }
-    P.multi = P.given && P.D == 1 && !P.gl && P.i0 > 1 && knobs().multi;
+    // given challenges, d = 1 (Alg. 1): k_multi passes, several rounds per read of the table (NEXT-1)
+    P.multi = P.given && P.D == 1 && !P.gl && P.i0 > 1;
     P.part_nv = P.multi ? (1u << kMultiM) : P.D + 1;
     const bool preserve = (b->flags & BZK_F_PRESERVE_INPUT) != 0;
     P.need_bufX = P.i0 > 2;
@@ -662,7 +653,6 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = (fe *)io.round_evals; rp.challenges = (fe *)io.challenges; rp.claims = (fe *)io.claims;
         rp.consts = ctx->consts;
-        rp.prefetch = knobs().prefetch_for(P.D);
         rp.given = P.given;
         rp.cluster = cluster_for(rp.ctas);
         if (i == 1) { rp.src = tab; rp.dst = nullptr; }
@@ -674,7 +664,6 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         memset(&tm, 0, sizeof tm);
         rp.tma = knobs().tma_for(D, i == 1);
         if (rp.tma) {
-            rp.prefetch = 0;
             const uint64_t E = i == 1 ? 2 : 4;   // raw entries per pair and table
             const uint32_t box = P.order == 0 ? (uint32_t)(E * 8) : 8u;
             if (!make_row_map(&tm, rp.src, io.nb * D * E * h / 4, box))

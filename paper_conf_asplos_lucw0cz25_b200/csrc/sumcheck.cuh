@@ -67,7 +67,6 @@ struct RoundParams {
     fe *challenges;       // [Bw][k]
     fe *claims;           // [Bw] (may be null)
     const fe *consts;     // kNumConsts
-    uint32_t prefetch;    // 1: bulk-prefetch the next iteration's tiles into L2
     uint32_t given;       // 1: challenges are inputs (BZK_F_GIVEN_CHALLENGES), no transcript
     uint32_t cluster;     // thread-block cluster size along x (1 = none); divides ctas
     uint32_t zero;        // always 0 (opaque to the compiler: orders the fold-table loads, fixmul_lz)
@@ -582,41 +581,6 @@ __device__ __forceinline__ fe tma_entry(const uint8_t *slot, uint32_t lane, int 
     return r;
 }
 
-#ifndef BZK_PF_DIST
-#define BZK_PF_DIST 1   // prefetch distance in loop iterations (grid strides): 1 beats 2 and 4
-#endif
-
-// L2 bulk prefetch of a contiguous byte range (cp.async.bulk.prefetch, sm_90+; no registers, no smem)
-__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes) {
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
-
-// Lane 0 of a warp prefetches into L2 the table ranges that the warp's 32 lanes will load for the
-// pairs j0 .. j0+31 (j0 = the warp's first pair index): one contiguous range per table for LSB,
-// two for MSB.
-template <int D, int ORDER, bool FIRST>
-__device__ __forceinline__ void prefetch_pairs(const fe *src, uint64_t h, uint64_t j0) {
-    if (j0 >= h) return;
-    const uint64_t n = (h - j0) < 32 ? (h - j0) : 32;
-#pragma unroll
-    for (int m = 0; m < D; ++m) {
-        if (FIRST) {
-            const fe *T = src + (size_t)m * (2 * h);
-            if (ORDER == 0) prefetch_l2(T + 2 * j0, (uint32_t)(n * 64));
-            else { prefetch_l2(T + j0, (uint32_t)(n * 32)); prefetch_l2(T + j0 + h, (uint32_t)(n * 32)); }
-        } else {
-            const fe *T = src + (size_t)m * (4 * h);
-            if (ORDER == 0) prefetch_l2(T + 4 * j0, (uint32_t)(n * 128));
-            else {
-                prefetch_l2(T + j0, (uint32_t)(n * 32));
-                prefetch_l2(T + j0 + h, (uint32_t)(n * 32));
-                prefetch_l2(T + j0 + 2 * h, (uint32_t)(n * 32));
-                prefetch_l2(T + j0 + 3 * h, (uint32_t)(n * 32));
-            }
-        }
-    }
-}
-
 template <int D, int ORDER, bool FIRST, bool TMA>
 __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
     k_round(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
@@ -716,7 +680,6 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
 #pragma unroll
         for (int t = 0; t < NV; ++t) uacc[t] = acc17_zero();
         for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
-            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + BZK_PF_DIST * stride);
             fe a[D], sv[D];
             load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
             eval_one<D, DERIVE>(a, sv, uacc);
@@ -727,7 +690,6 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
         fe ha[D], hs[D];
         bool held = false;
         for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < h; j += stride) {
-            if (P.prefetch && lane == 0) prefetch_pairs<D, ORDER, FIRST>(src, h, j + BZK_PF_DIST * stride);
             fe a[D], sv[D];
             load_pair<D, ORDER, FIRST>(src, dst, h, j, rm, sK, P.zero, a, sv);
             if (held) {
