@@ -177,7 +177,8 @@ def bzk_destroy(ctx) -> None:
 
 def make_batch(k, d, order, flags, batch, first_index, seed_buf, tables, tables_mem, outputs_mem, round_evals,
                challenges, final_evals, claims) -> bzk_batch:
-    return bzk_batch(k, d, order, flags, batch, first_index, ctypes.cast(seed_buf, ctypes.c_void_p), ptr(tables),
+    seed = ctypes.c_void_p(seed_buf) if isinstance(seed_buf, int) else ctypes.cast(seed_buf, ctypes.c_void_p)
+    return bzk_batch(k, d, order, flags, batch, first_index, seed, ptr(tables),
                      tables_mem, outputs_mem, ptr(round_evals), ptr(challenges), ptr(final_evals), ptr(claims))
 
 

@@ -269,3 +269,35 @@ def test_dual_stream_waves():
     r = subprocess.run([sys.executable, "-c", DUAL_SCRIPT.format(root=ROOT)], env=env, capture_output=True, text=True,
                        timeout=600)
     assert r.returncode == 0 and "dual ok" in r.stdout, r.stdout + r.stderr
+
+
+@pytest.mark.parametrize("gl", [False, True])
+def test_per_proof_device_seeds(prover, orc, gl):
+    """BZK_F_SEEDS_DEVICE: proof b's transcript starts from its own 32-byte seed (device [B][32]);
+    BN254 through both execution paths (k_small at k = 11, per-round kernels at k = 15) and Goldilocks."""
+    d, order = 2, 1
+    for k, B in ((11, 3), (15, 3)):
+        seeds = np.stack([np.frombuffer(bytes((7 * b + i) & 0xFF for i in range(32)), np.uint8) for b in range(B)])
+        sd = torch.from_numpy(seeds.copy()).cuda()
+        if gl:
+            t = torch.empty((B, d, 1 << k), dtype=torch.int64, device="cuda")
+            bzk.bzk_generate(t, B, d, k, 40, "gl_adversarial")
+            out = bzk.Prover.alloc_outputs_gl(B, k, d)
+            flags = bzk.BZK_F_FIELD_GOLDILOCKS
+        else:
+            t = dev_tables(B, d, k, 40, "adversarial")
+            out = bzk.Prover.alloc_outputs(B, k, d)
+            flags = 0
+        b = bzk.make_batch(k, d, order, flags | bzk.BZK_F_SEEDS_DEVICE | bzk.BZK_F_PRESERVE_INPUT, B, 40, sd.data_ptr(),
+                           t, bzk.BZK_MEM_DEVICE, bzk.BZK_MEM_DEVICE, out["round_evals"], out["challenges"],
+                           out["final_evals"], out["claims"])
+        bzk.bzk_prove(prover.ctx, b)
+        torch.cuda.synchronize()
+        host = np64(t)
+        for i in range(B):
+            if gl:
+                ref = orc.gl_prove(host[i], k, d, order, seeds[i].tobytes(), 40 + i)
+            else:
+                ref = orc.prove(host[i], k, d, order, seeds[i].tobytes(), 40 + i)
+            for key in KEYS:
+                assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), (key, i, k)
