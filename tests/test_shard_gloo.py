@@ -73,3 +73,38 @@ def test_two_rank_gloo_equals_single_process(orc):
     for k in KEYS:
         assert np.array_equal(res["outs"][k].view(np.uint64), single[k]), k
     assert res["tmax"] == 2.0 and res["ndig"] == 2
+
+
+def _gather_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        first, count = shard.shard_range(7, world, rank)           # uneven shards: 3 / 2 / 2
+        t = {"a": torch.arange(first * 4, (first + count) * 4, dtype=torch.int64).reshape(count, 4),
+             "b": torch.full((count, 2), rank, dtype=torch.int64)}
+        g = shard.gather_outputs(t, dist, dst=0)
+        if rank == 0:
+            q.put({k: v.numpy() for k, v in g.items()})
+        else:
+            assert g is None
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(300)
+def test_gather_to_rank0_uneven_shards():
+    """shard.gather_outputs: torch.distributed.gather to rank 0 only, shards of unequal size padded
+    and trimmed, concatenated in rank order (the c5 strong-scaling gather)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gather_worker, args=(r, 3, port, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=240)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert np.array_equal(res["a"], np.arange(28).reshape(7, 4))
+    assert res["b"][:, 0].tolist() == [0, 0, 0, 1, 1, 2, 2]
