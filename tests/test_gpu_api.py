@@ -301,3 +301,14 @@ def test_per_proof_device_seeds(prover, orc, gl):
                 ref = orc.prove(host[i], k, d, order, seeds[i].tobytes(), 40 + i)
             for key in KEYS:
                 assert np.array_equal(np64(out[key][i]).reshape(ref[key].shape), ref[key]), (key, i, k)
+
+
+@pytest.mark.parametrize("order", [0, 1])
+def test_single_large_proof(prover, orc, order):
+    """One proof with k = 22 (d = 2, 256 MiB of tables): many CTAs per proof in every global round
+    (the ticket reduction over hundreds of partials), full-field tables, against the oracle."""
+    k, d = 22, 2
+    t = dev_tables(1, d, k, 77)
+    out = prover.prove(t, k, d, order, first_index=77, flags=bzk.BZK_F_PRESERVE_INPUT)
+    torch.cuda.synchronize()
+    check(orc, np64(t), out, k, d, order, 77, [0])
