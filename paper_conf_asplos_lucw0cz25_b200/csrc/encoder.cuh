@@ -74,8 +74,11 @@ __device__ __forceinline__ fe ld_fe_hint(const fe *p, uint64_t pol) {
 #define BZK_ENC_TPB 128  // threads per CTA (4 warp slices; finer occupancy steps at ~100 registers)
 #endif
 
+// minBlocks = 1 in the launch bounds is not a no-op: ptxas then allocates 120 registers (4 CTAs/SM)
+// instead of 100 (5 CTAs/SM), and the 120-register schedule is 9 % faster on B200 (enc20 75.8 vs
+// 82.5 ms per step, profiles/r01l_bench_enc20.json vs r02/bench_enc20_r02z.json)
 template <int K, int U>
-__global__ void __launch_bounds__(BZK_ENC_TPB) k_spmv(SpmvParams p) {
+__global__ void __launch_bounds__(BZK_ENC_TPB, 1) k_spmv(SpmvParams p) {
     const uint32_t lane = threadIdx.x & 31;
     constexpr uint32_t SPC = BZK_ENC_TPB / 32;   // slices per CTA
     const uint32_t warp = threadIdx.x >> 5;
