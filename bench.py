@@ -753,6 +753,9 @@ def run_sumcheck(args, rank, world, local):
             dist.init_process_group(backend)
 
     B, d, k, order, gen_dist, desc = CONFIGS[args.config]
+    if args.k is not None:                        # size sweeps (Table 4 analogue): override k
+        desc = desc.replace("k=%d" % k, "k=%d" % args.k)
+        k = args.k
     strong = args.config == "c5"
     if strong:
         # configs[4]: the GLOBAL batch is fixed; rank r proves the contiguous indices shard_range(B, W, r)
@@ -954,6 +957,10 @@ def run_sumcheck(args, rank, world, local):
         line["dist"] = {"backend": dist.get_backend(), "world_size": dist.get_world_size(),
                         "nccl_version": ".".join(map(str, torch.cuda.nccl.version())) if dist.get_backend() == "nccl"
                         else None, "data_path_collectives": 0}
+    if args.config in ("m0", "m0lit"):
+        line["context"] = ("paper Table 4 (P:268-276): 5.622 proofs/ms at N = 2^20 on GH200 for Alg. 1 "
+                           "(single multilinear, pre-seeded challenges); 1.461 / 2.884 / 10.610 / 19.753 at "
+                           "2^22 / 2^21 / 2^19 / 2^18 -- other hardware, context only")
     if gathered:
         line["proofs_gathered"] = gathered
     if gold:
@@ -1153,6 +1160,7 @@ def main():
     ap.add_argument("--ref-proofs", type=int, default=None, help="oracle sample (default min(B, 4 x cores))")
     ap.add_argument("--vml-chunk", type=int, default=0, help="c4: images per job group (0 = all)")
     ap.add_argument("--wave", type=int, default=1024, help="c5: proofs per wave on each GPU (<= 1024)")
+    ap.add_argument("--k", type=int, default=None, help="sum-check configs: override k (size sweeps)")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
