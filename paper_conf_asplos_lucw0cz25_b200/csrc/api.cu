@@ -1681,7 +1681,7 @@ cudaError_t run_bench(uint32_t iters, double *rate, cudaStream_t s) {
 
 extern "C" {
 
-const char *bzk_version(void) { return "bzk 0.3 sm_100a (BN254 Fr + Goldilocks sum-check, SHA-256 Fiat-Shamir, batched Merkle trees, linear-time encoder)"; }
+const char *bzk_version(void) { return "bzk 0.4 sm_100a (BN254 Fr + Goldilocks sum-check, SHA-256 Fiat-Shamir, TMA-staged rounds, cluster small-batch kernel, known-challenge multi-round passes, batched Merkle trees, linear-time encoder, section-4 chain)"; }
 
 const char *bzk_strerror(bzk_status s) {
     switch (s) {
