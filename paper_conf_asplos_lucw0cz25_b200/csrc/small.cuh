@@ -43,7 +43,8 @@ __global__ void __launch_bounds__(256) k_small(SmallParams P) {
     namespace cg = cooperative_groups;
     cg::cluster_group cl = cg::this_cluster();
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ fe s_wpart[8][D + 1];      // this CTA's per-warp round partials (the leader reads them)
+    __shared__ fe s_wpart[8][D + 1];      // this CTA's per-warp round partials
+    __shared__ fe s_cpart[D + 1];         // this CTA's round partial (the leader reads it over DSMEM)
     __shared__ fe s_rm;                   // leader: r_i R for every CTA of the cluster
     __shared__ fe s_g[2][D][8];           // leader: the last c rounds on the gathered entries
     const uint32_t CS = 1u << P.cs_log, q = cl.block_rank();
@@ -55,7 +56,10 @@ __global__ void __launch_bounds__(256) k_small(SmallParams P) {
     fe *evals = P.round_evals + (size_t)b * k * (D + 1);
     fe *chals = P.challenges + (size_t)b * k;
     fe *claim = P.claims ? P.claims + b : nullptr;
-    ProofState &ps = P.ps[b];
+    // the transcript state lives in the leader's shared memory for the whole proof (the per-round
+    // finalisation is the serial critical path: no global-memory round trip for state_i)
+    __shared__ ProofState s_ps;
+    ProofState &ps = s_ps;
 
     if (q == 0 && threadIdx.x == 0 && !P.given) {    // state_0 (P:211 seed; reading R6)
         uint32_t st[8];
@@ -102,23 +106,40 @@ __global__ void __launch_bounds__(256) k_small(SmallParams P) {
     if (nl >= 2) eval_round(acc, nl);
     uint32_t round = 1;
     for (; nl >= 2; ++round) {
-        // warp sums -> shared memory; after the cluster barrier the leader warp sums the 8 CS warp
-        // partials of the whole cluster (one remote load per lane, shuffle tree)
+        // warp sums -> shared memory -> the CTA's partial (warp 0, lanes 0..7: local loads, 3-level
+        // shuffle tree); after the cluster barrier the leader warp's lanes 0..CS-1 each load ONE remote
+        // CTA partial and a 3-level shuffle tree sums them (phase trace: the previous one-warp gather of
+        // all 8 CS warp partials took 3.8 K cycles per round, profiles/r02/r02k_trace_small_c1.txt)
         warp_reduce<D + 1>(acc);
-        if ((threadIdx.x & 31) == 0)
+        const uint32_t lane = threadIdx.x & 31;
+        if (lane == 0)
 #pragma unroll
             for (int t = 0; t <= D; ++t) s_wpart[threadIdx.x >> 5][t] = acc[t];
-        cl.sync();                                    // partials visible cluster-wide
+        __syncthreads();
+        if (threadIdx.x < 32) {
+#pragma unroll
+            for (int t = 0; t <= D; ++t) acc[t] = lane < 8 ? s_wpart[lane][t] : fe_zero();
+#pragma unroll
+            for (int off = 4; off > 0; off >>= 1)
+#pragma unroll
+                for (int t = 0; t <= D; ++t) acc[t] = fe_add(acc[t], shfl_down_fe(acc[t], off));
+            if (lane == 0)
+#pragma unroll
+                for (int t = 0; t <= D; ++t) s_cpart[t] = acc[t];
+        }
+        cl.sync();                                    // CTA partials visible cluster-wide
         if (q == 0 && threadIdx.x < 32) {
-            const uint32_t lane = threadIdx.x;
 #pragma unroll
             for (int t = 0; t <= D; ++t) acc[t] = fe_zero();
-            for (uint32_t s2 = lane; s2 < CS * 8; s2 += 32) {
-                const fe *rp = cl.map_shared_rank(&s_wpart[s2 & 7][0], s2 >> 3);
+            if (lane < CS) {
+                const fe *rp = cl.map_shared_rank(s_cpart, lane);
 #pragma unroll
-                for (int t = 0; t <= D; ++t) acc[t] = fe_add(acc[t], rp[t]);
+                for (int t = 0; t <= D; ++t) acc[t] = rp[t];
             }
-            warp_reduce<D + 1>(acc);
+#pragma unroll
+            for (int off = 4; off > 0; off >>= 1)
+#pragma unroll
+                for (int t = 0; t <= D; ++t) acc[t] = fe_add(acc[t], shfl_down_fe(acc[t], off));
         }
         if (q == 0 && threadIdx.x == 0) {
             fe rm;

@@ -8,16 +8,15 @@ B, d, k = 16, 2, 12
 t = torch.empty((B, d, 1 << k, 4), dtype=torch.int64, device="cuda")
 bzk.bzk_generate(t, B, d, k, 0, "uniform")
 out = bzk.Prover.alloc_outputs(B, k, d)
-big = torch.zeros((B + 200, 4), dtype=torch.int64, device="cuda")
+big = torch.zeros((B + 400, 4), dtype=torch.int64, device="cuda")
 out["claims"] = big
 p = bzk.Prover(0)
 for _ in range(3):
     p.prove(t, k, d, 0, flags=bzk.BZK_F_PRESERVE_INPUT, out=out)
 torch.cuda.synchronize()
 raw = big.cpu().numpy().reshape(-1).view(np.int64)
-T = raw[15 * 4:15 * 4 + 800].reshape(-1, 8)
-names = ["eval", "blockred", "sync1", "gather", "finalize", "sync2", "fold+sync"]
+T = raw[15 * 4:15 * 4 + 1000].reshape(-1, 10)
+names = ["eval+warpreduce", "sync1", "gather(leader warp)", "load st", "sha256 x3", "stores", "r R", "sync2", "fold+next eval"]
 for r in range(1, 9):
     row = T[r]
-    print(r, " ".join(f"{n}={row[i+1]-row[i]}" for i, n in enumerate(["eval", "blockred", "sync1"])),
-          f"gather={row[4]-row[3]} finalize={row[5]-row[4]} sync2+wait={row[6]-row[5]} fold={row[7]-row[6]} total={row[7]-row[0]}")
+    print(r, " ".join(f"{n}={row[i+1]-row[i]}" for i, n in enumerate(names)), "total", row[9] - row[0])
