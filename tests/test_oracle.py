@@ -458,3 +458,43 @@ def test_c5_golden_digests_file(orc):
         for key in ("round_evals", "challenges", "final_evals", "claims"):
             h.update(out[key].astype("<u8").tobytes())
         assert h.hexdigest()[:16] == gold[i], i
+
+
+@pytest.mark.parametrize("order", [0, 1])
+def test_multiround_identity_reading_r26(order):
+    """Reading R26, checked in plain Python integers against Algorithm 1 run round by
+    round (oracle/py/sumcheck.py alg1 for MSB; the LSB fold for order 0): after m known-challenge rounds
+    A'[y] = sum_z w(z) A[y, z] with w the eq-weights of r_1..r_m, and the rounds' sums are the
+    w_{<i}-weighted column sums -- the identity k_multi evaluates."""
+    from oracle.py import sumcheck as ps
+    rnd = random.Random(26 + order)
+    P = ps.P
+    K, m = 7, 3
+    A = [rnd.randrange(P) for _ in range(1 << K)]
+    r = [rnd.randrange(P) for _ in range(m)]
+    # reference: m rounds of Alg. 1 (MSB pairs b, b + h) or the LSB pairing (2j, 2j + 1)
+    T, sums = list(A), []
+    for i in range(m):
+        h = len(T) // 2
+        pairs = [(T[j], T[j + h]) if order == 1 else (T[2 * j], T[2 * j + 1]) for j in range(h)]
+        sums.append((sum(a for a, _ in pairs) % P, sum(b for _, b in pairs) % P))
+        T = [(a + r[i] * (b - a)) % P for a, b in pairs]
+    if order == 1:
+        assert [tuple(x) for x in ps.alg1(A, r + [0] * (K - m))[:m]] == sums
+    # the identity
+    Ny = 1 << (K - m)
+    def bit(z, i):          # the bit of z bound in round i (1-based)
+        return (z >> (m - i)) & 1 if order == 1 else (z >> (i - 1)) & 1
+    def entry(y, z):
+        return A[y + z * Ny] if order == 1 else A[(y << m) + z]
+    def weight(z, upto):
+        w = 1
+        for i in range(1, upto + 1):
+            w = w * (r[i - 1] if bit(z, i) else (1 - r[i - 1])) % P
+        return w
+    assert [sum(weight(z, m) * entry(y, z) for z in range(1 << m)) % P for y in range(Ny)] == T
+    C = [sum(entry(y, z) for y in range(Ny)) % P for z in range(1 << m)]
+    for i in range(1, m + 1):
+        g0 = sum(weight(z, i - 1) * C[z] for z in range(1 << m) if bit(z, i) == 0) % P
+        g1 = sum(weight(z, i - 1) * C[z] for z in range(1 << m) if bit(z, i) == 1) % P
+        assert (g0, g1) == sums[i - 1], i
