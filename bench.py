@@ -667,6 +667,7 @@ GOLDEN_DIGESTS = os.path.join(ROOT, "tests", "golden", "c5_proof_digests.txt")
 # IMAD.WIDE = 2 fma-heavy slots.  Fixed-multiplier fold (fixmul_lz): 64 + 18 products; unreduced
 # 256 x 256-bit product into a 544-bit accumulator (mul_acc): 64; full Montgomery product: 136.
 SLOT_FIXMUL, SLOT_MULACC, SLOT_MONT = 164, 128, 272
+SLOT_TC_ROW = 185   # IMAD instructions in k_multi_tc's epilogue per output row (cuobjdump -sass)
 
 
 def multi_passes(k: int, m_max: int = 3):
@@ -681,6 +682,11 @@ def multi_passes(k: int, m_max: int = 3):
     return out
 
 
+def multi_tc_pass(K: int, m: int) -> bool:
+    """api.cu multi_use_tc: three-round passes over >= 2^10 entries run k_multi_tc (tensor cores)"""
+    return m == 3 and K >= 10 and os.environ.get("BZK_MULTI_TC", "1") != "0"
+
+
 def imad_slots(d: int, k: int, kind: str) -> int:
     """fma-heavy slots of the products one proof's launches of `kind` execute (the kernels' arithmetic,
     DESIGN.md sec. 6): round 1 sums d+1 points per pair, each (d-2) Montgomery products + 1 unreduced
@@ -693,8 +699,13 @@ def imad_slots(d: int, k: int, kind: str) -> int:
         return (d + 1) * point * (1 << (k - 1)) if i0 > 1 else 0
     if kind == "fused":
         return sum((2 * d * SLOT_FIXMUL + d * point) * (1 << (k - i)) for i in range(2, i0))
+    passes = multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3")))
     if kind == "multi":
-        return sum(SLOT_MULACC * (1 << K) for K, _ in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3"))))
+        return sum(SLOT_MULACC * (1 << K) for K, m in passes if not multi_tc_pass(K, m))
+    if kind == "multi_tc":
+        # k_multi_tc: the products run on the tensor cores; the integer pipe carries the epilogue
+        # (column values -> 16 words, one 9-word REDC) once per output row
+        return sum(SLOT_TC_ROW * (1 << (K - m)) for K, m in passes if multi_tc_pass(K, m))
     if kind == "small":
         # k_small: every round sums all d+1 points with (d-1) canonical Montgomery products each and
         # folds d entries per pair with one Montgomery product
@@ -702,9 +713,11 @@ def imad_slots(d: int, k: int, kind: str) -> int:
     raise ValueError(kind)
 
 
-def multi_bytes(k: int) -> int:
-    """algorithmic HBM bytes per proof of the k_multi passes: each reads its table once, writes 2^-m"""
-    return sum(32 * ((1 << K) + (1 << (K - m))) for K, m in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3"))))
+def multi_bytes(k: int, tc: bool | None = None) -> int:
+    """algorithmic HBM bytes per proof of the known-challenge passes (tc: only the k_multi_tc ones /
+    only the k_multi ones / None: all): each reads its table once, writes 2^-m"""
+    return sum(32 * ((1 << K) + (1 << (K - m))) for K, m in multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3")))
+               if tc is None or multi_tc_pass(K, m) == tc)
 
 
 def proof_digests(out: dict) -> list:
@@ -884,16 +897,18 @@ def run_sumcheck(args, rank, world, local):
 
     # ---------------- roofline of the dominant kernel
     hbm_peak, sm_max_mhz, peak_src = peaks()
-    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused", "multi_round": "multi", "small_cluster": "small"}
+    kinds = {"round1_eval": "round1", "fused_fold_eval": "fused", "multi_round": "multi", "small_cluster": "small",
+             "multi_round_tc": "multi_tc"}
     dom = max(kinds, key=lambda n: prof[n][0])
     dom_ms, dom_cnt = prof[dom]
     launches_per_step = max(1, dom_cnt / args.steps)
     avg_launch_s = dom_ms / max(1, dom_cnt) / 1000.0
     slot_peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6          # fma-heavy slots / s
     slots_per_launch = imad_slots(d, k, kinds[dom]) * count / launches_per_step
-    if kinds[dom] == "multi":
-        bytes_per_launch = multi_bytes(k) * count / launches_per_step
-        mulmods_per_launch = sum((1 << K) for K, _ in multi_passes(k)) * count / launches_per_step
+    if kinds[dom] in ("multi", "multi_tc"):
+        tc = kinds[dom] == "multi_tc"
+        bytes_per_launch = multi_bytes(k, tc) * count / launches_per_step
+        mulmods_per_launch = sum((1 << K) for K, m in multi_passes(k) if multi_tc_pass(K, m) == tc) * count / launches_per_step
     elif kinds[dom] == "small":
         bytes_per_launch = d * (1 << k) * esz * count / launches_per_step
         mulmods_per_launch = alg_mulmods(d, k, "total") * count / launches_per_step

@@ -26,9 +26,10 @@ BZK_MEM_DEVICE, BZK_MEM_HOST = 0, 1
 BZK_F_PRESERVE_INPUT, BZK_F_VALIDATE, BZK_F_SYNC, BZK_F_GRAPH, BZK_F_GIVEN_CHALLENGES = 1, 2, 4, 8, 16
 BZK_F_FIELD_GOLDILOCKS = 32
 BZK_F_SEEDS_DEVICE = 64
-BZK_PROF_KINDS = 11
+BZK_PROF_KINDS = 12
 PROF_KIND_NAMES = ["round1_eval", "fused_fold_eval", "tail", "transcript_init", "validate", "h2d_copy",
-                   "merkle_stage", "d2h_copy", "encoder_spmv", "multi_round", "small_cluster"]
+                   "merkle_stage", "d2h_copy", "encoder_spmv", "multi_round", "small_cluster",
+                   "multi_round_tc"]
 BZK_MERKLE_COMPRESS, BZK_MERKLE_SHA256 = 0, 1
 
 EXPORTS = ["bzk_create", "bzk_destroy", "bzk_workspace_size", "bzk_prove", "bzk_prove_ragged", "bzk_sync",

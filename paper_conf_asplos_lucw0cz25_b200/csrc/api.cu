@@ -188,7 +188,11 @@ struct Knobs {
     // fills the 148 SMs, so the overlap measured +0.2 % (c2), +0.4 % (c3), +0.9 % (m0) -- within noise
     // (profiles/r02/bench_*_dual*_r02p.json)
     uint32_t dual = 0;
+    // BZK_MULTI_TC=0/1: three-round known-challenge passes over >= 2^10 entries run k_multi_tc (the
+    // weighted row sums and column sums as u8 tensor-core products, multiround_tc.cuh) instead of k_multi
+    uint32_t multi_tc = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_MULTI_TC")) multi_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_DUAL")) dual = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
         if (const char *e = getenv("BZK_SMALL")) small = atoi(e) ? 1 : 0;
@@ -241,9 +245,28 @@ std::vector<std::pair<uint32_t, uint32_t>> multi_passes(uint32_t k, uint32_t i0)
     return v;
 }
 
+// k_multi_tc for a pass of 3 rounds whose output has at least one 128-column tile
+bool multi_use_tc(uint32_t K, uint32_t m) { return knobs().multi_tc && m == 3 && K >= 10; }
+
+// k_multi_tc CTAs per proof: one resident CTA per SM, so >= 2 x 148 CTAs in all when the batch is
+// small, >= 4 tiles per CTA, and <= 2^16 tiles per CTA (its TMEM column byte sums stay < 2^31)
+uint32_t multi_tc_ctas(uint64_t Ny, uint64_t nb) {
+    const uint64_t T = Ny / kTcTileRows;
+    // BZK_TC_CTAS (tests): force the CTAs per proof, clamped to [1, tiles] (ragged tile counts per CTA)
+    if (const char *e = getenv("BZK_TC_CTAS")) return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(T, atoi(e)));
+    uint64_t c = (2 * kSMs + nb - 1) / nb;
+    c = std::min<uint64_t>(c, std::max<uint64_t>(1, T / 4));
+    c = std::max<uint64_t>(c, (T + 65535) / 65536);
+    return (uint32_t)c;
+}
+
+uint32_t multi_pass_ctas(uint32_t K, uint32_t m, uint64_t nb) {
+    return multi_use_tc(K, m) ? multi_tc_ctas(1ull << (K - m), nb) : ctas_for(1ull << (K - m), nb);
+}
+
 uint32_t max_multi_ctas(uint32_t k, uint32_t i0, uint64_t nb) {
     uint32_t c = 1;
-    for (auto &pm : multi_passes(k, i0)) c = std::max(c, ctas_for(1ull << (pm.first - pm.second), nb));
+    for (auto &pm : multi_passes(k, i0)) c = std::max(c, multi_pass_ctas(pm.first, pm.second, nb));
     return c;
 }
 
@@ -456,6 +479,29 @@ bool make_row_map(CUtensorMap *tm, const void *base, uint64_t rows, uint32_t box
                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// k_multi_tc's tile map (multiround_tc.cuh): 32-byte rows (8 u32), 32-byte swizzle, 128 rows per box.
+// MSB: dims (8, Ny, 8 segments, B), one box = all 8 segments of a tile; LSB: dims (8, 8 entries of a
+// column, Ny, B), one box per segment.
+bool make_multi_tc_map(CUtensorMap *tm, uint32_t order, const void *base, uint64_t Ny, uint64_t stride,
+                       uint64_t nb) {
+    PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[4], strides[3];
+    cuuint32_t box[4], estr[4] = {1, 1, 1, 1};
+    if (order == 1) {
+        dims[0] = 8; dims[1] = Ny; dims[2] = 8; dims[3] = nb;
+        strides[0] = 32; strides[1] = Ny * 32; strides[2] = stride * 32;
+        box[0] = 8; box[1] = kTcTileRows; box[2] = 8; box[3] = 1;
+    } else {
+        dims[0] = 8; dims[1] = 8; dims[2] = Ny; dims[3] = nb;
+        strides[0] = 32; strides[1] = 256; strides[2] = stride * 32;
+        box[0] = 8; box[1] = 1; box[2] = kTcTileRows; box[3] = 1;
+    }
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, const_cast<void *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 cudaError_t dispatch_tail(uint32_t D, uint32_t order, uint32_t grid, size_t smem, cudaStream_t s,
                           const TailParams &p) {
     switch (D) {
@@ -623,18 +669,21 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
             else if (P.order == 1) { mp.dst = const_cast<fe *>(cur); mp.dst_stride = cur_stride; }
             else { mp.dst = (cur == bufX) ? bufY : bufX; mp.dst_stride = 1ull << (K - m); }
             mp.logK = K; mp.round0 = round; mp.k = k;
-            mp.ctas = ctas_for(1ull << (K - m), io.nb);
+            const bool use_tc = multi_use_tc(K, m);
+            mp.ctas = multi_pass_ctas(K, m, io.nb);
             mp.partials = part; mp.tickets = tick;
             mp.challenges = (const fe *)io.challenges; mp.round_evals = (fe *)io.round_evals;
             mp.claims = (fe *)io.claims;
             dim3 grid(mp.ctas, (uint32_t)io.nb);
             CUtensorMap tm;
             memset(&tm, 0, sizeof tm);
-            const bool tma = P.order == 1 && knobs().tma != 0;   // MSB: segment-wise TMA staging
+            const bool tma = !use_tc && P.order == 1 && knobs().tma != 0;   // MSB: segment-wise TMA staging
             if (tma && !make_row_map(&tm, mp.src, io.nb * cur_stride / 4, 8))
                 return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_multi)");
-            ProfScope ps_(ctx, s, 9);
-            cudaError_t e = multi_launch(P.order, m, tma, grid, s, mp, tm);
+            if (use_tc && !make_multi_tc_map(&tm, P.order, mp.src, 1ull << (K - m), cur_stride, io.nb))
+                return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_multi_tc)");
+            ProfScope ps_(ctx, s, use_tc ? 11 : 9);
+            cudaError_t e = use_tc ? multi_tc_launch(P.order, grid, s, mp, tm) : multi_launch(P.order, m, tma, grid, s, mp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_multi launch");
             cur = mp.dst; cur_stride = mp.dst_stride;

@@ -1,5 +1,6 @@
 // k_multi.cu -- instantiations of the known-challenge multi-round pass (multiround.cuh, NEXT-1)
 #include "multiround.cuh"
+#include "multiround_tc.cuh"
 
 namespace bzk {
 
@@ -23,7 +24,15 @@ cudaError_t multi_launch(uint32_t order, uint32_t m, bool tma, dim3 grid, cudaSt
     return tma ? multi_launch_o<1, true>(m, grid, s, p, tm) : multi_launch_o<1, false>(m, grid, s, p, tm);
 }
 
+cudaError_t multi_tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const MultiParams &p, const CUtensorMap &tm) {
+    if (order == 1) k_multi_tc<1><<<grid, kTcThreads, kTcSmem, s>>>(p, tm);
+    else k_multi_tc<0><<<grid, kTcThreads, kTcSmem, s>>>(p, tm);
+    return cudaGetLastError();
+}
+
 cudaError_t multi_set_attrs() {
+    cudaFuncSetAttribute(k_multi_tc<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcSmem);
+    cudaFuncSetAttribute(k_multi_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcSmem);
     cudaFuncSetAttribute(k_multi<1, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<1>());
     cudaFuncSetAttribute(k_multi<1, 2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<2>());
     return cudaFuncSetAttribute(k_multi<1, 3, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -43,6 +43,60 @@ struct MultiParams {
     fe *claims;           // [Bw] (may be null)
 };
 
+// The pass's round sums from the proof's column sums C_z (one thread): Alg. 1 lines 3-4 for the M
+// rounds, pi_i1 / pi_i2 = sum over z with bit_i(z) = 0 / 1 of w_{<i}(z) C_z (header comment); the
+// claim of round 1 is pi_11 + pi_12.  s_r holds r_i R and (1 - r_i) R.  (Inlined: as a separate call
+// it produced wrong sums inside the kernels with dynamic shared memory -- B200 bring-up of k_multi_tc.)
+template <int ORDER, int M>
+__device__ __forceinline__ void multi_evals(const MultiParams &P, uint32_t b, const fe (&cs)[1 << M], const fe (&s_r)[M][2]) {
+    constexpr int Z = 1 << M;
+    fe *ev = P.round_evals + ((size_t)b * P.k + (P.round0 - 1)) * 2;
+#pragma unroll 1
+    for (int i = 1; i <= M; ++i) {
+        fe g[2] = {fe_zero(), fe_zero()};
+#pragma unroll 1
+        for (int z = 0; z < Z; ++z) {
+            fe c = fe_const(1);                           // w_{<i}(z) R
+            for (int l = 1; l < i; ++l) {
+                const int bit = ORDER == 1 ? (z >> (M - l)) & 1 : (z >> (l - 1)) & 1;
+                c = mont_mul(c, s_r[l - 1][bit]);
+            }
+            const int bi = ORDER == 1 ? (z >> (M - i)) & 1 : (z >> (i - 1)) & 1;
+            g[bi] = fe_add(g[bi], mont_mul(cs[z], c));
+        }
+        st_fe(ev + 2 * (i - 1), g[0]);
+        st_fe(ev + 2 * (i - 1) + 1, g[1]);
+        if (P.round0 == 1 && i == 1 && P.claims) st_fe(P.claims + b, fe_add(g[0], g[1]));
+    }
+}
+
+// Pass setup shared by k_multi and k_multi_tc: s_r[i] = (r_i R, (1 - r_i) R) for the pass's rounds
+// (threads < M), then s_w[z] = w(z) 2^288 mod p (threads < 2^M; acc17_to_fe_288 divides by 2^288).
+template <int ORDER, int M>
+__device__ __forceinline__ void multi_weights(const MultiParams &P, uint32_t b, fe (&s_r)[M][2], fe (&s_w)[1 << M]) {
+    const fe *chal = P.challenges + (size_t)b * P.k + (P.round0 - 1);
+    if (threadIdx.x < M) {
+        const fe r = ld_fe(chal + threadIdx.x);
+        s_r[threadIdx.x][1] = mont_mul(r, fe_const(2));                          // r R
+        fe one = fe_zero();
+        one.l[0] = 1;
+        s_r[threadIdx.x][0] = mont_mul(fe_sub(one, r), fe_const(2));              // (1 - r) R
+    }
+    __syncthreads();
+    if (threadIdx.x < (1u << M)) {
+        fe w = fe_const(1);                                                       // R = 1 in Montgomery form
+#pragma unroll
+        for (int i = 1; i <= M; ++i) {
+            const int bit = ORDER == 1 ? (threadIdx.x >> (M - i)) & 1 : (threadIdx.x >> (i - 1)) & 1;
+            w = mont_mul(w, s_r[i - 1][bit]);
+        }
+        fe c288 = fe_const(1);                                                    // 2^256 mod p
+        for (int e = 0; e < 32; ++e) c288 = fe_add(c288, c288);                 // 2^288 mod p
+        s_w[threadIdx.x] = mont_mul(w, c288);                                     // (w R) 2^288 / R = w 2^288
+    }
+    __syncthreads();
+}
+
 // TMA = true (MSB only): the warp's 32 columns are streamed into shared memory segment by segment --
 // segment z holds entry z of the 32 columns, the 1 KiB A[y0 + z 2^(K-M) .. + 31] -- and each segment's
 // copy for the next grid-stride block is issued as soon as every lane has consumed it (sumcheck.cuh
@@ -55,27 +109,7 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P, const __grid_co
     __shared__ fe s_red[32 * Z];
     __shared__ int s_last;
     const uint32_t b = blockIdx.y;
-    const fe *chal = P.challenges + (size_t)b * P.k + (P.round0 - 1);
-    if (threadIdx.x < M) {
-        const fe r = ld_fe(chal + threadIdx.x);
-        s_r[threadIdx.x][1] = mont_mul(r, fe_const(2));                          // r R
-        fe one = fe_zero();
-        one.l[0] = 1;
-        s_r[threadIdx.x][0] = mont_mul(fe_sub(one, r), fe_const(2));              // (1 - r) R
-    }
-    __syncthreads();
-    if (threadIdx.x < Z) {
-        fe w = fe_const(1);                                                       // R = 1 in Montgomery form
-#pragma unroll
-        for (int i = 1; i <= M; ++i) {
-            const int bit = ORDER == 1 ? (threadIdx.x >> (M - i)) & 1 : (threadIdx.x >> (i - 1)) & 1;
-            w = mont_mul(w, s_r[i - 1][bit]);
-        }
-        fe c288 = fe_const(1);                                                    // 2^256 mod p
-        for (int e = 0; e < 32; ++e) c288 = fe_add(c288, c288);                 // 2^288 mod p
-        s_w[threadIdx.x] = mont_mul(w, c288);                                     // (w R) 2^288 / R = w 2^288
-    }
-    __syncthreads();
+    multi_weights<ORDER, M>(P, b, s_r, s_w);
 
     const uint64_t Ny = 1ull << (P.logK - M);         // outputs (columns) per proof
     const fe *src = P.src + (size_t)b * P.src_stride;
@@ -167,29 +201,15 @@ __global__ void __launch_bounds__(256, 2) k_multi(MultiParams P, const __grid_co
     }
     if (threadIdx.x != 0) return;
     if (P.ctas > 1) P.tickets[b] = 0;
-    fe *ev = P.round_evals + ((size_t)b * P.k + (P.round0 - 1)) * 2;
-#pragma unroll 1
-    for (int i = 1; i <= M; ++i) {
-        fe g[2] = {fe_zero(), fe_zero()};
-#pragma unroll 1
-        for (int z = 0; z < Z; ++z) {
-            fe c = fe_const(1);                           // w_{<i}(z) R
-            for (int l = 1; l < i; ++l) {
-                const int bit = ORDER == 1 ? (z >> (M - l)) & 1 : (z >> (l - 1)) & 1;
-                c = mont_mul(c, s_r[l - 1][bit]);
-            }
-            const int bi = ORDER == 1 ? (z >> (M - i)) & 1 : (z >> (i - 1)) & 1;
-            g[bi] = fe_add(g[bi], mont_mul(cs[z], c));
-        }
-        st_fe(ev + 2 * (i - 1), g[0]);
-        st_fe(ev + 2 * (i - 1) + 1, g[1]);
-        if (P.round0 == 1 && i == 1 && P.claims) st_fe(P.claims + b, fe_add(g[0], g[1]));
-    }
+    multi_evals<ORDER, M>(P, b, cs, s_r);
 }
 
 // k_multi.cu
 cudaError_t multi_launch(uint32_t order, uint32_t m, bool tma, dim3 grid, cudaStream_t s, const MultiParams &p,
                          const CUtensorMap &tm);
 cudaError_t multi_set_attrs();
+// k_multi_tc (multiround_tc.cuh): three rounds per pass, 128-column tiles, tensor-core row sums
+constexpr uint32_t kTcTileRows = 128;   // columns y per tile (the MMA's M)
+cudaError_t multi_tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const MultiParams &p, const CUtensorMap &tm);
 
 }  // namespace bzk

@@ -134,3 +134,69 @@ def test_m0lit_full_size(orc):
         for j in range(1, k):
             prev = (g[j - 1][0] + rr[j - 1] * (g[j - 1][1] - g[j - 1][0])) % P
             assert (g[j][0] + g[j][1]) % P == prev, (i, j)
+
+
+@pytest.mark.parametrize("order", [0, 1])
+@pytest.mark.parametrize("k,B", [(16, 1), (16, 3), (17, 2)])
+def test_multiround_tc_extremes(orc, order, k, B):
+    """k_multi_tc (tensor-core passes, csrc/multiround_tc.cuh) at the byte extremes: every entry p - 1
+    (all bytes near 255, the largest column values c_n and column byte sums), alternating 0 / p - 1,
+    and r in {0, 1, p - 1}; the profile shows the tensor-core kernel ran (k >= 16: too large for k_small)."""
+    N = 1 << k
+    pm1 = np.array(inputs.P_BN254, dtype=np.uint64).copy()
+    pm1[0] -= 1
+    host = np.zeros((B, 1, N, 4), dtype=np.uint64)
+    host[0, 0, :] = pm1
+    if B > 1:
+        host[1, 0, 1::2] = pm1
+    if B > 2:
+        host[2, 0, :] = inputs.gen_tables(1, 1, k, first_index=77, dist="adversarial")[0, 0]
+    t = torch.from_numpy(host.view(np.int64)).cuda()
+    r = challenges(orc, B, k, 31 + k, edge=True)
+    p = bzk.Prover(0)
+    bzk.bzk_profile_enable(p.ctx, 1)
+    out = run(p, t, k, order, r, flags=bzk.BZK_F_PRESERVE_INPUT)
+    prof = bzk.bzk_profile_read(p.ctx, 1)
+    p.close()
+    assert prof["multi_round_tc"][1] > 0, prof
+    for b in range(B):
+        ref = orc.prove_given(host[b], k, 1, order, r[b])
+        for key in KEYS:
+            assert np.array_equal(np64(out[key][b]).reshape(ref[key].shape), ref[key]), (key, b)
+
+
+TC_SCRIPT = r"""
+import sys, numpy as np, torch
+sys.path.insert(0, {root!r}); sys.path.insert(0, {root!r} + "/tests")
+import oracle
+from paper_conf_asplos_lucw0cz25_b200 import bzk
+from test_gpu_multiround import challenges, run, np64, KEYS
+oracle.build()
+for k, B, order in [(16, 2, 0), (16, 1, 1), (17, 1, 0)]:
+    t = torch.empty((B, 1, 1 << k, 4), dtype=torch.int64, device="cuda")
+    bzk.bzk_generate(t, B, 1, k, 500 + k, "adversarial")
+    r = challenges(oracle, B, k, 7 * k)
+    p = bzk.Prover(0)
+    out = run(p, t, k, order, r, first_index=500 + k, flags=bzk.BZK_F_PRESERVE_INPUT)
+    p.close()
+    host = np64(t)
+    for b in range(B):
+        ref = oracle.prove_given(host[b], k, 1, order, r[b])
+        for key in KEYS:
+            assert np.array_equal(np64(out[key][b]).reshape(ref[key].shape), ref[key]), (key, b, k, order)
+print("tc ok")
+"""
+
+
+@pytest.mark.parametrize("env", [{"BZK_TC_CTAS": "1"}, {"BZK_TC_CTAS": "7"}, {"BZK_TC_CTAS": "1000"},
+                                 {"BZK_MULTI_TC": "0"}])
+def test_multiround_tc_launch_shapes(env):
+    """k_multi_tc with one CTA per proof, 7 CTAs (ragged: 64 tiles -> 10 / 9 per CTA, last-CTA ticket), one
+    CTA per tile, and the CUDA-core k_multi instead (BZK_MULTI_TC=0); k_small off so every case runs the passes."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", TC_SCRIPT.format(root=root)], env=dict(os.environ, BZK_SMALL="0", **env),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "tc ok" in r.stdout, r.stdout + r.stderr
