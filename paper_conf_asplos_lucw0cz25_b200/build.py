@@ -14,7 +14,7 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 OBJ = os.environ.get("BZK_BUILD_DIR", os.path.join(HERE, "build"))
 LIB = os.environ.get("BZK_LIB_OUT", os.path.join(HERE, "libbzk.so"))
-SOURCES = ["api.cu", "k_d1.cu", "k_d2.cu", "k_d3.cu", "k_d4.cu", "k_gl.cu", "k_merkle.cu", "k_enc.cu", "k_multi.cu"]
+SOURCES = ["api.cu", "k_d1.cu", "k_d2.cu", "k_d3.cu", "k_d4.cu", "k_gl.cu", "k_merkle.cu", "k_enc.cu", "k_multi.cu", "k_r1tc.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-I", os.path.join(ROOT, "include")] + os.environ.get("BZK_NVCC_EXTRA", "").split()

@@ -191,7 +191,11 @@ struct Knobs {
     // BZK_MULTI_TC=0/1: three-round known-challenge passes over >= 2^10 entries run k_multi_tc (the
     // weighted row sums and column sums as u8 tensor-core products, multiround_tc.cuh) instead of k_multi
     uint32_t multi_tc = 1;
+    // BZK_R1_TC=0/1: round 1 of d = 2 BN254 proofs runs k_round1_tc (the three product sums as u8
+    // tensor-core products over the pairs, round1_tc.cuh) instead of k_round<2, ., FIRST>
+    uint32_t r1tc = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_R1_TC")) r1tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_TC")) multi_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_DUAL")) dual = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_CHAIN_CHUNKS")) chain_chunks = std::max(1, atoi(e));
@@ -257,6 +261,19 @@ uint32_t multi_tc_ctas(uint64_t Ny, uint64_t nb) {
     uint64_t c = (2 * kSMs + nb - 1) / nb;
     c = std::min<uint64_t>(c, std::max<uint64_t>(1, T / 4));
     c = std::max<uint64_t>(c, (T + 65535) / 65536);
+    return (uint32_t)c;
+}
+
+// k_round1_tc (d = 2 round 1): one resident CTA per SM, >= 2 x 148 CTAs in all when the batch is small,
+// >= 8 tiles of 128 pairs per CTA, <= 2^21 pairs per CTA (its 64-bit anti-diagonal sums stay < 2^43)
+bool r1_use_tc(uint32_t D, uint64_t h) { return knobs().r1tc && D == 2 && h >= 128; }
+uint32_t r1tc_ctas(uint64_t h, uint64_t nb) {
+    const uint64_t T = h / 128;
+    // BZK_R1TC_CTAS (tests): force the CTAs per proof, clamped to [1, tiles] (ragged tile counts per CTA)
+    if (const char *e = getenv("BZK_R1TC_CTAS")) return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(T, atoi(e)));
+    uint64_t c = (2 * kSMs + nb - 1) / nb;
+    c = std::min<uint64_t>(c, std::max<uint64_t>(1, T / 8));
+    c = std::max<uint64_t>(c, (h + (1ull << 21) - 1) >> 21);
     return (uint32_t)c;
 }
 
@@ -482,6 +499,28 @@ bool make_row_map(CUtensorMap *tm, const void *base, uint64_t rows, uint32_t box
 // k_multi_tc's tile map (multiround_tc.cuh): 32-byte rows (8 u32), 32-byte swizzle, 128 rows per box.
 // MSB: dims (8, Ny, 8 segments, B), one box = all 8 segments of a tile; LSB: dims (8, 8 entries of a
 // column, Ny, B), one box per segment.
+// k_round1_tc's map over the wave's round-1 tables ([tables][2h] entries of 32 bytes): 32-byte rows,
+// 32-byte swizzle, 128 pairs per box.  MSB (a = j, b = j + h): dims (8, h, 2, tables), one box holds
+// a table's a and b tiles; LSB (a = 2j, b = 2j + 1): dims (8, 2, h, tables), one box per tile.
+bool make_r1_map(CUtensorMap *tm, uint32_t order, const void *base, uint64_t h, uint64_t tables) {
+    PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
+    if (!enc) return false;
+    cuuint64_t dims[4], strides[3];
+    cuuint32_t box[4], estr[4] = {1, 1, 1, 1};
+    if (order == 1) {
+        dims[0] = 8; dims[1] = h; dims[2] = 2; dims[3] = tables;
+        strides[0] = 32; strides[1] = h * 32; strides[2] = 2 * h * 32;
+        box[0] = 8; box[1] = 128; box[2] = 2; box[3] = 1;
+    } else {
+        dims[0] = 8; dims[1] = 2; dims[2] = h; dims[3] = tables;
+        strides[0] = 32; strides[1] = 64; strides[2] = 2 * h * 32;
+        box[0] = 8; box[1] = 1; box[2] = 128; box[3] = 1;
+    }
+    return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, const_cast<void *>(base), dims, strides, box, estr,
+               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 bool make_multi_tc_map(CUtensorMap *tm, uint32_t order, const void *base, uint64_t Ny, uint64_t stride,
                        uint64_t nb) {
     PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
@@ -711,7 +750,14 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         }
         CUtensorMap tm;
         memset(&tm, 0, sizeof tm);
-        rp.tma = knobs().tma_for(D, i == 1);
+        const bool r1tc = i == 1 && r1_use_tc(D, h);
+        if (r1tc) {
+            rp.ctas = std::min(r1tc_ctas(h, io.nb), P.cmax);
+            rp.cluster = 1;
+            if (!make_r1_map(&tm, P.order, tab, h, io.nb * D))
+                return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_round1_tc)");
+        }
+        rp.tma = r1tc ? 0 : knobs().tma_for(D, i == 1);
         if (rp.tma) {
             const uint64_t E = i == 1 ? 2 : 4;   // raw entries per pair and table
             const uint32_t box = P.order == 0 ? (uint32_t)(E * 8) : 8u;
@@ -721,7 +767,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-            cudaError_t e = dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
+            cudaError_t e = r1tc ? r1tc_launch(P.order, grid, s, rp, tm) : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
         }
@@ -1808,6 +1854,7 @@ bzk_status bzk_create(int device, size_t workspace_limit, bzk_ctx **out) {
         set_kernel_attrs<4>();
         gl_set_attrs();
         multi_set_attrs();
+        r1tc_set_attrs();
         k_init_consts<<<1, 32, 0, ctx->copy_stream>>>(ctx->consts);
         ok = cudaStreamSynchronize(ctx->copy_stream) == cudaSuccess;
     }

@@ -1,5 +1,6 @@
 // k_multi.cu -- instantiations of the known-challenge multi-round pass (multiround.cuh, NEXT-1)
 #include "multiround.cuh"
+#include <stdlib.h>
 #include "multiround_tc.cuh"
 
 namespace bzk {
@@ -24,15 +25,33 @@ cudaError_t multi_launch(uint32_t order, uint32_t m, bool tma, dim3 grid, cudaSt
     return tma ? multi_launch_o<1, true>(m, grid, s, p, tm) : multi_launch_o<1, false>(m, grid, s, p, tm);
 }
 
+// k_multi_tc launch shapes (NS stages, EG epilogue groups, CM rows of the column-sum product);
+// BZK_TC_CFG=i picks one for A/B sweeps, default 0
+#define BZK_TC_SHAPES(X) X(4, 2, 128) X(4, 2, 64) X(6, 2, 64) X(4, 4, 64) X(6, 4, 64) X(6, 3, 64)
+static int tc_cfg() {
+    static int c = [] { const char *e = getenv("BZK_TC_CFG"); return e ? atoi(e) : 0; }();
+    return c;
+}
+
 cudaError_t multi_tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const MultiParams &p, const CUtensorMap &tm) {
-    if (order == 1) k_multi_tc<1><<<grid, kTcThreads, kTcSmem, s>>>(p, tm);
-    else k_multi_tc<0><<<grid, kTcThreads, kTcSmem, s>>>(p, tm);
-    return cudaGetLastError();
+    int i = 0;
+#define BZK_TC_LAUNCH(NS, EG, CM)                                                                        \
+    if (tc_cfg() == i++) {                                                                              \
+        if (order == 1) k_multi_tc<1, NS, EG, CM><<<grid, tc_threads(EG), tc_smem(NS), s>>>(p, tm);       \
+        else k_multi_tc<0, NS, EG, CM><<<grid, tc_threads(EG), tc_smem(NS), s>>>(p, tm);                   \
+        return cudaGetLastError();                                                                      \
+    }
+    BZK_TC_SHAPES(BZK_TC_LAUNCH)
+#undef BZK_TC_LAUNCH
+    return cudaErrorInvalidValue;
 }
 
 cudaError_t multi_set_attrs() {
-    cudaFuncSetAttribute(k_multi_tc<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcSmem);
-    cudaFuncSetAttribute(k_multi_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTcSmem);
+#define BZK_TC_ATTR(NS, EG, CM)                                                                                   \
+    cudaFuncSetAttribute(k_multi_tc<0, NS, EG, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem(NS)); \
+    cudaFuncSetAttribute(k_multi_tc<1, NS, EG, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tc_smem(NS));
+    BZK_TC_SHAPES(BZK_TC_ATTR)
+#undef BZK_TC_ATTR
     cudaFuncSetAttribute(k_multi<1, 1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<1>());
     cudaFuncSetAttribute(k_multi<1, 2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)multi_tma_smem<2>());
     return cudaFuncSetAttribute(k_multi<1, 3, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

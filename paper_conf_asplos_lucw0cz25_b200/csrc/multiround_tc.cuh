@@ -16,9 +16,9 @@
 // sum_i D2[(z,i)] 2^(8i).  So the integer pipe does ~30 operations per entry instead of a 256 x 256-bit
 // product, and the pass streams at the HBM rate.
 //
-// Roles (one CTA per SM, 320 threads): warp 0 issues the TMA loads (one 32 KiB stage = the 8
+// Roles (one CTA per SM, 64 + 128 EG threads): warp 0 issues the TMA loads (one 32 KiB stage = the 8
 // segments of 128 entries, 32-byte rows, 32-byte swizzle), warp 1 owns TMEM and issues the MMAs,
-// warps 2..9 are two epilogue groups of four warps (group g takes the tiles it = g mod 2 and TMEM
+// warps 2.. are EG epilogue groups of four warps (group g takes the tiles it = g mod EG and TMEM
 // accumulator g; warp w reads TMEM lanes 32 (w mod 4) ..).  MSB folds in place as k_multi does: the
 // output row y overwrites A[y + 0 Ny], which only this CTA's tile y reads, and only before.
 #pragma once
@@ -28,17 +28,20 @@
 
 namespace bzk {
 
-constexpr int kTcStages = 4;                                   // 32 KiB TMA stages
-constexpr int kTcThreads = 64 + 2 * 128;                       // TMA warp, MMA warp, 2 epilogue groups
-constexpr size_t kTcSmem = 1024 + (size_t)kTcStages * 32768 + 16384 + 4096;   // + B operand + ones
+// NS: 32 KiB TMA stages; EG: epilogue groups of 4 warps (one 64-column TMEM accumulator each, <= 4);
+// CM: M of the column-sum product (64 or 128 rows of ones: every row of D2 is the same vector, row 0
+// sits in TMEM lane 0 either way)
+constexpr int tc_threads(int EG) { return 64 + 128 * EG; }
+constexpr size_t tc_smem(int NS) { return 1024 + (size_t)NS * 32768 + 16384 + 4096; }   // + B operand + ones
 
-template <int ORDER>
-__global__ void __launch_bounds__(kTcThreads, 1) k_multi_tc(MultiParams P, const __grid_constant__ CUtensorMap tmap) {
-    constexpr int M = 3, Z = 8;
+template <int ORDER, int NS, int EG, int CM>
+__global__ void __launch_bounds__(tc_threads(EG), 1) k_multi_tc(MultiParams P, const __grid_constant__ CUtensorMap tmap) {
+    static_assert(EG >= 1 && EG <= 4 && (CM == 64 || CM == 128), "k_multi_tc shape");
+    constexpr int M = 3, Z = 8, kTcStages = NS;
     __shared__ fe s_w[Z];
     __shared__ fe s_r[M][2];
     __shared__ fe s_cs[Z];
-    __shared__ __align__(8) uint64_t full[kTcStages], empty[kTcStages], tfull[2], tempty[2], dfin;
+    __shared__ __align__(8) uint64_t full[kTcStages], empty[kTcStages], tfull[EG], tempty[EG], dfin;
     __shared__ uint32_t s_tmem;
     __shared__ int s_last;
     extern __shared__ uint8_t tc_raw[];
@@ -70,7 +73,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_multi_tc(MultiParams P, const
         *reinterpret_cast<uint4 *>(ones + c * 16) = make_uint4(0x01010101u, 0x01010101u, 0x01010101u, 0x01010101u);
     if (threadIdx.x == 0) {
         for (int s = 0; s < kTcStages; ++s) { tc::mbar_init_n(&full[s], 1); tc::mbar_init_n(&empty[s], 1); }
-        for (int g = 0; g < 2; ++g) { tc::mbar_init_n(&tfull[g], 1); tc::mbar_init_n(&tempty[g], 128); }
+        for (int g = 0; g < EG; ++g) { tc::mbar_init_n(&tfull[g], 1); tc::mbar_init_n(&tempty[g], 128); }
         tc::mbar_init_n(&dfin, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -103,12 +106,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_multi_tc(MultiParams P, const
         }
     } else if (warp == 1) {
         if (lane == 0) {
-            const uint32_t id_main = tc::idesc_u8(128, 64, false), id_col = tc::idesc_u8(128, 256, true);
+            const uint32_t id_main = tc::idesc_u8(128, 64, false), id_col = tc::idesc_u8(CM, 256, true);
             const uint32_t sb = tc::su32(stage0), bb = tc::su32(opB), ob = tc::su32(ones);
             for (uint32_t it = 0; it < nt; ++it) {
-                const uint32_t s = it % kTcStages, g = it & 1;
+                const uint32_t s = it % kTcStages, g = it % EG;
                 tc::mbar_wait(&full[s], (it / kTcStages) & 1);
-                if (it >= 2) tc::mbar_wait(&tempty[g], ((it >> 1) - 1) & 1);
+                if (it >= (uint32_t)EG) tc::mbar_wait(&tempty[g], ((it / EG) - 1) & 1);
                 tc::fence_after();
                 const uint32_t a0 = sb + s * 32768;
 #pragma unroll
@@ -129,8 +132,8 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_multi_tc(MultiParams P, const
         const uint32_t e = warp - 2, g = e >> 2, qd = warp & 3, row = qd * 32 + lane;
         const uint32_t ta = tmem + ((qd * 32) << 16) + g * 64;
         fe *dst = P.dst + (size_t)b * P.dst_stride;
-        for (uint32_t it = g; it < nt; it += 2) {
-            tc::mbar_wait(&tfull[g], (it >> 1) & 1);
+        for (uint32_t it = g; it < nt; it += EG) {
+            tc::mbar_wait(&tfull[g], (it / EG) & 1);
             tc::fence_after();
             uint32_t c0[32], c1[32];
             tc::ld_x32(ta, c0);

@@ -581,6 +581,82 @@ __device__ __forceinline__ fe tma_entry(const uint8_t *slot, uint32_t lane, int 
     return r;
 }
 
+// End of a global round kernel, every thread of the CTA: the CTA's sums (acc, per thread) are
+// reduced; one partial per CTA (or per thread-block cluster, through DSMEM) goes through the
+// last-CTA ticket; the proof's last CTA finalises the round (transcript, r_i, outputs, next claim).
+template <int D, bool DERIVE>
+__device__ __forceinline__ void round_finish(const RoundParams &P, uint32_t b, fe (&acc)[Pts<D, DERIVE>::NV], fe *s_red,
+                                             fe *s_clu, int *s_last_p) {
+    constexpr int NV = Pts<D, DERIVE>::NV;
+    int &s_last = *s_last_p;
+    block_reduce<NV>(acc, s_red);
+    fe *evals = P.round_evals + (size_t)b * P.k * (D + 1);
+    fe *chals = P.challenges + (size_t)b * P.k;
+    fe *claim = P.claims ? P.claims + b : nullptr;
+    __shared__ fe s_g[D + 1];
+    __shared__ fe s_rm;
+    if (P.ctas == 1) {
+        if (threadIdx.x < 32) {
+            if (threadIdx.x == 0)
+                finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
+            __syncwarp();
+            const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
+            if (threadIdx.x == 0) P.ps[b].claim = c;
+        }
+        return;
+    }
+    // Thread-block cluster (launched with cluster dims (cs, 1, 1), cs <= 8, all CTAs of one proof):
+    // the cluster's CTA sums are combined through distributed shared memory, so only one partial
+    // per cluster goes to global memory and through the last-CTA ticket.
+    namespace cg = cooperative_groups;
+    cg::cluster_group cluster = cg::this_cluster();
+    const uint32_t cs = cluster.num_blocks();
+    if (cs > 1) {
+        if (threadIdx.x == 0)
+#pragma unroll
+            for (int t = 0; t < NV; ++t) s_clu[t] = acc[t];
+        cluster.sync();
+        const bool leader = cluster.block_rank() == 0;
+        if (leader && threadIdx.x == 0) {
+            for (uint32_t r = 1; r < cs; ++r) {
+                const fe *rem = cluster.map_shared_rank(s_clu, r);
+#pragma unroll
+                for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], rem[t]);
+            }
+        }
+        cluster.sync();   // remote shared memory must outlive the leader's reads
+        if (!leader) return;
+    }
+    const uint32_t nparts = P.ctas / cs, pidx = blockIdx.x / cs;
+    fe *part = P.partials + (size_t)b * P.ctas * NV;
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int t = 0; t < NV; ++t) st_fe_cg(&part[(size_t)pidx * NV + t], acc[t]);
+        __threadfence();
+        uint32_t old = atomicAdd(&P.tickets[b], 1u);
+        s_last = (old == nparts - 1);
+    }
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    // last CTA of proof b: cooperative sum of all partials
+#pragma unroll
+    for (int t = 0; t < NV; ++t) acc[t] = fe_zero();
+    for (uint32_t c = threadIdx.x; c < nparts; c += blockDim.x)
+#pragma unroll
+        for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], ld_fe_cg(&part[(size_t)c * NV + t]));
+    block_reduce<NV>(acc, s_red);
+    if (threadIdx.x < 32) {
+        if (threadIdx.x == 0) {
+            P.tickets[b] = 0;
+            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
+        }
+        __syncwarp();
+        const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
+        if (threadIdx.x == 0) P.ps[b].claim = c;
+    }
+}
+
 template <int D, int ORDER, bool FIRST, bool TMA>
 __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
     k_round(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
@@ -711,72 +787,7 @@ __global__ void __launch_bounds__(BZK_RT, (D <= 2 ? BZK_ROUND_OCC : 1))
     fe acc[NV];
 #pragma unroll
     for (int t = 0; t < NV; ++t) acc[t] = acc9_to_fe(wacc[t]);
-    block_reduce<NV>(acc, s_red);
-    fe *evals = P.round_evals + (size_t)b * P.k * (D + 1);
-    fe *chals = P.challenges + (size_t)b * P.k;
-    fe *claim = P.claims ? P.claims + b : nullptr;
-    __shared__ fe s_g[D + 1];
-    __shared__ fe s_rm;
-    if (P.ctas == 1) {
-        if (threadIdx.x < 32) {
-            if (threadIdx.x == 0)
-                finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
-            __syncwarp();
-            const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
-            if (threadIdx.x == 0) P.ps[b].claim = c;
-        }
-        return;
-    }
-    // Thread-block cluster (launched with cluster dims (cs, 1, 1), cs <= 8, all CTAs of one proof):
-    // the cluster's CTA sums are combined through distributed shared memory, so only one partial
-    // per cluster goes to global memory and through the last-CTA ticket.
-    namespace cg = cooperative_groups;
-    cg::cluster_group cluster = cg::this_cluster();
-    const uint32_t cs = cluster.num_blocks();
-    if (cs > 1) {
-        if (threadIdx.x == 0)
-#pragma unroll
-            for (int t = 0; t < NV; ++t) s_clu[t] = acc[t];
-        cluster.sync();
-        const bool leader = cluster.block_rank() == 0;
-        if (leader && threadIdx.x == 0) {
-            for (uint32_t r = 1; r < cs; ++r) {
-                const fe *rem = cluster.map_shared_rank(s_clu, r);
-#pragma unroll
-                for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], rem[t]);
-            }
-        }
-        cluster.sync();   // remote shared memory must outlive the leader's reads
-        if (!leader) return;
-    }
-    const uint32_t nparts = P.ctas / cs, pidx = blockIdx.x / cs;
-    fe *part = P.partials + (size_t)b * P.ctas * NV;
-    if (threadIdx.x == 0) {
-#pragma unroll
-        for (int t = 0; t < NV; ++t) st_fe_cg(&part[(size_t)pidx * NV + t], acc[t]);
-        __threadfence();
-        uint32_t old = atomicAdd(&P.tickets[b], 1u);
-        s_last = (old == nparts - 1);
-    }
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    // last CTA of proof b: cooperative sum of all partials
-#pragma unroll
-    for (int t = 0; t < NV; ++t) acc[t] = fe_zero();
-    for (uint32_t c = threadIdx.x; c < nparts; c += blockDim.x)
-#pragma unroll
-        for (int t = 0; t < NV; ++t) acc[t] = fe_add(acc[t], ld_fe_cg(&part[(size_t)c * NV + t]));
-    block_reduce<NV>(acc, s_red);
-    if (threadIdx.x < 32) {
-        if (threadIdx.x == 0) {
-            P.tickets[b] = 0;
-            finalize_round<D, DERIVE ? 2 : 1>(acc, P.round, P.ps[b], evals, chals, claim, &s_rm, s_g, P.given);
-        }
-        __syncwarp();
-        const fe c = lagrange_warp<D>(s_g, s_rm, P.consts);
-        if (threadIdx.x == 0) P.ps[b].claim = c;
-    }
+    round_finish<D, DERIVE>(P, b, acc, s_red, s_clu, &s_last);
 }
 
 // ---------------------------------------------------------------- on-chip tail
@@ -904,5 +915,8 @@ cudaError_t launch_tail(uint32_t order, uint32_t grid, uint32_t threads, size_t 
                         const TailParams &p);
 template <int D>
 cudaError_t set_kernel_attrs();   // once per process, before any launch or graph capture
+// k_round1_tc (round1_tc.cuh, k_r1tc.cu): d = 2 round 1 on the tensor cores
+cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm);
+cudaError_t r1tc_set_attrs();
 
 }  // namespace bzk
