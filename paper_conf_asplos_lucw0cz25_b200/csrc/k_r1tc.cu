@@ -1,17 +1,35 @@
 // k_r1tc.cu -- instantiations of the tensor-core round-1 kernel for d = 2 (round1_tc.cuh)
+#include <stdlib.h>
 #include "round1_tc.cuh"
 
 namespace bzk {
 
+// launch shape: 6 stages, 4 D-prep warps.  Sweep on B200 (c2 round 1 per step, profiles/r02/
+// bench_c2_r1cfg*_r02r1s.json): (6, 2) 14.6 ms, (8, 2) 15.2, (6, 4) 11.6, (8, 4) 11.7 -- the D = b + p - a
+// pass sits on every stage's critical path, so its width matters and the stage count does not.
+#define BZK_R1_SHAPES(X) X(6, 4)
+static int r1_cfg() { return 0; }
+
 cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
-    if (order == 1) k_round1_tc<1><<<grid, kR1Threads, kR1Smem, s>>>(p, tm);
-    else k_round1_tc<0><<<grid, kR1Threads, kR1Smem, s>>>(p, tm);
-    return cudaGetLastError();
+    int i = 0;
+#define BZK_R1_LAUNCH(NS, PW)                                                                            \
+    if (r1_cfg() == i++) {                                                                              \
+        if (order == 1) k_round1_tc<1, NS, PW><<<grid, r1_threads(PW), r1_smem(NS), s>>>(p, tm);          \
+        else k_round1_tc<0, NS, PW><<<grid, r1_threads(PW), r1_smem(NS), s>>>(p, tm);                      \
+        return cudaGetLastError();                                                                      \
+    }
+    BZK_R1_SHAPES(BZK_R1_LAUNCH)
+#undef BZK_R1_LAUNCH
+    return cudaErrorInvalidValue;
 }
 
 cudaError_t r1tc_set_attrs() {
-    cudaFuncSetAttribute(k_round1_tc<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kR1Smem);
-    return cudaFuncSetAttribute(k_round1_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kR1Smem);
+#define BZK_R1_ATTR(NS, PW)                                                                                  \
+    cudaFuncSetAttribute(k_round1_tc<0, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS)); \
+    cudaFuncSetAttribute(k_round1_tc<1, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS));
+    BZK_R1_SHAPES(BZK_R1_ATTR)
+#undef BZK_R1_ATTR
+    return cudaGetLastError();
 }
 
 }  // namespace bzk

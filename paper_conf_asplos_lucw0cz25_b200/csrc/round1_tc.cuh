@@ -19,8 +19,8 @@
 // (< 2^544, 17 words), acc17_to_fe(S) = S R^-1 mod p -- the same canonical per-CTA partial k_round's
 // acc17 path produces -- then round_finish (ticket, transcript, r_1, outputs) as every global round.
 //
-// Roles (1 CTA per SM, 256 threads): warp 0 TMA (a and b tiles of both tables, 32-byte rows,
-// 32-byte swizzle), warp 1 TMEM + MMA issue, warps 2-3 form D = b + p - a in shared memory, warps 4-7
+// Roles (1 CTA per SM, 32 (6 + PW) threads): warp 0 TMA (a and b tiles of both tables, 32-byte rows,
+// 32-byte swizzle), warp 1 TMEM + MMA issue, PW warps form D = b + p - a in shared memory, the last 4 warps
 // the epilogue (warp w reads TMEM lanes 32 (w mod 4): rows 0..95 = the a, b, D blocks).
 #pragma once
 #include <stdint.h>
@@ -29,15 +29,17 @@
 
 namespace bzk {
 
-constexpr int kR1Stages = 6;                       // 24 KiB stages: [a0][b0][D0][a1][b1][D1] x 128 pairs
-constexpr int kR1Threads = 256;                    // 8 warps: TMA, MMA, 2 x D-prep, 4 x epilogue
+// NS: 24 KiB stages ([a0][b0][D0][a1][b1][D1] x 128 pairs); PW: D-prep warps (2 or 4)
 constexpr uint32_t kR1Tile = 128;                  // pairs per tile
 constexpr uint32_t kR1Chunk = 128;                 // tiles per TMEM accumulation chunk (16384 pairs)
-constexpr size_t kR1Smem = 1024 + (size_t)kR1Stages * 24576;
+constexpr int r1_threads(int PW) { return 32 * (2 + PW + 4); }
+constexpr size_t r1_smem(int NS) { return 1024 + (size_t)NS * 24576; }
 
-template <int ORDER>
-__global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
+template <int ORDER, int NS, int PW>
+__global__ void __launch_bounds__(r1_threads(PW), 1) k_round1_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
     constexpr int D = 2, NV = Pts<2, false>::NV;   // points 0, 1, inf
+    constexpr int kR1Stages = NS;
+    static_assert(PW == 2 || PW == 4, "D-prep warps");
     __shared__ fe s_red[32 * NV];
     __shared__ fe s_clu[NV];
     __shared__ int s_last;
@@ -55,7 +57,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
     if (threadIdx.x == 0) {
         for (int s = 0; s < kR1Stages; ++s) {
             tc::mbar_init_n(&full[s], 1);
-            tc::mbar_init_n(&prep[s], 64);
+            tc::mbar_init_n(&prep[s], 32 * PW);
             tc::mbar_init_n(&empty[s], 1);
         }
         for (int g = 0; g < 2; ++g) { tc::mbar_init_n(&dready[g], 1); tc::mbar_init_n(&dempty[g], 128); }
@@ -109,7 +111,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
             }
         }
         __syncwarp();
-    } else if (warp < 4) {
+    } else if (warp < 2 + PW) {
         // D = b + p - a for 2 x 128 rows per tile (rows of 32 bytes, 32-byte swizzle)
         const uint32_t t = threadIdx.x - 64;
         const uint32_t Pw[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
@@ -118,8 +120,8 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
             tc::mbar_wait(&full[s], (it / kR1Stages) & 1);
             uint8_t *st = base + s * 24576;
 #pragma unroll
-            for (int e = 0; e < 4; ++e) {
-                const uint32_t r = t + 64 * e, m = r >> 7, j = r & 127;
+            for (int e = 0; e < 8 / PW; ++e) {
+                const uint32_t r = t + 32 * PW * e, m = r >> 7, j = r & 127;
                 const uint32_t sw = (j >> 2) & 1, o0 = j * 32 + (sw << 4), o1 = j * 32 + ((1 - sw) << 4);
                 uint8_t *tb = st + m * 12288;
                 const uint4 a_lo = *reinterpret_cast<const uint4 *>(tb + o0), a_hi = *reinterpret_cast<const uint4 *>(tb + o1);
@@ -150,6 +152,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
         }
     } else {
         const uint32_t q = warp & 3;                // TMEM lanes 32 q ..: rows of the a / b / D / unused block
+                                                    // (the 4 epilogue warps cover q = 0..3 for PW = 2 or 4)
         for (uint32_t c = 0; c < nch; ++c) {
             const uint32_t g = c & 1;
             tc::mbar_wait(&dready[g], (c >> 1) & 1);
@@ -174,7 +177,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
     // anti-diagonal sums s_n = sum_{i+i'=n} M[i][i'] of the three blocks, then S -> acc17 -> fe
     if (threadIdx.x < 3 * 64) s_diag[threadIdx.x >> 6][threadIdx.x & 63] = 0;
     __syncthreads();
-    if (warp >= 4 && (warp & 3) < 3) {
+    if (warp >= 2 + PW && (warp & 3) < 3) {
 #pragma unroll
         for (int i = 0; i < 32; ++i)
             atomicAdd(&s_diag[warp & 3][lane + i], macc[i]);
