@@ -194,7 +194,11 @@ struct Knobs {
     // BZK_R1_TC=0/1: round 1 of d = 2 BN254 proofs runs k_round1_tc (the three product sums as u8
     // tensor-core products over the pairs, round1_tc.cuh) instead of k_round<2, ., FIRST>
     uint32_t r1tc = 1;
+    // BZK_FUSED_TC=0/1: the fused rounds of d = 2 BN254 proofs run k_fused_tc (folds on the integer
+    // pipe, the two evaluation sums as u8 tensor-core products, fused_tc.cuh) instead of k_round
+    uint32_t fused_tc = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_FUSED_TC")) fused_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_R1_TC")) r1tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_TC")) multi_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_DUAL")) dual = atoi(e) ? 1 : 0;
@@ -229,9 +233,22 @@ uint32_t ctas_for(uint64_t h, uint64_t nb) {
 
 // CTAs per proof over every global round i < i0 (ctas_for is not monotone in h: ppt is floored).
 // The partials buffer is sized with this maximum; each round indexes it with its own stride.
-uint32_t max_round_ctas(uint32_t k, uint32_t i0, uint64_t nb) {
+bool r1_use_tc(uint32_t D, uint64_t h);
+uint32_t r1tc_ctas(uint64_t h, uint64_t nb);
+bool ftc_use(uint32_t D, uint32_t i) { return knobs().fused_tc && D == 2 && i >= 2; }
+
+// CTAs per proof of global round i (h pairs): k_round1_tc / k_fused_tc (<= 32768 pairs per CTA: its
+// s32 accumulator bound) / k_round
+uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb) {
+    if (i == 1 && r1_use_tc(D, h)) return r1tc_ctas(h, nb);
+    uint32_t c = ctas_for(h, nb);
+    if (ftc_use(D, i)) c = std::max<uint32_t>(c, (uint32_t)((h + 32767) / 32768));
+    return c;
+}
+
+uint32_t max_round_ctas(uint32_t D, uint32_t k, uint32_t i0, uint64_t nb) {
     uint32_t c = 1;
-    for (uint32_t i = 1; i < i0; ++i) c = std::max(c, ctas_for(1ull << (k - i), nb));
+    for (uint32_t i = 1; i < i0; ++i) c = std::max(c, round_ctas(D, i, 1ull << (k - i), nb));
     return c;
 }
 
@@ -359,7 +376,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
         size_t s = std::max(sizeof(ProofState), sizeof(gl::State)) + 4;
-        uint32_t c = P.k ? (P.multi ? max_multi_ctas(P.k, P.i0, bw) : max_round_ctas(P.k, P.i0, bw)) : 1;
+        uint32_t c = P.k ? (P.multi ? max_multi_ctas(P.k, P.i0, bw) : max_round_ctas(P.D, P.k, P.i0, bw)) : 1;
         s += (size_t)c * P.part_nv * P.esz;
         if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * P.esz;
         if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * P.esz;
@@ -381,7 +398,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
              small_cs_log(P.D, P.k, P.B) < 0;
     if (P.dual) { nw = 2; bw = (P.B + 1) / 2; }   // two waves of B/2: the same scratch as one wave of B
     P.Bw = bw; P.nwaves = nw;
-    P.cmax = P.k ? std::max(max_round_ctas(P.k, P.i0, bw), max_round_ctas(P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
+    P.cmax = P.k ? std::max(max_round_ctas(P.D, P.k, P.i0, bw), max_round_ctas(P.D, P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
     if (P.multi) P.cmax = std::max(max_multi_ctas(P.k, P.i0, bw), max_multi_ctas(P.k, P.i0, P.B - (nw - 1) * bw));
 
     size_t off = 0;
@@ -750,14 +767,14 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         }
         CUtensorMap tm;
         memset(&tm, 0, sizeof tm);
-        const bool r1tc = i == 1 && r1_use_tc(D, h);
-        if (r1tc) {
-            rp.ctas = std::min(r1tc_ctas(h, io.nb), P.cmax);
+        const bool r1tc = i == 1 && r1_use_tc(D, h), ftc = ftc_use(D, i);
+        if (r1tc || ftc) {
+            rp.ctas = round_ctas(D, i, h, io.nb);
             rp.cluster = 1;
-            if (!make_r1_map(&tm, P.order, tab, h, io.nb * D))
-                return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_round1_tc)");
         }
-        rp.tma = r1tc ? 0 : knobs().tma_for(D, i == 1);
+        if (r1tc && !make_r1_map(&tm, P.order, tab, h, io.nb * D))
+            return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (k_round1_tc)");
+        rp.tma = r1tc ? 0 : ftc ? 1 : knobs().tma_for(D, i == 1);
         if (rp.tma) {
             const uint64_t E = i == 1 ? 2 : 4;   // raw entries per pair and table
             const uint32_t box = P.order == 0 ? (uint32_t)(E * 8) : 8u;
@@ -767,7 +784,9 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-            cudaError_t e = r1tc ? r1tc_launch(P.order, grid, s, rp, tm) : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
+            cudaError_t e = r1tc  ? r1tc_launch(P.order, grid, s, rp, tm)
+                            : ftc ? ftc_launch(P.order, grid, s, rp, tm)
+                                  : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
         }

@@ -1,5 +1,7 @@
-// k_r1tc.cu -- instantiations of the tensor-core round-1 kernel for d = 2 (round1_tc.cuh)
+// k_r1tc.cu -- instantiations of the tensor-core round kernels for d = 2: round 1 (round1_tc.cuh) and
+// the fused fold + eval rounds (fused_tc.cuh)
 #include <stdlib.h>
+#include "fused_tc.cuh"
 #include "round1_tc.cuh"
 
 namespace bzk {
@@ -23,7 +25,15 @@ cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundPa
     return cudaErrorInvalidValue;
 }
 
+cudaError_t ftc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
+    if (order == 1) k_fused_tc<1><<<grid, kFtThreads, kFtSmem, s>>>(p, tm);
+    else k_fused_tc<0><<<grid, kFtThreads, kFtSmem, s>>>(p, tm);
+    return cudaGetLastError();
+}
+
 cudaError_t r1tc_set_attrs() {
+    cudaFuncSetAttribute(k_fused_tc<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFtSmem);
+    cudaFuncSetAttribute(k_fused_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFtSmem);
 #define BZK_R1_ATTR(NS, PW)                                                                                  \
     cudaFuncSetAttribute(k_round1_tc<0, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS)); \
     cudaFuncSetAttribute(k_round1_tc<1, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS));

@@ -917,6 +917,8 @@ template <int D>
 cudaError_t set_kernel_attrs();   // once per process, before any launch or graph capture
 // k_round1_tc (round1_tc.cuh, k_r1tc.cu): d = 2 round 1 on the tensor cores
 cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm);
-cudaError_t r1tc_set_attrs();
+cudaError_t r1tc_set_attrs();   // and k_fused_tc's
+// k_fused_tc (fused_tc.cuh, k_r1tc.cu): d = 2 fused rounds with the evaluation sums on the tensor cores
+cudaError_t ftc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm);
 
 }  // namespace bzk
