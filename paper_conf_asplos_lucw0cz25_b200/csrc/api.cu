@@ -197,7 +197,11 @@ struct Knobs {
     // BZK_FUSED_TC=0/1: the fused rounds of d = 2 BN254 proofs run k_fused_tc (folds on the integer
     // pipe, the two evaluation sums as u8 tensor-core products, fused_tc.cuh) instead of k_round
     uint32_t fused_tc = 1;
+    // BZK_D3_TC=0/1: round 1 and the fused rounds of d = 3 BN254 proofs run k_fused_tc<3, ...> (the
+    // last product of every point as a u8 tensor-core sum over the pairs, fused_tc.cuh) instead of k_round
+    uint32_t d3tc = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_D3_TC")) d3tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_FUSED_TC")) fused_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_R1_TC")) r1tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_MULTI_TC")) multi_tc = atoi(e) ? 1 : 0;
@@ -235,7 +239,9 @@ uint32_t ctas_for(uint64_t h, uint64_t nb) {
 // The partials buffer is sized with this maximum; each round indexes it with its own stride.
 bool r1_use_tc(uint32_t D, uint64_t h);
 uint32_t r1tc_ctas(uint64_t h, uint64_t nb);
-bool ftc_use(uint32_t D, uint32_t i) { return knobs().fused_tc && D == 2 && i >= 2; }
+bool ftc_use(uint32_t D, uint32_t i) {
+    return (knobs().fused_tc && D == 2 && i >= 2) || (knobs().d3tc && D == 3);
+}
 
 // CTAs per proof of global round i (h pairs): k_round1_tc / k_fused_tc (<= 32768 pairs per CTA: its
 // s32 accumulator bound) / k_round
@@ -785,7 +791,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
             cudaError_t e = r1tc  ? r1tc_launch(P.order, grid, s, rp, tm)
-                            : ftc ? ftc_launch(P.order, grid, s, rp, tm)
+                            : ftc ? ftc_launch(D, i == 1, P.order, grid, s, rp, tm)
                                   : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");

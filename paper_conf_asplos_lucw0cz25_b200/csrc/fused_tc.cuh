@@ -1,21 +1,25 @@
-// fused_tc.cuh -- the fused fold(r_{i-1}) + eval(i) round of d = 2 BN254 proofs with the evaluation
-// sums on the tensor cores (tcgen05 kind::i8); the folds stay on the integer pipe.
+// fused_tc.cuh -- sum-check rounds with the evaluation sums on the tensor cores (tcgen05 kind::i8);
+// the folds and the first d - 2 products of every point stay on the integer pipe.
 //
-// Same round as k_round<2, ORDER, FIRST = false, TMA = true> (sumcheck.cuh: TMA-staged raw entries,
-// fixed-multiplier folds written to the other ping-pong buffer), but the two summed points of
-// a fused round (Pts<2, DERIVE>: t = 0 and the leading coefficient) are
-//   g(0) = sum_j a0_j a1_j,   c_inf = sum_j D0_j D1_j       (a = folded entry, D = lazy b - a)
-// computed as u8 products over the pairs (round1_tc.cuh header: sum_j x_j y_j = sum M[i][i'] 2^(8(i+i'))
-// with M = X^T Y, K = the pairs).  Each compute warp writes its 32 pairs' (a0 | D0 | a1 | D1) bytes into
-// its own 4 KiB tile (32 rows x 32 bytes per vector, 32-byte swizzle, MN-major operands) and signals
-// the MMA warp, which issues one M = 128 (a0 | D0 | a1 | D1), N = 64 (a1 | D1), K = 32 product per tile
-// into the CTA's TMEM accumulator; the diagonal blocks (a0 x a1, D0 x D1) are the two M's.  At most
-// 32768 pairs per CTA keep every s32 entry < 32768 * 255^2 < 2^31, so one accumulator lasts the CTA.
-// After the loop: anti-diagonal sums -> S (< 2^527) -> acc17_to_fe = the canonical partial k_round's
-// acc17 path produces (same integers, same residue), then round_finish.
+// Same rounds as k_round<D, ORDER, FIRST, TMA = true> (sumcheck.cuh: TMA-staged raw entries,
+// fixed-multiplier folds written to the other ping-pong buffer), but the LAST product of every
+// summed point -- eval_one's mul_acc(acc_t, X_t, Y_t), a 256 x 256-bit product added unreduced into a
+// 544-bit accumulator -- is a sum over the pairs sum_j X_t(j) Y_t(j) computed as u8 products
+// (round1_tc.cuh header: sum_j x_j y_j = sum M[i][i'] 2^(8(i+i')) with M = X^T Y, K = the pairs):
+//   d = 2 fused rounds (points 0, inf):      X = a0 | D0,            Y = a1 | D1       (a = folded entry,
+//                                                                                       D = lazy b - a)
+//   d = 3 fused rounds (points 0, 2, inf):   X_t = x0(t) x1(t) R^-1, Y_t = x2(t)
+//   d = 3 round 1 (points 0, 1, 2, inf):     same, x_m(t) from the raw (a, b)
+// Each compute warp writes its 32 pairs' operand bytes into its own tile (32 rows x 32 bytes per vector,
+// 32-byte swizzle, MN-major operands; FtGeo) and signals the MMA warp, which issues one M = 128, N = 32 NV
+// (d = 2: 64), K = 32 product per tile into the CTA's TMEM accumulator; the diagonal blocks are the M_t.
+// At most 32768 pairs per CTA keep every s32 entry < 32768 * 255^2 < 2^31, so one accumulator lasts the
+// CTA.  After the loop: anti-diagonal sums -> S (< 2^527) -> acc17_to_fe = the canonical partial
+// k_round's acc17 path produces (same integers, same residue), then round_finish.
 //
-// This removes the two 256 x 256-bit products per pair (256 of ~910 integer-pipe slots) from the
-// integer pipe, which the folds and the products shared (ncu r02c: fma-heavy 75 %, DRAM 64 %).
+// d = 2 removes the two 256 x 256-bit products per pair (256 of ~910 integer-pipe slots) from the
+// integer pipe, which the folds and the products shared (ncu r02c: fma-heavy 75 %, DRAM 64 %); d = 3
+// removes NV of its 2 NV products per pair (the Montgomery products x0 x1 stay on the integer pipe).
 #pragma once
 #include <stdint.h>
 #include "sumcheck.cuh"
@@ -23,20 +27,57 @@
 
 namespace bzk {
 
-constexpr int kFtCompute = 256;                    // compute threads (8 warps, as k_round)
-constexpr int kFtThreads = kFtCompute + 32;        // + the MMA warp
+// compute warps per CTA: 8 (as k_round); the d = 3 fused rounds (6 folds + 3 Montgomery products per
+// pair, one CTA per SM by shared memory) run 12 for latency hiding
+template <int D, bool FIRST> __host__ __device__ constexpr int ft_nw() { return (D == 3 && !FIRST) ? 12 : 8; }
+template <int D, bool FIRST> __host__ __device__ constexpr int ft_threads() { return 32 * ft_nw<D, FIRST>() + 32; }   // + the MMA warp
 constexpr uint64_t kFtMaxPairs = 32768;            // pairs per CTA (s32 accumulator bound)
-constexpr size_t kFtSmem = 1024 + (size_t)(kFtCompute / 32) * 2 * 4096 + (size_t)(kFtCompute / 32) * 4096;
 
-template <int ORDER>
-__global__ void __launch_bounds__(kFtThreads, 2) k_fused_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
-    constexpr int D = 2, NV = Pts<2, true>::NV;    // t = 0, inf
-    using G = TmaGeo<ORDER, false>;
-    static_assert(G::NSTAGE == 1 && G::SLOT == 4096, "fused-round TMA geometry");
+// Per-warp operand tile of one MMA (32 pairs = K), MN-major 32-byte rows, 1 KiB per vector:
+//   d = 2 fused:   A = (a0 | D0 | a1 | D1) M = 128, B = (a1 | D1) at +2 KiB, N = 64   (points 0, inf)
+//   d = 3 fused:   A = (X0 | X2 | Xinf | Y0), B = (Y0 | Y2 | Yinf) at +3 KiB, N = 96 (points 0, 2, inf)
+//   d = 3 round 1: A = (X0 | X1 | X2 | Xinf), B = (Y0 | Y1 | Y2 | Yinf) at +4 KiB, N = 128
+// with X_t = x0(t) x1(t) R^-1 (the lazy Montgomery product eval_one forms, < 2p) and Y_t = x2(t) (lazy,
+// < 2p): eval_one's mul_acc(acc_t, X_t, Y_t) summed on the tensor cores.  Diagonal block t (rows 32t,
+// columns 32t) of D is M_t = X_t^T Y_t.  Rows 96..127 of the d = 3 fused A overlap B's first
+// vector (those D rows are never read).
+template <int D, bool FIRST> struct FtGeo;
+template <> struct FtGeo<2, false> { static constexpr uint32_t TILE = 4096, BOFF = 2048, N = 64, TCOLS = 64; };
+template <> struct FtGeo<3, false> { static constexpr uint32_t TILE = 6144, BOFF = 3072, N = 96, TCOLS = 128; };
+template <> struct FtGeo<3, true> { static constexpr uint32_t TILE = 8192, BOFF = 4096, N = 128, TCOLS = 128; };
+
+template <int D, bool FIRST>
+constexpr size_t ft_smem() {
+    return 1024 + (size_t)ft_nw<D, FIRST>() * D * TmaGeo<0, FIRST>::NSTAGE * TmaGeo<0, FIRST>::SLOT +
+           (size_t)ft_nw<D, FIRST>() * FtGeo<D, FIRST>::TILE;
+}
+constexpr size_t kFtSmem = ft_smem<2, false>();
+
+// d = 3: table m's value at summed point idx (Pts<3, DERIVE> order), exactly as eval_one forms it
+// (a = entry / folded entry, s = b (round 1) or the lazy delta (fused rounds), dl = round 1's delta)
+template <bool DERIVE>
+__device__ __forceinline__ fe d3_point(const fe &a, const fe &s, const fe &dl, int idx) {
+    const int t = point_t<3, DERIVE>(idx);
+    if (t == 0) return a;
+    if (t == 1) return s;
+    if (t < 0) return DERIVE ? s : dl;
+    // t == 2
+    if (DERIVE) return lz_red(lz_add(lz_red(lz_add(a, s)), s));
+    return lz_red(lz_add(s, dl));
+}
+
+template <int D, int ORDER, bool FIRST>
+__global__ void __launch_bounds__(ft_threads<D, FIRST>(), (D == 2 ? 2 : 1)) k_fused_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
+    static_assert(D == 2 ? !FIRST : D == 3, "k_fused_tc shapes: d = 2 fused rounds, d = 3 round 1 and fused rounds");
+    constexpr bool DERIVE = !FIRST;
+    constexpr int NV = Pts<D, DERIVE>::NV;
+    using G = TmaGeo<ORDER, FIRST>;
+    using FG = FtGeo<D, FIRST>;
+    constexpr int NS = G::NSTAGE, NW = ft_nw<D, FIRST>(), kFtCompute = 32 * NW;
     __shared__ fe s_red[32 * NV];
     __shared__ fe s_clu[NV];
     __shared__ int s_last;
-    __shared__ __align__(8) uint64_t bars[(kFtCompute / 32) * D], tfull[kFtCompute / 32], tempty[kFtCompute / 32], dfin;
+    __shared__ __align__(8) uint64_t bars[NW * D * NS], tfull[NW], tempty[NW], dfin;
     __shared__ uint32_t s_tmem;
     __shared__ __align__(16) fe sK[8];
     extern __shared__ uint8_t ft_raw[];
@@ -44,119 +85,156 @@ __global__ void __launch_bounds__(kFtThreads, 2) k_fused_tc(RoundParams P, const
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t h = 1ull << P.log_h;
     const uint64_t stride = (uint64_t)P.ctas * kFtCompute;
-    const fe *src = P.src + (size_t)b * D * (4 * h);
-    fe *dst = P.dst + (size_t)b * D * (2 * h);
-    (void)src;
+    fe *dst = FIRST ? nullptr : P.dst + (size_t)b * D * (2 * h);
 
-    if (threadIdx.x < 8) sK[threadIdx.x] = mont_mul(P.ps[b].rmont, P.consts[kConstPow2 + threadIdx.x]);   // r 2^(32t+64)
+    if (!FIRST && threadIdx.x < 8)
+        sK[threadIdx.x] = mont_mul(P.ps[b].rmont, P.consts[kConstPow2 + threadIdx.x]);   // r 2^(32t+64)
     if (threadIdx.x == 0) {
-        for (int w = 0; w < kFtCompute / 32; ++w) {
-            tc::mbar_init_n(&bars[2 * w], 1);
-            tc::mbar_init_n(&bars[2 * w + 1], 1);
+        for (int q = 0; q < NW * D * NS; ++q) tc::mbar_init_n(&bars[q], 1);
+        for (int w = 0; w < NW; ++w) {
             tc::mbar_init_n(&tfull[w], 1);
             tc::mbar_init_n(&tempty[w], 1);
         }
         tc::mbar_init_n(&dfin, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    if (warp == kFtCompute / 32) tc::tmem_alloc<64>(&s_tmem);
+    if (warp == NW) tc::tmem_alloc<FG::TCOLS>(&s_tmem);
     tc::fence_before();
     __syncthreads();
     tc::fence_after();
     const uint32_t tmem = s_tmem;
-    uint8_t *tiles = base + (size_t)(kFtCompute / 32) * D * G::SLOT;   // [warp][a0 | D0 | a1 | D1][32 rows][32 B]
+    uint8_t *tiles = base + (size_t)NW * D * NS * G::SLOT;   // [warp][vectors][32 rows][32 B]
 
-    if (warp < kFtCompute / 32) {
-        uint8_t *wslots = base + (size_t)warp * D * G::SLOT;
-        uint64_t *wbars = bars + warp * D;
-        uint8_t *tile = tiles + warp * 4096;
+    if (warp < NW) {
+        uint8_t *wslots = base + (size_t)warp * D * NS * G::SLOT;
+        uint64_t *wbars = bars + warp * D * NS;
+        uint8_t *tile = tiles + warp * FG::TILE;
         const uint64_t row0 = (uint64_t)b * D * (G::E * h / 4);
         const uint64_t trows = G::E * h / 4;
         const uint64_t j0 = (uint64_t)blockIdx.x * kFtCompute + warp * 32;
-        if (lane == 0 && j0 < h)
+        if (lane == 0)
 #pragma unroll
-            for (int m = 0; m < D; ++m)
-                tma_issue<ORDER, false>(&tmap, wslots + m * G::SLOT, &wbars[m], row0 + m * trows, h, j0);
+            for (int st = 0; st < (FIRST ? NS - 1 : 1); ++st)
+                if (j0 + st * stride < h)
+#pragma unroll
+                    for (int m = 0; m < D; ++m)
+                        tma_issue<ORDER, FIRST>(&tmap, wslots + (st * D + m) * G::SLOT, &wbars[st * D + m],
+                                                row0 + m * trows, h, j0 + st * stride);
+        const uint32_t sw = (lane >> 2) & 1, o0 = lane * 32 + (sw << 4), o1 = lane * 32 + ((1 - sw) << 4);
+        auto put = [&](int v, const fe &x) {
+            *reinterpret_cast<uint4 *>(tile + v * 1024 + o0) = make_uint4(x.l[0], x.l[1], x.l[2], x.l[3]);
+            *reinterpret_cast<uint4 *>(tile + v * 1024 + o1) = make_uint4(x.l[4], x.l[5], x.l[6], x.l[7]);
+        };
         uint32_t it = 0;
         for (uint64_t jw = j0; jw < h; jw += stride, ++it) {
+            const uint32_t st = NS == 1 ? 0 : it % NS;
+            const uint32_t par = NS == 1 ? (it & 1) : ((it / NS) & 1);
             const uint64_t j = jw + lane;
+            if (FIRST && lane == 0 && jw + (NS - 1) * stride < h) {
+                // the stage of tile it + NS - 1 was consumed by iteration it - 1 (__syncwarp below)
+                const uint32_t sn = (it + NS - 1) % NS;
+#pragma unroll
+                for (int m = 0; m < D; ++m)
+                    tma_issue<ORDER, FIRST>(&tmap, wslots + (sn * D + m) * G::SLOT, &wbars[sn * D + m],
+                                            row0 + m * trows, h, jw + (NS - 1) * stride);
+            }
             fe a[D], sv[D];
 #pragma unroll
             for (int m = 0; m < D; ++m) {
-                uint8_t *slot = wslots + m * G::SLOT;
-                mbar_wait(&wbars[m], it & 1);
+                uint8_t *slot = wslots + (st * D + m) * G::SLOT;
+                mbar_wait(&wbars[st * D + m], par);
                 fe x[G::E];
 #pragma unroll
-                for (int e = 0; e < G::E; ++e) x[e] = tma_entry<ORDER, false>(slot, lane, e);
-                fold_group<D, ORDER, false>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
-                __syncwarp();                  // every lane has consumed the slot
-                if (lane == 0 && jw + stride < h)
-                    tma_issue<ORDER, false>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);
+                for (int e = 0; e < G::E; ++e) x[e] = tma_entry<ORDER, FIRST>(slot, lane, e);
+                fold_group<D, ORDER, FIRST>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
+                if (!FIRST) {
+                    __syncwarp();              // every lane has consumed the slot
+                    if (lane == 0 && jw + stride < h)
+                        tma_issue<ORDER, FIRST>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);
+                }
             }
+            if (FIRST) __syncwarp();           // every lane has read stage st (refilled at the next iteration)
             // the previous tile's product has read this warp's tile
             if (it > 0) tc::mbar_wait(&tempty[warp], (it - 1) & 1);
-            const uint32_t sw = (lane >> 2) & 1, o0 = lane * 32 + (sw << 4), o1 = lane * 32 + ((1 - sw) << 4);
-            auto put = [&](int v, const fe &x) {
-                *reinterpret_cast<uint4 *>(tile + v * 1024 + o0) = make_uint4(x.l[0], x.l[1], x.l[2], x.l[3]);
-                *reinterpret_cast<uint4 *>(tile + v * 1024 + o1) = make_uint4(x.l[4], x.l[5], x.l[6], x.l[7]);
-            };
-            put(0, a[0]);
-            put(1, sv[0]);
-            put(2, a[1]);
-            put(3, sv[1]);
+            if constexpr (D == 2) {
+                put(0, a[0]);
+                put(1, sv[0]);
+                put(2, a[1]);
+                put(3, sv[1]);
+            } else {
+                fe dl[D];
+#pragma unroll
+                for (int m = 0; m < D; ++m) dl[m] = FIRST ? lz_red(lz_sub(sv[m], a[m])) : sv[m];
+#pragma unroll
+                for (int idx = 0; idx < NV; ++idx) {
+                    const fe x0 = d3_point<DERIVE>(a[0], sv[0], dl[0], idx);
+                    const fe x1 = d3_point<DERIVE>(a[1], sv[1], dl[1], idx);
+                    put(idx, mont_mul_lz(x0, x1));
+                    put(FG::BOFF / 1024 + idx, d3_point<DERIVE>(a[2], sv[2], dl[2], idx));
+                }
+            }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // tile (generic writes) -> MMA reads
             __syncwarp();
             if (lane == 0) tc::mbar_arrive(&tfull[warp]);
         }
     } else if (lane == 0) {
-        // MMA warp: one product per compute-warp tile, warps visited round-robin
-        const uint32_t idesc = tc::idesc_u8(128, 64, true) | (1u << 15);   // A and B MN-major
+        // MMA warp: one product per compute-warp tile, issued for whichever warp's tile is ready (a fixed
+        // round-robin order would hold every warp to the slowest one: each has a single tile)
+        const uint32_t idesc = tc::idesc_u8(128, FG::N, true) | (1u << 15);   // A and B MN-major
         const uint32_t tb = smem_u32(tiles);
-        uint32_t nw[kFtCompute / 32], nmax = 0;
+        uint32_t nw[NW], done[NW], left = 0, nmax = 0;
 #pragma unroll
-        for (int w = 0; w < kFtCompute / 32; ++w) {
+        for (int w = 0; w < NW; ++w) {
             const uint64_t j0 = (uint64_t)blockIdx.x * kFtCompute + w * 32;
             nw[w] = j0 < h ? (uint32_t)((h - 1 - j0) / stride + 1) : 0;
+            done[w] = 0;
+            left += nw[w];
             nmax = nw[w] > nmax ? nw[w] : nmax;
         }
         bool first = true;
-        for (uint32_t it = 0; it < nmax; ++it) {
+        while (left) {
+            bool issued = false;
 #pragma unroll
-            for (int w = 0; w < kFtCompute / 32; ++w) {
-                if (it >= nw[w]) continue;
-                tc::mbar_wait(&tfull[w], it & 1);
-                tc::fence_after();
-                const uint32_t t0 = tb + w * 4096;
-                tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + 2048, 1024, 256), idesc, !first);
-                first = false;
-                tc::commit(&tempty[w]);
+            for (int w = 0; w < NW; ++w) {
+                if (done[w] < nw[w] && tc::mbar_test(&tfull[w], done[w] & 1)) {
+                    tc::fence_after();
+                    const uint32_t t0 = tb + w * FG::TILE;
+                    tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + FG::BOFF, 1024, 256), idesc,
+                               !first);
+                    first = false;
+                    tc::commit(&tempty[w]);
+                    ++done[w];
+                    --left;
+                    issued = true;
+                }
             }
+            if (!issued) __nanosleep(100);   // a tile takes microseconds to build: keep this warp off the issue slots
         }
         if (nmax > 0) tc::commit(&dfin);
     }
     __syncwarp();
-    // anti-diagonal sums of the two diagonal blocks (warps 0 and 1 read TMEM lanes 0..31 / 32..63)
-    uint32_t *sM = reinterpret_cast<uint32_t *>(base);   // [2][32][33] (reuses the TMA slots)
-    __shared__ unsigned long long s_diag[2][64];
+    // anti-diagonal sums of the NV diagonal blocks (warp t reads TMEM lanes 32t.., columns 32t..)
+    uint32_t *sM = reinterpret_cast<uint32_t *>(base);   // [NV][32][33] (reuses the TMA slots)
+    __shared__ unsigned long long s_diag[NV][64];
     const bool any = (uint64_t)blockIdx.x * kFtCompute < h;
     tc::fence_before();
     __syncthreads();
-    if (warp < 2 && any) {
+    if (warp < (uint32_t)NV && any) {
         tc::mbar_wait(&dfin, 0);
         tc::fence_after();
         uint32_t v[32];
         tc::ld_x32(tmem + ((warp * 32) << 16) + warp * 32, v);
         tc::wait_ld();
 #pragma unroll
-        for (int i = 0; i < 32; ++i) sM[(warp * 32 + lane) * 33 + i] = v[i];   // row = byte `lane` of a0 / D0
+        for (int i = 0; i < 32; ++i) sM[(warp * 32 + lane) * 33 + i] = v[i];   // row = byte `lane` of X_t
     }
     tc::fence_before();
     __syncthreads();
-    if (warp == kFtCompute / 32) {
+    if (warp == NW) {
         tc::fence_after();
-        tc::tmem_dealloc<64>(tmem);
+        tc::tmem_dealloc<FG::TCOLS>(tmem);
     }
-    if (threadIdx.x < 128) {
+    if (threadIdx.x < NV * 64) {
         const uint32_t t = threadIdx.x >> 6, n = threadIdx.x & 63;
         unsigned long long s = 0;
         if (any)
@@ -182,12 +260,12 @@ __global__ void __launch_bounds__(kFtThreads, 2) k_fused_tc(RoundParams P, const
                 carry = (carry >> 32) + (cur >> 32);
             }
         }
-        const fe f = acc17_to_fe(S);   // thread 0: g(0) partial, thread 1: c_inf partial
+        const fe f = acc17_to_fe(S);   // thread t: point t's partial (Pts<D, DERIVE> order)
 #pragma unroll
         for (int t = 0; t < NV; ++t)
             if (t == (int)threadIdx.x) acc[t] = f;
     }
-    round_finish<D, true>(P, b, acc, s_red, s_clu, &s_last);
+    round_finish<D, DERIVE>(P, b, acc, s_red, s_clu, &s_last);
 }
 
 }  // namespace bzk

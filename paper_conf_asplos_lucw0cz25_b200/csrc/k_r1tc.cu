@@ -1,5 +1,5 @@
-// k_r1tc.cu -- instantiations of the tensor-core round kernels for d = 2: round 1 (round1_tc.cuh) and
-// the fused fold + eval rounds (fused_tc.cuh)
+// k_r1tc.cu -- instantiations of the tensor-core round kernels: d = 2 round 1 (round1_tc.cuh), d = 2
+// fused rounds and d = 3 round 1 + fused rounds (fused_tc.cuh)
 #include <stdlib.h>
 #include "fused_tc.cuh"
 #include "round1_tc.cuh"
@@ -25,15 +25,30 @@ cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundPa
     return cudaErrorInvalidValue;
 }
 
-cudaError_t ftc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
-    if (order == 1) k_fused_tc<1><<<grid, kFtThreads, kFtSmem, s>>>(p, tm);
-    else k_fused_tc<0><<<grid, kFtThreads, kFtSmem, s>>>(p, tm);
+template <int D, bool FIRST>
+static cudaError_t ftc_launch_t(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
+    if (order == 1) k_fused_tc<D, 1, FIRST><<<grid, ft_threads<D, FIRST>(), ft_smem<D, FIRST>(), s>>>(p, tm);
+    else k_fused_tc<D, 0, FIRST><<<grid, ft_threads<D, FIRST>(), ft_smem<D, FIRST>(), s>>>(p, tm);
     return cudaGetLastError();
 }
 
+cudaError_t ftc_launch(uint32_t D, bool first, uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p,
+                       const CUtensorMap &tm) {
+    if (D == 2 && !first) return ftc_launch_t<2, false>(order, grid, s, p, tm);
+    if (D == 3) return first ? ftc_launch_t<3, true>(order, grid, s, p, tm) : ftc_launch_t<3, false>(order, grid, s, p, tm);
+    return cudaErrorInvalidValue;
+}
+
+template <int D, bool FIRST>
+static void ftc_attrs() {
+    cudaFuncSetAttribute(k_fused_tc<D, 0, FIRST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ft_smem<D, FIRST>());
+    cudaFuncSetAttribute(k_fused_tc<D, 1, FIRST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ft_smem<D, FIRST>());
+}
+
 cudaError_t r1tc_set_attrs() {
-    cudaFuncSetAttribute(k_fused_tc<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFtSmem);
-    cudaFuncSetAttribute(k_fused_tc<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kFtSmem);
+    ftc_attrs<2, false>();
+    ftc_attrs<3, false>();
+    ftc_attrs<3, true>();
 #define BZK_R1_ATTR(NS, PW)                                                                                  \
     cudaFuncSetAttribute(k_round1_tc<0, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS)); \
     cudaFuncSetAttribute(k_round1_tc<1, NS, PW>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(NS));

@@ -918,7 +918,9 @@ cudaError_t set_kernel_attrs();   // once per process, before any launch or grap
 // k_round1_tc (round1_tc.cuh, k_r1tc.cu): d = 2 round 1 on the tensor cores
 cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm);
 cudaError_t r1tc_set_attrs();   // and k_fused_tc's
-// k_fused_tc (fused_tc.cuh, k_r1tc.cu): d = 2 fused rounds with the evaluation sums on the tensor cores
-cudaError_t ftc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm);
+// k_fused_tc (fused_tc.cuh, k_r1tc.cu): d = 2 fused rounds, d = 3 round 1 and fused rounds with the
+// evaluation sums on the tensor cores
+cudaError_t ftc_launch(uint32_t D, bool first, uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p,
+                       const CUtensorMap &tm);
 
 }  // namespace bzk

@@ -89,6 +89,15 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
                  "@!P1 bra TC_WAIT;\n\t}" ::"r"(su32(bar)), "r"(parity) : "memory");
 }
 
+// non-blocking probe of an mbarrier phase
+__device__ __forceinline__ bool mbar_test(uint64_t *bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile("{\n\t.reg .pred P1;\n\t"
+                 "mbarrier.test_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+                 "selp.u32 %0, 1, 0, P1;\n\t}" : "=r"(ok) : "r"(su32(bar)), "r"(parity) : "memory");
+    return ok != 0;
+}
+
 // TMA tile loads (32-byte rows), completing on an mbarrier
 __device__ __forceinline__ void tma3(void *dst, const void *tm, int c0, int c1, int c2, uint64_t *bar) {
     asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
