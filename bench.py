@@ -687,18 +687,34 @@ def multi_tc_pass(K: int, m: int) -> bool:
     return m == 3 and K >= 10 and os.environ.get("BZK_MULTI_TC", "1") != "0"
 
 
-def imad_slots(d: int, k: int, kind: str) -> int:
-    """fma-heavy slots of the products one proof's launches of `kind` execute (the kernels' arithmetic,
-    DESIGN.md sec. 6): round 1 sums d+1 points per pair, each (d-2) Montgomery products + 1 unreduced
-    product; a fused round folds 2d entries per pair and sums d points (g(1) derived); a k_multi pass
-    does one unreduced product per entry."""
+def tc_rounds(d: int, gl: bool = False) -> tuple[bool, bool]:
+    """api.cu r1_use_tc / ftc_use: (round 1, fused rounds) sum the last product of every point on the
+    u8 tensor cores (BN254 d = 2: k_round1_tc, k_fused_tc<2>; d = 3: k_fused_tc<3, ., FIRST>)"""
+    if gl:
+        return False, False
+    on = lambda v: os.environ.get(v, "1") != "0"
+    if d == 2:
+        return on("BZK_R1_TC"), on("BZK_FUSED_TC")
+    if d == 3:
+        return on("BZK_D3_TC"), on("BZK_D3_TC")
+    return False, False
+
+
+def imad_slots(d: int, k: int, kind: str, gl: bool = False) -> int:
+    """fma-heavy slots of the products one proof's launches of `kind` execute on the integer pipe (the
+    kernels' arithmetic): round 1 sums d+1 points per pair, each (d-2) Montgomery
+    products + 1 unreduced product; a fused round folds 2d entries per pair and sums d points (g(1)
+    derived); a k_multi pass does one unreduced product per entry.  Where a kernel sums the last
+    product of every point on the tensor cores (tc_rounds) that unreduced product leaves the count."""
     tail_log = 8
     i0 = 1 if k - 1 <= tail_log else k - tail_log
+    tc1, tcf = tc_rounds(d, gl)
     point = 0 if d == 1 else (d - 2) * SLOT_MONT + SLOT_MULACC
     if kind == "round1":
-        return (d + 1) * point * (1 << (k - 1)) if i0 > 1 else 0
+        return (d + 1) * (point - (SLOT_MULACC if tc1 else 0)) * (1 << (k - 1)) if i0 > 1 else 0
     if kind == "fused":
-        return sum((2 * d * SLOT_FIXMUL + d * point) * (1 << (k - i)) for i in range(2, i0))
+        pf = point - (SLOT_MULACC if tcf else 0)
+        return sum((2 * d * SLOT_FIXMUL + d * pf) * (1 << (k - i)) for i in range(2, i0))
     passes = multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3")))
     if kind == "multi":
         return sum(SLOT_MULACC * (1 << K) for K, m in passes if not multi_tc_pass(K, m))
@@ -904,7 +920,7 @@ def run_sumcheck(args, rank, world, local):
     launches_per_step = max(1, dom_cnt / args.steps)
     avg_launch_s = dom_ms / max(1, dom_cnt) / 1000.0
     slot_peak = SMS * IMAD_PER_CLK_SM * sm_max_mhz * 1e6          # fma-heavy slots / s
-    slots_per_launch = imad_slots(d, k, kinds[dom]) * count / launches_per_step
+    slots_per_launch = imad_slots(d, k, kinds[dom], gl) * count / launches_per_step
     if kinds[dom] in ("multi", "multi_tc"):
         tc = kinds[dom] == "multi_tc"
         bytes_per_launch = multi_bytes(k, tc) * count / launches_per_step
@@ -938,8 +954,10 @@ def run_sumcheck(args, rank, world, local):
                     "frac": round(ach_slots / slot_peak, 4), "traffic": traffic,
                     "peak_source": f"guide unit counts: {SMS} SMs x {IMAD_PER_CLK_SM} fma-heavy slots/clk x "
                                    f"{sm_max_mhz:.0f} MHz ({peak_src} max clock); achieved = the kernel's product "
-                                   "slots per launch (fixmul fold 164, unreduced 256x256 product 128, Montgomery "
-                                   "product 272; DESIGN.md sec. 6) / CUDA-event launch time"}
+                                   "slots per launch on the integer pipe (fixmul fold 164, unreduced 256x256 product "
+                                   "128, Montgomery product 272; products summed on the tensor cores excluded; "
+                                   "DESIGN.md sec. 6) / CUDA-event launch time",
+                    "tensor_core_sums": dict(zip(("round1", "fused"), tc_rounds(d, gl)))}
     else:
         roofline = {"bound": "hbm", "kernel": dom, "achieved": round(ach_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
                     "frac": round(ach_gbs / hbm_peak, 4), "traffic": traffic,

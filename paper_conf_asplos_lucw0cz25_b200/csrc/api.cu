@@ -200,7 +200,11 @@ struct Knobs {
     // BZK_D3_TC=0/1: round 1 and the fused rounds of d = 3 BN254 proofs run k_fused_tc<3, ...> (the
     // last product of every point as a u8 tensor-core sum over the pairs, fused_tc.cuh) instead of k_round
     uint32_t d3tc = 1;
+    // BZK_FTC_SMALL_LOG=L: d = 2 fused rounds with h <= 2^L pairs per proof run the 2-warp k_fused_tc
+    // (one CTA per proof up to 2^11 pairs, fused_tc.cuh); 0 = off
+    uint32_t ftc_small_log = 12;
     Knobs() {
+        if (const char *e = getenv("BZK_FTC_SMALL_LOG")) ftc_small_log = (uint32_t)std::max(0, atoi(e));
         if (const char *e = getenv("BZK_D3_TC")) d3tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_FUSED_TC")) fused_tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_R1_TC")) r1tc = atoi(e) ? 1 : 0;
@@ -243,10 +247,17 @@ bool ftc_use(uint32_t D, uint32_t i) {
     return (knobs().fused_tc && D == 2 && i >= 2) || (knobs().d3tc && D == 3);
 }
 
+// the 2-warp k_fused_tc for the small late d = 2 rounds: 2048 pairs (32 per warp-iteration, 32
+// iterations) per CTA
+bool ftc_small(uint32_t D, uint32_t i, uint64_t h) {
+    return ftc_use(D, i) && D == 2 && knobs().ftc_small_log && h <= (1ull << knobs().ftc_small_log);
+}
+
 // CTAs per proof of global round i (h pairs): k_round1_tc / k_fused_tc (<= 32768 pairs per CTA: its
 // s32 accumulator bound) / k_round
 uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb) {
     if (i == 1 && r1_use_tc(D, h)) return r1tc_ctas(h, nb);
+    if (ftc_small(D, i, h)) return (uint32_t)std::max<uint64_t>(1, h / 2048);
     uint32_t c = ctas_for(h, nb);
     if (ftc_use(D, i)) c = std::max<uint32_t>(c, (uint32_t)((h + 32767) / 32768));
     return c;
@@ -791,7 +802,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
             cudaError_t e = r1tc  ? r1tc_launch(P.order, grid, s, rp, tm)
-                            : ftc ? ftc_launch(D, i == 1, P.order, grid, s, rp, tm)
+                            : ftc ? ftc_launch(D, i == 1, ftc_small(D, i, h), P.order, grid, s, rp, tm)
                                   : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");

@@ -27,10 +27,18 @@
 
 namespace bzk {
 
-// compute warps per CTA: 8 (as k_round); the d = 3 fused rounds (6 folds + 3 Montgomery products per
-// pair, one CTA per SM by shared memory) run 12 for latency hiding
-template <int D, bool FIRST> __host__ __device__ constexpr int ft_nw() { return (D == 3 && !FIRST) ? 12 : 8; }
-template <int D, bool FIRST> __host__ __device__ constexpr int ft_threads() { return 32 * ft_nw<D, FIRST>() + 32; }   // + the MMA warp
+// compute warps per CTA: 8 for d = 2 (two CTAs per SM); d = 3 (one CTA per SM by shared memory, long
+// integer-pipe chains per pair: 6 folds + 3 Montgomery products, or round 1's 4 Montgomery products)
+// runs 12 for latency hiding.  One TMA slot per (warp, table): the copy of the warp's next tile is issued
+// as soon as every lane has consumed the slot, so it lands while the rest of the iteration computes.
+// The small late fused rounds of d = 2 (h <= 2^12 pairs per proof: a few microseconds of work per CTA,
+// dominated by the CTA's fixed costs and the proof's serial finalisation) run NW = 2: one CTA of 96
+// threads per proof (two above 2^11), 7 resident per SM (registers), so a 1024-proof wave is one
+// CTA wave instead of several.
+template <int D, bool FIRST> __host__ __device__ constexpr int ft_nw() { return D == 3 ? 12 : 8; }
+constexpr int kFtSmallNW = 2;
+__host__ __device__ constexpr int ft_threads(int nw) { return 32 * nw + 32; }   // + the MMA warp
+__host__ __device__ constexpr int ft_minb(int D, int nw) { return D == 3 ? 1 : nw == kFtSmallNW ? 7 : 2; }
 constexpr uint64_t kFtMaxPairs = 32768;            // pairs per CTA (s32 accumulator bound)
 
 // Per-warp operand tile of one MMA (32 pairs = K), MN-major 32-byte rows, 1 KiB per vector:
@@ -46,12 +54,10 @@ template <> struct FtGeo<2, false> { static constexpr uint32_t TILE = 4096, BOFF
 template <> struct FtGeo<3, false> { static constexpr uint32_t TILE = 6144, BOFF = 3072, N = 96, TCOLS = 128; };
 template <> struct FtGeo<3, true> { static constexpr uint32_t TILE = 8192, BOFF = 4096, N = 128, TCOLS = 128; };
 
-template <int D, bool FIRST>
+template <int D, bool FIRST, int NW = ft_nw<D, FIRST>()>
 constexpr size_t ft_smem() {
-    return 1024 + (size_t)ft_nw<D, FIRST>() * D * TmaGeo<0, FIRST>::NSTAGE * TmaGeo<0, FIRST>::SLOT +
-           (size_t)ft_nw<D, FIRST>() * FtGeo<D, FIRST>::TILE;
+    return 1024 + (size_t)NW * D * TmaGeo<0, FIRST>::SLOT + (size_t)NW * FtGeo<D, FIRST>::TILE;
 }
-constexpr size_t kFtSmem = ft_smem<2, false>();
 
 // d = 3: table m's value at summed point idx (Pts<3, DERIVE> order), exactly as eval_one forms it
 // (a = entry / folded entry, s = b (round 1) or the lazy delta (fused rounds), dl = round 1's delta)
@@ -66,14 +72,15 @@ __device__ __forceinline__ fe d3_point(const fe &a, const fe &s, const fe &dl, i
     return lz_red(lz_add(s, dl));
 }
 
-template <int D, int ORDER, bool FIRST>
-__global__ void __launch_bounds__(ft_threads<D, FIRST>(), (D == 2 ? 2 : 1)) k_fused_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
+template <int D, int ORDER, bool FIRST, int NW>
+__global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
     static_assert(D == 2 ? !FIRST : D == 3, "k_fused_tc shapes: d = 2 fused rounds, d = 3 round 1 and fused rounds");
+    static_assert(NW >= Pts<D, !FIRST>::NV, "the epilogue reads one TMEM block per compute warp");
     constexpr bool DERIVE = !FIRST;
     constexpr int NV = Pts<D, DERIVE>::NV;
     using G = TmaGeo<ORDER, FIRST>;
     using FG = FtGeo<D, FIRST>;
-    constexpr int NS = G::NSTAGE, NW = ft_nw<D, FIRST>(), kFtCompute = 32 * NW;
+    constexpr int NS = 1, kFtCompute = 32 * NW;
     __shared__ fe s_red[32 * NV];
     __shared__ fe s_clu[NV];
     __shared__ int s_last;
@@ -112,14 +119,10 @@ __global__ void __launch_bounds__(ft_threads<D, FIRST>(), (D == 2 ? 2 : 1)) k_fu
         const uint64_t row0 = (uint64_t)b * D * (G::E * h / 4);
         const uint64_t trows = G::E * h / 4;
         const uint64_t j0 = (uint64_t)blockIdx.x * kFtCompute + warp * 32;
-        if (lane == 0)
+        if (lane == 0 && j0 < h)
 #pragma unroll
-            for (int st = 0; st < (FIRST ? NS - 1 : 1); ++st)
-                if (j0 + st * stride < h)
-#pragma unroll
-                    for (int m = 0; m < D; ++m)
-                        tma_issue<ORDER, FIRST>(&tmap, wslots + (st * D + m) * G::SLOT, &wbars[st * D + m],
-                                                row0 + m * trows, h, j0 + st * stride);
+            for (int m = 0; m < D; ++m)
+                tma_issue<ORDER, FIRST>(&tmap, wslots + m * G::SLOT, &wbars[m], row0 + m * trows, h, j0);
         const uint32_t sw = (lane >> 2) & 1, o0 = lane * 32 + (sw << 4), o1 = lane * 32 + ((1 - sw) << 4);
         auto put = [&](int v, const fe &x) {
             *reinterpret_cast<uint4 *>(tile + v * 1024 + o0) = make_uint4(x.l[0], x.l[1], x.l[2], x.l[3]);
@@ -127,33 +130,20 @@ __global__ void __launch_bounds__(ft_threads<D, FIRST>(), (D == 2 ? 2 : 1)) k_fu
         };
         uint32_t it = 0;
         for (uint64_t jw = j0; jw < h; jw += stride, ++it) {
-            const uint32_t st = NS == 1 ? 0 : it % NS;
-            const uint32_t par = NS == 1 ? (it & 1) : ((it / NS) & 1);
             const uint64_t j = jw + lane;
-            if (FIRST && lane == 0 && jw + (NS - 1) * stride < h) {
-                // the stage of tile it + NS - 1 was consumed by iteration it - 1 (__syncwarp below)
-                const uint32_t sn = (it + NS - 1) % NS;
-#pragma unroll
-                for (int m = 0; m < D; ++m)
-                    tma_issue<ORDER, FIRST>(&tmap, wslots + (sn * D + m) * G::SLOT, &wbars[sn * D + m],
-                                            row0 + m * trows, h, jw + (NS - 1) * stride);
-            }
             fe a[D], sv[D];
 #pragma unroll
             for (int m = 0; m < D; ++m) {
-                uint8_t *slot = wslots + (st * D + m) * G::SLOT;
-                mbar_wait(&wbars[st * D + m], par);
+                uint8_t *slot = wslots + m * G::SLOT;
+                mbar_wait(&wbars[m], it & 1);
                 fe x[G::E];
 #pragma unroll
                 for (int e = 0; e < G::E; ++e) x[e] = tma_entry<ORDER, FIRST>(slot, lane, e);
                 fold_group<D, ORDER, FIRST>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
-                if (!FIRST) {
-                    __syncwarp();              // every lane has consumed the slot
-                    if (lane == 0 && jw + stride < h)
-                        tma_issue<ORDER, FIRST>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);
-                }
+                __syncwarp();                  // every lane has consumed the slot
+                if (lane == 0 && jw + stride < h)
+                    tma_issue<ORDER, FIRST>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);
             }
-            if (FIRST) __syncwarp();           // every lane has read stage st (refilled at the next iteration)
             // the previous tile's product has read this warp's tile
             if (it > 0) tc::mbar_wait(&tempty[warp], (it - 1) & 1);
             if constexpr (D == 2) {
@@ -234,8 +224,8 @@ __global__ void __launch_bounds__(ft_threads<D, FIRST>(), (D == 2 ? 2 : 1)) k_fu
         tc::fence_after();
         tc::tmem_dealloc<FG::TCOLS>(tmem);
     }
-    if (threadIdx.x < NV * 64) {
-        const uint32_t t = threadIdx.x >> 6, n = threadIdx.x & 63;
+    for (uint32_t q = threadIdx.x; q < NV * 64; q += blockDim.x) {   // NW = 2: fewer threads than sums
+        const uint32_t t = q >> 6, n = q & 63;
         unsigned long long s = 0;
         if (any)
             for (int i = 0; i < 32; ++i)

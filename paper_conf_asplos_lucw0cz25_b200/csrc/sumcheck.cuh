@@ -920,7 +920,8 @@ cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundPa
 cudaError_t r1tc_set_attrs();   // and k_fused_tc's
 // k_fused_tc (fused_tc.cuh, k_r1tc.cu): d = 2 fused rounds, d = 3 round 1 and fused rounds with the
 // evaluation sums on the tensor cores
-cudaError_t ftc_launch(uint32_t D, bool first, uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p,
-                       const CUtensorMap &tm);
+// (small: the NW = 2 variant of the d = 2 fused rounds, api.cu ftc_small)
+cudaError_t ftc_launch(uint32_t D, bool first, bool small, uint32_t order, dim3 grid, cudaStream_t s,
+                       const RoundParams &p, const CUtensorMap &tm);
 
 }  // namespace bzk
