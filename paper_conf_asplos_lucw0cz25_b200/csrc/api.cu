@@ -203,7 +203,11 @@ struct Knobs {
     // BZK_FTC_SMALL_LOG=L: d = 2 fused rounds with h <= 2^L pairs per proof run the 2-warp k_fused_tc
     // (one CTA per proof up to 2^11 pairs, fused_tc.cuh); 0 = off
     uint32_t ftc_small_log = 12;
+    // BZK_R1_SW64=0/1: LSB round 1 of k_round1_tc loads each table's pairs as 64-byte rows (a_j | b_j), one
+    // TMA box per table, 64-byte swizzle; 0: a and b as separate boxes of 32-byte rows
+    uint32_t r1_sw64 = 1;
     Knobs() {
+        if (const char *e = getenv("BZK_R1_SW64")) r1_sw64 = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_FTC_SMALL_LOG")) ftc_small_log = (uint32_t)std::max(0, atoi(e));
         if (const char *e = getenv("BZK_D3_TC")) d3tc = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_FUSED_TC")) fused_tc = atoi(e) ? 1 : 0;
@@ -539,6 +543,13 @@ bool make_row_map(CUtensorMap *tm, const void *base, uint64_t rows, uint32_t box
 bool make_r1_map(CUtensorMap *tm, uint32_t order, const void *base, uint64_t h, uint64_t tables) {
     PFN_cuTensorMapEncodeTiled_v12000 enc = tensor_map_encoder();
     if (!enc) return false;
+    if (order == 0 && knobs().r1_sw64) {   // rows (a_j | b_j) of 64 bytes: dims (16 w, h, tables)
+        cuuint64_t dims3[3] = {16, h, tables}, strides3[2] = {64, 2 * h * 32};
+        cuuint32_t box3[3] = {16, 128, 1}, estr3[3] = {1, 1, 1};
+        return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT32, 3, const_cast<void *>(base), dims3, strides3, box3, estr3,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    }
     cuuint64_t dims[4], strides[3];
     cuuint32_t box[4], estr[4] = {1, 1, 1, 1};
     if (order == 1) {
@@ -801,7 +812,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-            cudaError_t e = r1tc  ? r1tc_launch(P.order, grid, s, rp, tm)
+            cudaError_t e = r1tc  ? r1tc_launch(P.order, P.order == 0 && knobs().r1_sw64, grid, s, rp, tm)
                             : ftc ? ftc_launch(D, i == 1, ftc_small(D, i, h), P.order, grid, s, rp, tm)
                                   : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
             ++ctx->launches;

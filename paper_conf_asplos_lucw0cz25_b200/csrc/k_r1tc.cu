@@ -9,9 +9,10 @@ namespace bzk {
 // launch shape: NS stages of 16 KiB (one CTA per SM)
 constexpr int kR1Stages = 12;
 
-cudaError_t r1tc_launch(uint32_t order, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
-    if (order == 1) k_round1_tc<1, kR1Stages><<<grid, kR1Threads, r1_smem(kR1Stages), s>>>(p, tm);
-    else k_round1_tc<0, kR1Stages><<<grid, kR1Threads, r1_smem(kR1Stages), s>>>(p, tm);
+cudaError_t r1tc_launch(uint32_t order, bool sw64, dim3 grid, cudaStream_t s, const RoundParams &p, const CUtensorMap &tm) {
+    if (order == 1) k_round1_tc<1, kR1Stages, false><<<grid, kR1Threads, r1_smem(kR1Stages), s>>>(p, tm);
+    else if (sw64) k_round1_tc<0, kR1Stages, true><<<grid, kR1Threads, r1_smem(kR1Stages), s>>>(p, tm);
+    else k_round1_tc<0, kR1Stages, false><<<grid, kR1Threads, r1_smem(kR1Stages), s>>>(p, tm);
     return cudaGetLastError();
 }
 
@@ -41,8 +42,9 @@ cudaError_t r1tc_set_attrs() {
     ftc_attrs<2, false, kFtSmallNW>();
     ftc_attrs<3, false>();
     ftc_attrs<3, true>();
-    cudaFuncSetAttribute(k_round1_tc<0, kR1Stages>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(kR1Stages));
-    cudaFuncSetAttribute(k_round1_tc<1, kR1Stages>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(kR1Stages));
+    cudaFuncSetAttribute(k_round1_tc<0, kR1Stages, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(kR1Stages));
+    cudaFuncSetAttribute(k_round1_tc<0, kR1Stages, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(kR1Stages));
+    cudaFuncSetAttribute(k_round1_tc<1, kR1Stages, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)r1_smem(kR1Stages));
     return cudaGetLastError();
 }
 

@@ -38,8 +38,13 @@ constexpr uint32_t kR1Stage = 16384;
 constexpr int kR1Threads = 128;
 constexpr size_t r1_smem(int NS) { return 1024 + (size_t)NS * kR1Stage; }
 
-template <int ORDER, int NS>
+// SW64 (LSB only): the stage holds each table's 128 pairs as contiguous 64-byte rows (a_j | b_j), one TMA
+// box of 8 KiB per table with the 64-byte swizzle, read by the MMA as 64-element MN blocks (the byte
+// rows 0..63 / 64..127 of A and the columns of B are the same (a | b) vectors as in the 32-byte
+// layout); otherwise a and b arrive as separate 4 KiB boxes of 32-byte rows (LSB: every other entry).
+template <int ORDER, int NS, bool SW64>
 __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, const __grid_constant__ CUtensorMap tmap) {
+    static_assert(!SW64 || ORDER == 0, "64-byte rows (a_j | b_j) exist in LSB order only");
     constexpr int D = 2, NV = Pts<2, false>::NV;   // points 0, 1, inf
     __shared__ fe s_red[32 * NV];
     __shared__ fe s_clu[NV];
@@ -84,7 +89,9 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
                 for (int m = 0; m < D; ++m) {
                     const int tab = (int)(b * D + m);
                     uint8_t *dstm = st + (1 - m) * 8192;   // table 1 first: A = (a1 | b1 | a0 | b0)
-                    if (ORDER == 1) {   // dims (8 w, h, 2: a / b, tables): a and b tiles in one box
+                    if (SW64) {         // dims (16 w, h, tables): rows (a_j | b_j)
+                        tc::tma3(dstm, &tmap, 0, j0, tab, &full[s]);
+                    } else if (ORDER == 1) {   // dims (8 w, h, 2: a / b, tables): a and b tiles in one box
                         tc::tma4(dstm, &tmap, 0, j0, 0, tab, &full[s]);
                     } else {            // dims (8 w, 2: a / b, h, tables)
                         tc::tma4(dstm, &tmap, 0, 0, j0, tab, &full[s]);
@@ -104,9 +111,10 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
                 tc::fence_after();
                 const uint32_t a0 = sb + s * kR1Stage;
 #pragma unroll
-                for (int q = 0; q < 4; ++q)   // K = 32 pairs per instruction
-                    tc::mma_u8(tmem + g * 64, tc::desc_sw32(a0 + q * 1024, 4096, 256),
-                               tc::desc_sw32(a0 + q * 1024, 4096, 256), idesc, !(first && q == 0));
+                for (int q = 0; q < 4; ++q) {   // K = 32 pairs per instruction
+                    const uint64_t da = SW64 ? tc::desc_sw64(a0 + q * 2048, 8192, 512) : tc::desc_sw32(a0 + q * 1024, 4096, 256);
+                    tc::mma_u8(tmem + g * 64, da, da, idesc, !(first && q == 0));
+                }
                 tc::commit(&empty[s]);
                 if (it % kR1Chunk == kR1Chunk - 1 || it == nt - 1) tc::commit(&dready[g]);
             }

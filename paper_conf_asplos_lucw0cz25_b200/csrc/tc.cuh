@@ -25,6 +25,14 @@ __device__ __forceinline__ uint64_t desc_sw32(uint32_t saddr, uint32_t lbo, uint
            ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (6ull << 61);
 }
 
+// 64-byte-swizzle descriptor (layout 4): rows of 64 bytes, 8-row atoms of 512 bytes (a TMA box with a
+// 64-byte inner dimension and CU_TENSOR_MAP_SWIZZLE_64B).  MN-major: lbo = stride between 64-element
+// MN blocks, sbo = between 8-row K groups.
+__device__ __forceinline__ uint64_t desc_sw64(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | (1ull << 46) | (4ull << 61);
+}
+
 // u8 x u8 -> s32, M x N tile, A K-major, B K-major (b_mn = false) or MN-major (b_mn = true)
 __host__ __device__ constexpr uint32_t idesc_u8(uint32_t M, uint32_t N, bool b_mn) {
     return (2u << 4) | (0u << 7) | (0u << 10) | ((b_mn ? 1u : 0u) << 16) | ((N >> 3) << 17) | ((M >> 4) << 24);
