@@ -773,7 +773,9 @@ def run_sumcheck(args, rank, world, local):
     from paper_conf_asplos_lucw0cz25_b200 import bzk
     torch.cuda.set_device(local)
     dist = None
-    if world > 1:
+    # BZK_DIST_FORCE=1 (under torchrun): the process group, the max-over-ranks timing and the gather of
+    # the proofs to rank 0 run even at world size 1 (the NCCL path on a one-GPU box)
+    if world > 1 or (os.environ.get("BZK_DIST_FORCE") == "1" and "RANK" in os.environ):
         import torch.distributed as dist
         backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
         if backend == "nccl":

@@ -564,89 +564,6 @@ __device__ __forceinline__ fe fixmul_lz(const fe &x, const fe *K, uint32_t zmask
     return r;
 }
 
-// Two fixed-multiplier products with the same table (the lo / hi folds of one table's pair group): the
-// rows of both run in lockstep on one set of K_i loads, so the two carry chains interleave (the
-// single-product chain is latency-bound: "wait" stalls dominate the fused rounds, ncu r02y).
-__device__ __forceinline__ void fm_row0(uint32_t A[9], uint32_t B[9], const uint32_t k[8], uint32_t x0) {
-    asm("mul.lo.u32 %0, %9,  %13;\n\t"
-        "mul.hi.u32 %1, %9,  %13;\n\t"
-        "mul.lo.u32 %2, %10, %13;\n\t"
-        "mul.hi.u32 %3, %10, %13;\n\t"
-        "mul.lo.u32 %4, %11, %13;\n\t"
-        "mul.hi.u32 %5, %11, %13;\n\t"
-        "mul.lo.u32 %6, %12, %13;\n\t"
-        "mul.hi.u32 %7, %12, %13;\n\t"
-        "mov.u32    %8, 0;"
-        : "=r"(A[0]), "=r"(A[1]), "=r"(A[2]), "=r"(A[3]), "=r"(A[4]), "=r"(A[5]), "=r"(A[6]), "=r"(A[7]),
-          "=r"(A[8])
-        : "r"(k[0]), "r"(k[2]), "r"(k[4]), "r"(k[6]), "r"(x0));
-    asm("mul.lo.u32 %0, %9,  %13;\n\t"
-        "mul.hi.u32 %1, %9,  %13;\n\t"
-        "mul.lo.u32 %2, %10, %13;\n\t"
-        "mul.hi.u32 %3, %10, %13;\n\t"
-        "mul.lo.u32 %4, %11, %13;\n\t"
-        "mul.hi.u32 %5, %11, %13;\n\t"
-        "mul.lo.u32 %6, %12, %13;\n\t"
-        "mul.hi.u32 %7, %12, %13;\n\t"
-        "mov.u32    %8, 0;"
-        : "=r"(B[0]), "=r"(B[1]), "=r"(B[2]), "=r"(B[3]), "=r"(B[4]), "=r"(B[5]), "=r"(B[6]), "=r"(B[7]),
-          "=r"(B[8])
-        : "r"(k[1]), "r"(k[3]), "r"(k[5]), "r"(k[7]), "r"(x0));
-}
-
-// two Montgomery word steps (divide by 2^64) and the final column add of fixmul_lz
-__device__ __forceinline__ fe fm_finish(uint32_t A[9], uint32_t B[9]) {
-    uint32_t L = 0;
-#pragma unroll
-    for (int s = 0; s < 2; ++s) {
-        if (s > 0) add_l(A, L);
-        const uint32_t m = mont_m(A[0]);
-        red_a(A, m);
-        red_b(B, m);
-        L = A[1];
-        uint32_t nA[9], nB[9];
-#pragma unroll
-        for (int q = 0; q < 9; ++q) nA[q] = B[q];
-#pragma unroll
-        for (int q = 0; q < 7; ++q) nB[q] = A[q + 2];
-        nB[7] = 0;
-        nB[8] = 0;
-#pragma unroll
-        for (int q = 0; q < 9; ++q) { A[q] = nA[q]; B[q] = nB[q]; }
-    }
-    fe r;   // A + L + (B << 32) < 2^255: A8, B7, B8 are zero
-    asm("add.cc.u32  %0, %8,  %16;\n\t"
-        "addc.cc.u32 %1, %9,  %17;\n\t"
-        "addc.cc.u32 %2, %10, %18;\n\t"
-        "addc.cc.u32 %3, %11, %19;\n\t"
-        "addc.cc.u32 %4, %12, %20;\n\t"
-        "addc.cc.u32 %5, %13, %21;\n\t"
-        "addc.cc.u32 %6, %14, %22;\n\t"
-        "addc.u32    %7, %15, %23;"
-        : "=r"(r.l[0]), "=r"(r.l[1]), "=r"(r.l[2]), "=r"(r.l[3]), "=r"(r.l[4]), "=r"(r.l[5]), "=r"(r.l[6]),
-          "=r"(r.l[7])
-        : "r"(A[0]), "r"(A[1]), "r"(A[2]), "r"(A[3]), "r"(A[4]), "r"(A[5]), "r"(A[6]), "r"(A[7]),
-          "r"(L), "r"(B[0]), "r"(B[1]), "r"(B[2]), "r"(B[3]), "r"(B[4]), "r"(B[5]), "r"(B[6]));
-    return r;
-}
-
-__device__ __forceinline__ void fixmul2_lz(const fe &x, const fe &y, const fe *K, uint32_t zmask, fe &rx, fe &ry) {
-    uint32_t A[9], B[9], C[9], E[9], k[8];
-    lds_k(k, K, x.l[0], zmask);
-    fm_row0(A, B, k, x.l[0]);
-    fm_row0(C, E, k, y.l[0]);
-#pragma unroll
-    for (int i = 1; i < 8; ++i) {
-        lds_k(k, K + i, A[0] ^ C[0], zmask);
-        row_a(A, k, x.l[i]);
-        row_b_nl(B, k, x.l[i]);
-        row_a(C, k, y.l[i]);
-        row_b_nl(E, k, y.l[i]);
-    }
-    rx = fm_finish(A, B);
-    ry = fm_finish(C, E);
-}
-
 // (x*y + u*v) * R^{-1} mod p, canonical; x, y, u, v canonical (result of the lazy form < 3p)
 __device__ __forceinline__ fe mont_mul2(const fe &x, const fe &y, const fe &u, const fe &v) {
     return fe_reduce_once(fe_reduce_once(mont_mul2_lz(x, y, u, v)));

@@ -279,20 +279,8 @@ __device__ __forceinline__ fe fold_fx(const fe &a, const fe &b, const fe *K, uin
     return lz_red(lz_add(a, fixmul_lz(lz_sub(b, a), K, zmask)));
 }
 
-// both folds of a pair group (a0, b0) -> lo, (a1, b1) -> hi with one table walk (fixmul2_lz)
-__device__ __forceinline__ void fold_fx2(const fe &a0, const fe &b0, const fe &a1, const fe &b1, const fe *K,
-                                         uint32_t zmask, fe &lo, fe &hi) {
-    fe p0, p1;
-    fixmul2_lz(lz_sub(b0, a0), lz_sub(b1, a1), K, zmask, p0, p1);
-    lo = lz_red(lz_add(a0, p0));
-    hi = lz_red(lz_add(a1, p1));
-}
-
 // fused-round folds use the per-(proof, round) table K_i = r 2^(32i+64) (fixmul_lz)
 #define BZK_FOLD(a, b) fold_fx(a, b, sK, zmask)
-#ifndef BZK_FOLD2
-#define BZK_FOLD2 0   // 1: the two folds of a pair group in lockstep (fixmul2_lz)
-#endif
 
 // ---------------------------------------------------------------- per-round finalisation
 
@@ -487,12 +475,8 @@ __device__ __forceinline__ void fold_group(const fe (&x)[Geo<ORDER, FIRST>::E], 
         lo = x[0];
         hi = x[1];
     } else {
-        if (BZK_FOLD2) {
-            fold_fx2(x[0], x[1], x[2], x[3], sK, zmask, lo, hi);
-        } else {
-            lo = BZK_FOLD(x[0], x[1]);
-            hi = BZK_FOLD(x[2], x[3]);
-        }
+        lo = BZK_FOLD(x[0], x[1]);
+        hi = BZK_FOLD(x[2], x[3]);
         fe *U = dst + (size_t)m * (2 * h);
         if (ORDER == 0) { st_fe(U + 2 * j, lo); st_fe(U + 2 * j + 1, hi); }
         else            { st_fe(U + j, lo);     st_fe(U + j + h, hi); }
