@@ -17,8 +17,9 @@ def kind_of(name):
         return "small_cluster"
     if "k_round1_tc" in name:
         return "round1_eval"
-    if "k_fused_tc" in name:
-        return "fused_fold_eval"
+    if "k_fused_tc" in name:   # k_fused_tc<D, ORDER, FIRST, NW>
+        first = name.split("<", 1)[1].split(">")[0].split(",")[2].strip()
+        return "round1_eval" if first in ("1", "true") else "fused_fold_eval"
     args = name.split("<", 1)[1].split(">")[0].split(",")      # k_round<D, ORDER, FIRST, TMA>, k_gl_round<D, ORDER, FIRST>
     first = args[2].strip()
     return "round1_eval" if first in ("1", "true") else "fused_fold_eval"
