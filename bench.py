@@ -74,6 +74,20 @@ SMS = 148
 IMAD_PER_MULMOD = 272
 
 
+def init_pg_quiet(dist, backend, **kw):
+    """init_process_group with the process's stdout pointed at stderr: NCCL prints its version banner
+    (NCCL_DEBUG=VERSION) to fd 1 at communicator creation, and stdout carries only the JSON line"""
+    sys.stdout.flush()
+    saved = os.dup(1)
+    try:
+        os.dup2(2, 1)
+        dist.init_process_group(backend, **kw)
+    finally:
+        sys.stdout.flush()
+        os.dup2(saved, 1)
+        os.close(saved)
+
+
 def peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
@@ -403,7 +417,7 @@ def run_merkle(args, rank, world):
         import torch.distributed as dist
         backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            init_pg_quiet(dist, "nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
     B, mode, n, _, _, desc = CONFIGS[args.config]
@@ -544,7 +558,7 @@ def run_encoder(args, rank, world):
         import torch.distributed as dist
         backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            init_pg_quiet(dist, "nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
     B, _, log_n, _, _, desc = CONFIGS[args.config]
@@ -779,7 +793,7 @@ def run_sumcheck(args, rank, world, local):
         import torch.distributed as dist
         backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            init_pg_quiet(dist, "nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
 
@@ -967,7 +981,8 @@ def run_sumcheck(args, rank, world, local):
                                    "launch / CUDA-event launch time"}
     roofline.update({"alg_bytes_per_launch": bytes_per_launch, "imad_slots_per_launch": slots_per_launch,
                      "alu_time_at_peak_ms": round(t_alu * 1000, 4), "hbm_time_at_peak_ms": round(t_hbm * 1000, 4),
-                     "imad_frac": round(ach_slots / slot_peak, 4), "hbm_frac": round(ach_gbs / hbm_peak, 4),
+                     # (Goldilocks: 64-bit products, not the BN254 slot counts of imad_slots)
+                     "imad_frac": None if gl else round(ach_slots / slot_peak, 4), "hbm_frac": round(ach_gbs / hbm_peak, 4),
                      "mulmod_equiv": {"achieved": round(mulmod_rate, 2), "peak": round(int_peak, 2),
                                       "unit": "Gmulmod/s (272-slot schoolbook unit, r01)",
                                       "frac": round(mulmod_rate / int_peak, 4)},
@@ -1074,7 +1089,7 @@ def run_chain(args, rank, world, local):
         import torch.distributed as dist
         backend = os.environ.get("BZK_DIST_BACKEND", "nccl")
         if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            init_pg_quiet(dist, "nccl", device_id=torch.device("cuda", local))
         else:
             dist.init_process_group(backend)
     B, d, k, order, _, desc = CONFIGS[args.config]

@@ -259,7 +259,8 @@ bool ftc_small(uint32_t D, uint32_t i, uint64_t h) {
 
 // CTAs per proof of global round i (h pairs): k_round1_tc / k_fused_tc (<= 32768 pairs per CTA: its
 // s32 accumulator bound) / k_round
-uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb) {
+uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb, bool gl) {
+    if (gl) return ctas_for(h, nb);   // k_gl_round (Goldilocks: no tensor-core variants)
     if (i == 1 && r1_use_tc(D, h)) return r1tc_ctas(h, nb);
     if (ftc_small(D, i, h)) return (uint32_t)std::max<uint64_t>(1, h / 2048);
     uint32_t c = ctas_for(h, nb);
@@ -267,9 +268,9 @@ uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb) {
     return c;
 }
 
-uint32_t max_round_ctas(uint32_t D, uint32_t k, uint32_t i0, uint64_t nb) {
+uint32_t max_round_ctas(uint32_t D, uint32_t k, uint32_t i0, uint64_t nb, bool gl) {
     uint32_t c = 1;
-    for (uint32_t i = 1; i < i0; ++i) c = std::max(c, round_ctas(D, i, 1ull << (k - i), nb));
+    for (uint32_t i = 1; i < i0; ++i) c = std::max(c, round_ctas(D, i, 1ull << (k - i), nb, gl));
     return c;
 }
 
@@ -397,7 +398,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
     auto per_proof = [&](uint64_t bw) -> size_t {
         (void)bw;
         size_t s = std::max(sizeof(ProofState), sizeof(gl::State)) + 4;
-        uint32_t c = P.k ? (P.multi ? max_multi_ctas(P.k, P.i0, bw) : max_round_ctas(P.D, P.k, P.i0, bw)) : 1;
+        uint32_t c = P.k ? (P.multi ? max_multi_ctas(P.k, P.i0, bw) : max_round_ctas(P.D, P.k, P.i0, bw, P.gl)) : 1;
         s += (size_t)c * P.part_nv * P.esz;
         if (P.need_bufX) s += (size_t)P.D * (P.N / 2) * P.esz;
         if (P.need_bufY && !P.bufY_alias_input) s += (size_t)P.D * (P.N / 4) * P.esz;
@@ -419,7 +420,7 @@ bzk_status make_plan(bzk_ctx *ctx, const bzk_batch *b, Plan &P) {
              small_cs_log(P.D, P.k, P.B) < 0;
     if (P.dual) { nw = 2; bw = (P.B + 1) / 2; }   // two waves of B/2: the same scratch as one wave of B
     P.Bw = bw; P.nwaves = nw;
-    P.cmax = P.k ? std::max(max_round_ctas(P.D, P.k, P.i0, bw), max_round_ctas(P.D, P.k, P.i0, P.B - (nw - 1) * bw)) : 1;
+    P.cmax = P.k ? std::max(max_round_ctas(P.D, P.k, P.i0, bw, P.gl), max_round_ctas(P.D, P.k, P.i0, P.B - (nw - 1) * bw, P.gl)) : 1;
     if (P.multi) P.cmax = std::max(max_multi_ctas(P.k, P.i0, bw), max_multi_ctas(P.k, P.i0, P.B - (nw - 1) * bw));
 
     size_t off = 0;
@@ -642,7 +643,7 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
         gl::RoundParams rp;
         memset(&rp, 0, sizeof rp);
         rp.log_h = k - i; rp.round = i; rp.k = k; rp.order = P.order; rp.given = P.given;
-        rp.ctas = ctas_for(1ull << rp.log_h, io.nb);
+        rp.ctas = round_ctas(D, i, 1ull << rp.log_h, io.nb, true);   // the partials are sized with the same count
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = (uint64_t *)io.round_evals; rp.challenges = (uint64_t *)io.challenges;
         rp.claims = (uint64_t *)io.claims;
@@ -651,6 +652,8 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
             rp.src = (i == 2) ? tab : ((i - 1) % 2 == 0 ? bufX : bufY);
             rp.dst = (i % 2 == 0) ? bufX : bufY;
         }
+        if (rp.ctas > P.cmax)   // the per-CTA partials are sized for P.cmax CTAs per proof (round_ctas)
+            return fail(ctx, BZK_ECUDA, "internal: round CTA count above the partials' sizing");
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
         cudaError_t e = gl_launch_round(D, P.order, i == 1, grid, kThreads, s, rp);
@@ -797,7 +800,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         memset(&tm, 0, sizeof tm);
         const bool r1tc = i == 1 && r1_use_tc(D, h), ftc = ftc_use(D, i);
         if (r1tc || ftc) {
-            rp.ctas = round_ctas(D, i, h, io.nb);
+            rp.ctas = round_ctas(D, i, h, io.nb, false);
             rp.cluster = 1;
         }
         if (r1tc && !make_r1_map(&tm, P.order, tab, h, io.nb * D))
@@ -809,6 +812,8 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
             if (!make_row_map(&tm, rp.src, io.nb * D * E * h / 4, box))
                 return fail(ctx, BZK_ECUDA, "cuTensorMapEncodeTiled failed (TMA staging)");
         }
+        if (rp.ctas > P.cmax)   // the per-CTA partials are sized for P.cmax CTAs per proof (round_ctas)
+            return fail(ctx, BZK_ECUDA, "internal: round CTA count above the partials' sizing");
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         {
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);

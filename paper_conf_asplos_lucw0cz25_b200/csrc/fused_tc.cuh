@@ -89,6 +89,8 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
     __shared__ __align__(16) fe sK[8];
     extern __shared__ uint8_t ft_raw[];
     uint8_t *base = ft_raw + ((1024 - (smem_u32(ft_raw) & 1023)) & 1023);
+    BZK_ASSERT((size_t)(base - ft_raw) + (size_t)NW * (D * G::SLOT + FG::TILE) <= dyn_smem_bytes() &&
+               (size_t)NV * 32 * 33 * 4 <= (size_t)NW * D * G::SLOT);
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t h = 1ull << P.log_h;
     const uint64_t stride = (uint64_t)P.ctas * kFtCompute;
@@ -125,6 +127,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
                 tma_issue<ORDER, FIRST>(&tmap, wslots + m * G::SLOT, &wbars[m], row0 + m * trows, h, j0);
         const uint32_t sw = (lane >> 2) & 1, o0 = lane * 32 + (sw << 4), o1 = lane * 32 + ((1 - sw) << 4);
         auto put = [&](int v, const fe &x) {
+            BZK_ASSERT((uint32_t)v * 1024 + 1024 <= FG::TILE);
             *reinterpret_cast<uint4 *>(tile + v * 1024 + o0) = make_uint4(x.l[0], x.l[1], x.l[2], x.l[3]);
             *reinterpret_cast<uint4 *>(tile + v * 1024 + o1) = make_uint4(x.l[4], x.l[5], x.l[6], x.l[7]);
         };

@@ -49,6 +49,7 @@ __global__ void __launch_bounds__(tc_threads(EG), 1) k_multi_tc(MultiParams P, c
     uint8_t *stage0 = base;                                    // [stage][z][128 rows][32 B], swizzled
     uint8_t *opB = base + kTcStages * 32768;                   // [z][64 rows n][32 B], swizzled
     uint8_t *ones = opB + 16384;                               // 128 x 32 bytes of 1
+    BZK_ASSERT((size_t)(ones + 4096 - tc_raw) <= dyn_smem_bytes());
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
     multi_weights<ORDER, M>(P, b, s_r, s_w);

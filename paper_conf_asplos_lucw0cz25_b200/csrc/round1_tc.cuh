@@ -54,6 +54,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
     __shared__ unsigned long long s_diag[4][64];   // blocks aa, ab, ba, bb
     extern __shared__ uint8_t r1_raw[];
     uint8_t *base = r1_raw + ((1024 - (tc::su32(r1_raw) & 1023)) & 1023);
+    BZK_ASSERT((size_t)(base - r1_raw) + (size_t)NS * kR1Stage <= dyn_smem_bytes());
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t h = 1ull << P.log_h;
     const uint32_t T = (uint32_t)(h / kR1Tile);
@@ -83,6 +84,7 @@ __global__ void __launch_bounds__(kR1Threads, 1) k_round1_tc(RoundParams P, cons
                 const uint32_t s = it % NS;
                 if (it >= (uint32_t)NS) tc::mbar_wait(&empty[s], ((it / NS) - 1) & 1);
                 const int j0 = (int)((blockIdx.x + it * P.ctas) * kR1Tile);
+                BZK_ASSERT((uint64_t)j0 + kR1Tile <= h);
                 uint8_t *st = base + s * kR1Stage;
                 tc::mbar_tx(&full[s], kR1Stage);
 #pragma unroll

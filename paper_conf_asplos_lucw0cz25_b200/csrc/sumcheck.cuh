@@ -36,6 +36,16 @@
 #endif
 #include "sha256.cuh"
 
+// BZK_CHECK builds (scripts/gpu_r02chk.sh; compute-sanitizer is closed on the GPU pool): device-side
+// asserts on the hot path's indices -- pair index within the round, partial slot within the proof's
+// CTAs, shared-memory tiles and slots within the launch's dynamic shared memory.  A failed check traps
+// (the call returns BZK_ECUDA).  Compiled out otherwise.
+#ifdef BZK_CHECK
+#define BZK_ASSERT(...) do { if (!(__VA_ARGS__)) __trap(); } while (0)
+#else
+#define BZK_ASSERT(...) do { } while (0)
+#endif
+
 namespace bzk {
 
 struct ProofState {
@@ -478,6 +488,7 @@ __device__ __forceinline__ void fold_group(const fe (&x)[Geo<ORDER, FIRST>::E], 
         lo = BZK_FOLD(x[0], x[1]);
         hi = BZK_FOLD(x[2], x[3]);
         fe *U = dst + (size_t)m * (2 * h);
+        BZK_ASSERT(j < h);
         if (ORDER == 0) { st_fe(U + 2 * j, lo); st_fe(U + 2 * j + 1, hi); }
         else            { st_fe(U + j, lo);     st_fe(U + j + h, hi); }
     }
@@ -528,6 +539,11 @@ constexpr size_t tma_smem_bytes() {   // + 1 KiB: the dynamic base is aligned up
 }
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ uint32_t dyn_smem_bytes() {
+    uint32_t r;
+    asm("mov.u32 %0, %%dynamic_smem_size;" : "=r"(r));
+    return r;
+}
 
 __device__ __forceinline__ void mbar_init(uint64_t *bar) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
@@ -572,6 +588,7 @@ __device__ __forceinline__ fe tma_entry(const uint8_t *slot, uint32_t lane, int 
     } else {
         seg = e; row = lane >> 2; c0 = 2 * (lane & 3);
     }
+    BZK_ASSERT((seg + 1) * 1024 <= TmaGeo<ORDER, FIRST>::SLOT && row < 8 * (ORDER == 0 ? TmaGeo<ORDER, FIRST>::E : 1));
     const uint8_t *base = slot + seg * 1024 + row * 128;
     const uint4 x = *reinterpret_cast<const uint4 *>(base + ((c0 ^ (row & 7)) << 4));
     const uint4 y = *reinterpret_cast<const uint4 *>(base + (((c0 + 1) ^ (row & 7)) << 4));
@@ -628,6 +645,7 @@ __device__ __forceinline__ void round_finish(const RoundParams &P, uint32_t b, f
         if (!leader) return;
     }
     const uint32_t nparts = P.ctas / cs, pidx = blockIdx.x / cs;
+    BZK_ASSERT(pidx < nparts && blockIdx.x < P.ctas);
     fe *part = P.partials + (size_t)b * P.ctas * NV;
     if (threadIdx.x == 0) {
 #pragma unroll

@@ -189,10 +189,11 @@ print("tc ok")
 
 
 @pytest.mark.parametrize("env", [{"BZK_TC_CTAS": "1"}, {"BZK_TC_CTAS": "7"}, {"BZK_TC_CTAS": "1000"},
-                                 {"BZK_MULTI_TC": "0"}])
+                                 {"BZK_MULTI_TC": "0"}, {"BZK_MULTI_M": "1"}, {"BZK_MULTI_M": "2"}])
 def test_multiround_tc_launch_shapes(env):
     """k_multi_tc with one CTA per proof, 7 CTAs (ragged: 64 tiles -> 10 / 9 per CTA, last-CTA ticket), one
-    CTA per tile, and the CUDA-core k_multi instead (BZK_MULTI_TC=0); k_small off so every case runs the passes."""
+    CTA per tile, and the CUDA-core k_multi instead (BZK_MULTI_TC=0); passes of 1 and 2 rounds (BZK_MULTI_M, the
+    CUDA-core k_multi: k_multi_tc takes 3-round passes only); k_small off so every case runs the passes."""
     import os
     import subprocess
     import sys

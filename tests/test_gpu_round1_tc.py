@@ -102,12 +102,15 @@ print("r1tc ok")
 
 @pytest.mark.parametrize("env", [{"BZK_R1TC_CTAS": "1"}, {"BZK_R1TC_CTAS": "7"}, {"BZK_R1TC_CTAS": "100000"},
                                  {"BZK_R1_TC": "0"}, {"BZK_FTC_SMALL_LOG": "0"}, {"BZK_FTC_SMALL_LOG": "17"},
-                                 {"BZK_R1_SW64": "0"}, {"BZK_R1_SW64": "0", "BZK_R1TC_CTAS": "7"}])
+                                 {"BZK_R1_SW64": "0"}, {"BZK_R1_SW64": "0", "BZK_R1TC_CTAS": "7"},
+                                 {"BZK_FUSED_TC": "0", "BZK_R1_TC": "0"}, {"BZK_FUSED_TC": "0", "BZK_TMA": "0"},
+                                 {"BZK_FUSED_TC": "0", "BZK_R1_TC": "0", "BZK_TMA": "1"}])
 def test_round1_tc_launch_shapes(env):
     """one CTA per proof, 7 CTAs (ragged: 256 tiles -> 37 / 36 per CTA), one CTA per tile, and the
     CUDA-core round 1 (BZK_R1_TC=0); the 2-warp k_fused_tc of the late d = 2 rounds off, and on for
     every fused round (several CTAs per proof); LSB round 1 from separate a / b boxes of 32-byte rows
-    instead of one box of 64-byte (a | b) rows"""
+    instead of one box of 64-byte (a | b) rows; the CUDA-core k_round for round 1 and the fused rounds
+    (BZK_FUSED_TC=0, BZK_R1_TC=0) with its TMA staging at the default, off and forced on"""
     r = subprocess.run([sys.executable, "-c", SCRIPT.format(root=ROOT)], env=dict(os.environ, **env),
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "r1tc ok" in r.stdout, r.stdout + r.stderr
