@@ -142,7 +142,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
                 fe x[G::E];
 #pragma unroll
                 for (int e = 0; e < G::E; ++e) x[e] = tma_entry<ORDER, FIRST>(slot, lane, e);
-                fold_group<D, ORDER, FIRST>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
+                fold_group<D, ORDER, FIRST, D == 2>(x, m, dst, h, j, sK, P.zero, a[m], sv[m]);
                 __syncwarp();                  // every lane has consumed the slot
                 if (lane == 0 && jw + stride < h)
                     tma_issue<ORDER, FIRST>(&tmap, slot, &wbars[m], row0 + m * trows, h, jw + stride);

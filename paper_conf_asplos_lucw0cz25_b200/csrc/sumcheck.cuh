@@ -477,7 +477,9 @@ __device__ __forceinline__ uint64_t raw_off(uint64_t h, uint64_t j, int e) {
 
 // From the raw entries x[] of table m: round 1 -> (a, b); fused round -> fold both pairs with
 // r_{i-1}, store the folded pair to the other ping-pong buffer (Fig. 5), return (a, b - a).
-template <int D, int ORDER, bool FIRST>
+// RAWD: the delta only feeds a tensor-core sum (k_fused_tc<2>), where any operand < 2^256 is exact, so
+// it stays b + 2p - a < 4p for every table (no lz_red)
+template <int D, int ORDER, bool FIRST, bool RAWD = false>
 __device__ __forceinline__ void fold_group(const fe (&x)[Geo<ORDER, FIRST>::E], int m, fe *dst, uint64_t h,
                                            uint64_t j, const fe *sK, uint32_t zmask, fe &a, fe &sv) {
     fe lo, hi;
@@ -495,7 +497,7 @@ __device__ __forceinline__ void fold_group(const fe (&x)[Geo<ORDER, FIRST>::E], 
     a = lo;
     // round 1: b; fused rounds: delta (for d = 2 the table-0 delta may stay < 4p: it only
     // meets mul_acc, a full 512-bit product < 8p^2)
-    sv = FIRST ? hi : ((D == 2 && m == 0) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
+    sv = FIRST ? hi : ((RAWD || (D == 2 && m == 0)) ? lz_sub(hi, lo) : lz_red(lz_sub(hi, lo)));
 }
 
 template <int D, int ORDER, bool FIRST>
