@@ -206,7 +206,12 @@ struct Knobs {
     // BZK_R1_SW64=0/1: LSB round 1 of k_round1_tc loads each table's pairs as 64-byte rows (a_j | b_j), one
     // TMA box per table, 64-byte swizzle; 0: a and b as separate boxes of 32-byte rows
     uint32_t r1_sw64 = 1;
+    // BZK_SMALL_ROUND_LOG=L: the CUDA-core global rounds without TMA staging (k_round d = 1, k_gl_round)
+    // with h <= 2^L pairs per proof run CTAs of 64 threads, one per 2048 pairs (as the 2-warp k_fused_tc);
+    // 0 = off
+    uint32_t small_round_log = 12;
     Knobs() {
+        if (const char *e = getenv("BZK_SMALL_ROUND_LOG")) small_round_log = (uint32_t)std::max(0, atoi(e));
         if (const char *e = getenv("BZK_R1_SW64")) r1_sw64 = atoi(e) ? 1 : 0;
         if (const char *e = getenv("BZK_FTC_SMALL_LOG")) ftc_small_log = (uint32_t)std::max(0, atoi(e));
         if (const char *e = getenv("BZK_D3_TC")) d3tc = atoi(e) ? 1 : 0;
@@ -257,9 +262,17 @@ bool ftc_small(uint32_t D, uint32_t i, uint64_t h) {
     return ftc_use(D, i) && D == 2 && knobs().ftc_small_log && h <= (1ull << knobs().ftc_small_log);
 }
 
+// the 64-thread CTAs of the late CUDA-core rounds (BZK_SMALL_ROUND_LOG)
+constexpr uint32_t kSmallRoundThreads = 64;
+bool small_round(uint32_t D, uint32_t i, uint64_t h, bool gl) {
+    if (i < 2 || !knobs().small_round_log || h > (1ull << knobs().small_round_log)) return false;
+    return gl || (!ftc_use(D, i) && !knobs().tma_for(D, false));
+}
+
 // CTAs per proof of global round i (h pairs): k_round1_tc / k_fused_tc (<= 32768 pairs per CTA: its
 // s32 accumulator bound) / k_round
 uint32_t round_ctas(uint32_t D, uint32_t i, uint64_t h, uint64_t nb, bool gl) {
+    if (small_round(D, i, h, gl)) return (uint32_t)std::max<uint64_t>(1, h / 2048);
     if (gl) return ctas_for(h, nb);   // k_gl_round (Goldilocks: no tensor-core variants)
     if (i == 1 && r1_use_tc(D, h)) return r1tc_ctas(h, nb);
     if (ftc_small(D, i, h)) return (uint32_t)std::max<uint64_t>(1, h / 2048);
@@ -497,13 +510,13 @@ bzk_status ensure_stage(bzk_ctx *ctx, size_t bytes) {
 
 // ---------------------------------------------------------------- kernel dispatch
 
-cudaError_t dispatch_round(uint32_t D, uint32_t order, bool first, dim3 grid, cudaStream_t s,
+cudaError_t dispatch_round(uint32_t D, uint32_t order, bool first, dim3 grid, uint32_t threads, cudaStream_t s,
                            const RoundParams &p, const CUtensorMap &tm) {
     switch (D) {
-        case 1: return launch_round<1>(order, first, grid, kRoundThreads, s, p, tm);
-        case 2: return launch_round<2>(order, first, grid, kRoundThreads, s, p, tm);
-        case 3: return launch_round<3>(order, first, grid, kRoundThreads, s, p, tm);
-        case 4: return launch_round<4>(order, first, grid, kRoundThreads, s, p, tm);
+        case 1: return launch_round<1>(order, first, grid, threads, s, p, tm);
+        case 2: return launch_round<2>(order, first, grid, threads, s, p, tm);
+        case 3: return launch_round<3>(order, first, grid, threads, s, p, tm);
+        case 4: return launch_round<4>(order, first, grid, threads, s, p, tm);
     }
     return cudaErrorInvalidValue;
 }
@@ -656,7 +669,8 @@ bzk_status run_wave_gl(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream
             return fail(ctx, BZK_ECUDA, "internal: round CTA count above the partials' sizing");
         dim3 grid(rp.ctas, (uint32_t)io.nb);
         ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
-        cudaError_t e = gl_launch_round(D, P.order, i == 1, grid, kThreads, s, rp);
+        cudaError_t e = gl_launch_round(D, P.order, i == 1, grid,
+                                        small_round(D, i, 1ull << rp.log_h, true) ? kSmallRoundThreads : kThreads, s, rp);
         ++ctx->launches;
         if (e != cudaSuccess) return cuda_fail(ctx, e, "k_gl_round launch");
     }
@@ -785,7 +799,7 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
         rp.log_h = k - i;
         rp.round = i; rp.k = k; rp.order = P.order;
         const uint64_t h = 1ull << rp.log_h;
-        rp.ctas = ctas_for(h, io.nb);
+        rp.ctas = round_ctas(D, i, h, io.nb, false);
         rp.partials = part; rp.tickets = tick; rp.ps = ps;
         rp.round_evals = (fe *)io.round_evals; rp.challenges = (fe *)io.challenges; rp.claims = (fe *)io.claims;
         rp.consts = ctx->consts;
@@ -819,7 +833,9 @@ bzk_status run_wave(bzk_ctx *ctx, const Plan &P, const WaveIO &io, cudaStream_t 
             ProfScope ps_(ctx, s, i == 1 ? 0 : 1);
             cudaError_t e = r1tc  ? r1tc_launch(P.order, P.order == 0 && knobs().r1_sw64, grid, s, rp, tm)
                             : ftc ? ftc_launch(D, i == 1, ftc_small(D, i, h), P.order, grid, s, rp, tm)
-                                  : dispatch_round(D, P.order, i == 1, grid, s, rp, tm);
+                                  : dispatch_round(D, P.order, i == 1, grid,
+                                                   small_round(D, i, h, false) ? kSmallRoundThreads : kRoundThreads,
+                                                   s, rp, tm);
             ++ctx->launches;
             if (e != cudaSuccess) return cuda_fail(ctx, e, "k_round launch");
         }
