@@ -726,8 +726,11 @@ def imad_slots(d: int, k: int, kind: str, gl: bool = False) -> int:
     point = 0 if d == 1 else (d - 2) * SLOT_MONT + SLOT_MULACC
     if kind == "round1":
         # k_fused_tc<3, ., 1>: x0(t) x1(t) is a quadratic in t, so its t = 2 value is derived from t = 0, 1, inf
-        npts = d if (tc1 and d == 3) else d + 1
-        return npts * (point - (SLOT_MULACC if tc1 else 0)) * (1 << (k - 1)) if i0 > 1 else 0
+        # and its x0(t) x1(t) are unreduced 512-bit products (64 limb products, SLOT_MULACC) summed on the
+        # tensor cores
+        if tc1 and d == 3:
+            return d * SLOT_MULACC * (1 << (k - 1)) if i0 > 1 else 0
+        return (d + 1) * (point - (SLOT_MULACC if tc1 else 0)) * (1 << (k - 1)) if i0 > 1 else 0
     if kind == "fused":
         pf = point - (SLOT_MULACC if tcf else 0)
         return sum((2 * d * SLOT_FIXMUL + d * pf) * (1 << (k - i)) for i in range(2, i0))

@@ -52,7 +52,11 @@ constexpr uint64_t kFtMaxPairs = 32768;            // pairs per CTA (s32 accumul
 template <int D, bool FIRST> struct FtGeo;
 template <> struct FtGeo<2, false> { static constexpr uint32_t TILE = 4096, BOFF = 2048, N = 64, TCOLS = 64; };
 template <> struct FtGeo<3, false> { static constexpr uint32_t TILE = 6144, BOFF = 3072, N = 96, TCOLS = 128; };
-template <> struct FtGeo<3, true> { static constexpr uint32_t TILE = 8192, BOFF = 4096, N = 128, TCOLS = 128; };
+// d = 3 round 1 ("wide"): X_t = x0(t) x1(t) UNREDUCED (512 bits = two 32-byte vectors, lo | hi), so the
+// integer pipe does 64 limb products per point instead of a Montgomery product's 136; vectors
+// 0..7 = X0 lo|hi, X1 lo|hi, X2 lo|hi, Xinf lo|hi, 8..11 = Y0, Y1, Y2, Yinf.  Two MMAs per tile into two
+// 64-column TMEM accumulators: (X0, X1) x (Y0 | Y1) and (X2, Xinf) x (Y2 | Yinf).
+template <> struct FtGeo<3, true> { static constexpr uint32_t TILE = 12288, BOFF = 8192, N = 64, TCOLS = 128; };
 
 template <int D, bool FIRST, int NW = ft_nw<D, FIRST>()>
 constexpr size_t ft_smem() {
@@ -90,7 +94,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
     extern __shared__ uint8_t ft_raw[];
     uint8_t *base = ft_raw + ((1024 - (smem_u32(ft_raw) & 1023)) & 1023);
     BZK_ASSERT((size_t)(base - ft_raw) + (size_t)NW * (D * G::SLOT + FG::TILE) <= dyn_smem_bytes() &&
-               (size_t)NV * 32 * 33 * 4 <= (size_t)NW * D * G::SLOT);
+               (size_t)(D == 3 && FIRST ? 8 : NV) * 32 * 33 * 4 <= (size_t)NW * D * G::SLOT);
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t h = 1ull << P.log_h;
     const uint64_t stride = (uint64_t)P.ctas * kFtCompute;
@@ -159,21 +163,48 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
 #pragma unroll
                 for (int m = 0; m < D; ++m) dl[m] = FIRST ? lz_red(lz_sub(sv[m], a[m])) : sv[m];
                 if constexpr (FIRST) {
-                    // x0(t) x1(t) is a quadratic in t: X_2 = 2 X_1 - X_0 + 2 X_inf (the same residue as the
-                    // Montgomery product at t = 2, without it): 3 products instead of 4; lazy bounds
-                    // X_t < 1.76p, (X_1 + X_inf) -> < 2p, doubled -> < 2p, + 2p - X_0 -> < 4p < 2^256
-                    fe X[NV];
+                    // x0(t) x1(t) is a quadratic in t, so X_2 = 2 X_1 + 2 X_inf - X_0 (+ 4p^2, a multiple of p
+                    // that keeps it non-negative): the same residue as x0(2) x1(2) with 3 products per pair.
+                    // Bounds: x_m(t) < 2p, so X_t < 4p^2 and X_2 < 14p^2 < 2^512.
+                    const uint32_t P4[16] = {0x80000004u, 0x230fac9fu, 0x72cd0000u, 0x1fc9888fu, 0xa326edffu,
+                                             0xffa698b1u, 0xa08776c3u, 0x9b3865d7u, 0x1ed8bf9eu, 0xb1dd49edu,
+                                             0x4de74f7cu, 0x17dceec3u, 0x0d234872u, 0x6669bdf0u, 0xd8f2fe71u,
+                                             0x249712e1u};   // 4 p^2
+                    uint32_t X2[16];
 #pragma unroll
                     for (int idx = 0; idx < NV; ++idx) {
-                        if (idx != 2) {
-                            X[idx] = mont_mul_lz(d3_point<DERIVE>(a[0], sv[0], dl[0], idx),
-                                                 d3_point<DERIVE>(a[1], sv[1], dl[1], idx));
-                            put(idx, X[idx]);
+                        put(8 + idx, d3_point<DERIVE>(a[2], sv[2], dl[2], idx));
+                        if (idx == 2) continue;
+                        acc17 W = acc17_zero();
+                        mul_acc(W, d3_point<DERIVE>(a[0], sv[0], dl[0], idx), d3_point<DERIVE>(a[1], sv[1], dl[1], idx));
+                        fe lo, hi;
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) { lo.l[q] = W.w[q]; hi.l[q] = W.w[8 + q]; }
+                        put(2 * idx, lo);
+                        put(2 * idx + 1, hi);
+                        if (idx == 0) {   // X2 = 4p^2 - X0
+                            int64_t br = 0;
+#pragma unroll
+                            for (int q = 0; q < 16; ++q) {
+                                const int64_t v = (int64_t)P4[q] - (int64_t)W.w[q] + br;
+                                X2[q] = (uint32_t)v;
+                                br = v >> 32;
+                            }
+                        } else {          // X2 += 2 X_1, 2 X_inf
+                            uint64_t c = 0;
+#pragma unroll
+                            for (int q = 0; q < 16; ++q) {
+                                c += (uint64_t)X2[q] + 2ull * W.w[q];
+                                X2[q] = (uint32_t)c;
+                                c >>= 32;
+                            }
                         }
-                        put(FG::BOFF / 1024 + idx, d3_point<DERIVE>(a[2], sv[2], dl[2], idx));
                     }
-                    const fe s1 = lz_red(lz_add(X[1], X[3]));
-                    put(2, lz_sub(lz_red(lz_add(s1, s1)), X[0]));
+                    fe lo, hi;
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) { lo.l[q] = X2[q]; hi.l[q] = X2[8 + q]; }
+                    put(4, lo);
+                    put(5, hi);
                 } else {
 #pragma unroll
                     for (int idx = 0; idx < NV; ++idx) {
@@ -210,8 +241,14 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
                 if (done[w] < nw[w] && tc::mbar_test(&tfull[w], done[w] & 1)) {
                     tc::fence_after();
                     const uint32_t t0 = tb + w * FG::TILE;
-                    tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + FG::BOFF, 1024, 256), idesc,
-                               !first);
+                    if constexpr (D == 3 && FIRST) {   // (X0 | X1) x (Y0 | Y1), (X2 | Xinf) x (Y2 | Yinf)
+                        tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + 8192, 1024, 256), idesc, !first);
+                        tc::mma_u8(tmem + 64, tc::desc_sw32(t0 + 4096, 1024, 256), tc::desc_sw32(t0 + 10240, 1024, 256),
+                                   idesc, !first);
+                    } else {
+                        tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + FG::BOFF, 1024, 256), idesc,
+                                   !first);
+                    }
                     first = false;
                     tc::commit(&tempty[w]);
                     ++done[w];
@@ -224,20 +261,28 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
         if (nmax > 0) tc::commit(&dfin);
     }
     __syncwarp();
-    // anti-diagonal sums of the NV diagonal blocks (warp t reads TMEM lanes 32t.., columns 32t..)
-    uint32_t *sM = reinterpret_cast<uint32_t *>(base);   // [NV][32][33] (reuses the TMA slots)
-    __shared__ unsigned long long s_diag[NV][64];
+    // anti-diagonal sums of the diagonal blocks (warp t reads TMEM lanes 32t.., columns 32t..; the wide
+    // d = 3 round 1 has NB = 8 blocks: warp q reads its quadrant of both accumulators)
+    constexpr bool WIDE = D == 3 && FIRST;
+    constexpr int NB = WIDE ? 8 : NV;
+    uint32_t *sM = reinterpret_cast<uint32_t *>(base);   // [NB][32][33] (reuses the TMA slots)
+    __shared__ unsigned long long s_diag[NB][64];
     const bool any = (uint64_t)blockIdx.x * kFtCompute < h;
     tc::fence_before();
     __syncthreads();
-    if (warp < (uint32_t)NV && any) {
+    if (warp < (uint32_t)(WIDE ? 4 : NV) && any) {
         tc::mbar_wait(&dfin, 0);
         tc::fence_after();
-        uint32_t v[32];
-        tc::ld_x32(tmem + ((warp * 32) << 16) + warp * 32, v);
-        tc::wait_ld();
 #pragma unroll
-        for (int i = 0; i < 32; ++i) sM[(warp * 32 + lane) * 33 + i] = v[i];   // row = byte `lane` of X_t
+        for (int g = 0; g < (WIDE ? 2 : 1); ++g) {
+            uint32_t v[32];
+            const uint32_t col = WIDE ? g * 64 + (warp >> 1) * 32 : warp * 32;
+            tc::ld_x32(tmem + ((warp * 32) << 16) + col, v);
+            tc::wait_ld();
+            const uint32_t blk = WIDE ? g * 4 + warp : warp;
+#pragma unroll
+            for (int i = 0; i < 32; ++i) sM[(blk * 32 + lane) * 33 + i] = v[i];   // row = byte `lane` of X_t
+        }
     }
     tc::fence_before();
     __syncthreads();
@@ -245,7 +290,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
         tc::fence_after();
         tc::tmem_dealloc<FG::TCOLS>(tmem);
     }
-    for (uint32_t q = threadIdx.x; q < NV * 64; q += blockDim.x) {   // NW = 2: fewer threads than sums
+    for (uint32_t q = threadIdx.x; q < NB * 64; q += blockDim.x) {   // NW = 2: fewer threads than sums
         const uint32_t t = q >> 6, n = q & 63;
         unsigned long long s = 0;
         if (any)
@@ -258,20 +303,62 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
 #pragma unroll
     for (int t = 0; t < NV; ++t) acc[t] = fe_zero();
     if (threadIdx.x < NV && any) {
-        acc17 S = acc17_zero();
-        for (int n = 0; n < 63; ++n) {   // add s_n 2^(8n) (s_n < 2^36)
-            const unsigned long long v = s_diag[threadIdx.x][n];
-            const int w0 = (8 * n) >> 5, sh = (8 * n) & 31;
-            uint64_t cur = (uint64_t)S.w[w0] + (uint32_t)(v << sh);
-            S.w[w0] = (uint32_t)cur;
-            uint64_t carry = (cur >> 32) + (sh ? (v >> (32 - sh)) : (v >> 32));
-            for (int w = w0 + 1; w < 17 && carry; ++w) {
-                cur = (uint64_t)S.w[w] + (uint32_t)carry;
-                S.w[w] = (uint32_t)cur;
-                carry = (carry >> 32) + (cur >> 32);
+        fe f;
+        if constexpr (WIDE) {
+            // S_t = sum_j X_t Y_t = B_lo + 2^256 B_hi (< 2^784, 25 words); partial = S_t R^-2 mod p (the
+            // Montgomery products of the narrow path carried one R^-1 each): 16 REDC word steps
+            const uint32_t Pw[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
+            uint32_t T[26];
+            for (int q = 0; q < 26; ++q) T[q] = 0;
+            for (int half = 0; half < 2; ++half)
+                for (int n = 0; n < 63; ++n) {   // add s_n 2^(8n + 256 half) (s_n < 2^36)
+                    const unsigned long long v = s_diag[2 * threadIdx.x + half][n];
+                    const int w0 = ((8 * n) >> 5) + 8 * half, sh = (8 * n) & 31;
+                    uint64_t cur = (uint64_t)T[w0] + (uint32_t)(v << sh);
+                    T[w0] = (uint32_t)cur;
+                    uint64_t carry = (cur >> 32) + (sh ? (v >> (32 - sh)) : (v >> 32));
+                    for (int w = w0 + 1; w < 26 && carry; ++w) {
+                        cur = (uint64_t)T[w] + (uint32_t)carry;
+                        T[w] = (uint32_t)cur;
+                        carry = (carry >> 32) + (cur >> 32);
+                    }
+                }
+            for (int i = 0; i < 16; ++i) {   // T += m p 2^(32 i) clears word i
+                const uint32_t m = T[i] * BZK_NP0;
+                uint64_t c = 0;
+                for (int j = 0; j < 8; ++j) {
+                    const uint64_t x = (uint64_t)m * Pw[j] + T[i + j] + c;
+                    T[i + j] = (uint32_t)x;
+                    c = x >> 32;
+                }
+                for (int j = i + 8; j < 26 && c; ++j) {
+                    const uint64_t x = (uint64_t)T[j] + c;
+                    T[j] = (uint32_t)x;
+                    c = x >> 32;
+                }
             }
+            // W = T[16..25] = (S + q p) / 2^512 < 2^272 + p:  W = lo + hi 2^256,  hi 2^256 = mont_mul(hi, R^2)
+            fe lo, hi = fe_zero();
+            for (int q = 0; q < 8; ++q) lo.l[q] = T[16 + q];
+            hi.l[0] = T[24];
+            hi.l[1] = T[25];
+            f = fe_add(fe_reduce_256(lo), mont_mul(hi, fe_const(2)));
+        } else {
+            acc17 S = acc17_zero();
+            for (int n = 0; n < 63; ++n) {   // add s_n 2^(8n) (s_n < 2^36)
+                const unsigned long long v = s_diag[threadIdx.x][n];
+                const int w0 = (8 * n) >> 5, sh = (8 * n) & 31;
+                uint64_t cur = (uint64_t)S.w[w0] + (uint32_t)(v << sh);
+                S.w[w0] = (uint32_t)cur;
+                uint64_t carry = (cur >> 32) + (sh ? (v >> (32 - sh)) : (v >> 32));
+                for (int w = w0 + 1; w < 17 && carry; ++w) {
+                    cur = (uint64_t)S.w[w] + (uint32_t)carry;
+                    S.w[w] = (uint32_t)cur;
+                    carry = (carry >> 32) + (cur >> 32);
+                }
+            }
+            f = acc17_to_fe(S);   // thread t: point t's partial (Pts<D, DERIVE> order)
         }
-        const fe f = acc17_to_fe(S);   // thread t: point t's partial (Pts<D, DERIVE> order)
 #pragma unroll
         for (int t = 0; t < NV; ++t)
             if (t == (int)threadIdx.x) acc[t] = f;
