@@ -732,7 +732,8 @@ def imad_slots(d: int, k: int, kind: str, gl: bool = False) -> int:
             return d * SLOT_MULACC * (1 << (k - 1)) if i0 > 1 else 0
         return (d + 1) * (point - (SLOT_MULACC if tc1 else 0)) * (1 << (k - 1)) if i0 > 1 else 0
     if kind == "fused":
-        pf = point - (SLOT_MULACC if tcf else 0)
+        # k_fused_tc<3, ., 0>: the x0(t) x1(t) products are unreduced 512-bit (64 limb products) too
+        pf = (d - 2) * SLOT_MULACC if (tcf and d == 3) else point - (SLOT_MULACC if tcf else 0)
         return sum((2 * d * SLOT_FIXMUL + d * pf) * (1 << (k - i)) for i in range(2, i0))
     passes = multi_passes(k, int(os.environ.get("BZK_MULTI_M", "3")))
     if kind == "multi":

@@ -35,7 +35,7 @@ namespace bzk {
 // dominated by the CTA's fixed costs and the proof's serial finalisation) run NW = 2: one CTA of 96
 // threads per proof (two above 2^11), 7 resident per SM (registers), so a 1024-proof wave is one
 // CTA wave instead of several.
-template <int D, bool FIRST> __host__ __device__ constexpr int ft_nw() { return D == 3 ? 12 : 8; }
+template <int D, bool FIRST> __host__ __device__ constexpr int ft_nw() { return D == 3 ? (FIRST ? 12 : 10) : 8; }
 constexpr int kFtSmallNW = 2;
 __host__ __device__ constexpr int ft_threads(int nw) { return 32 * nw + 32; }   // + the MMA warp
 __host__ __device__ constexpr int ft_minb(int D, int nw) { return D == 3 ? 1 : nw == kFtSmallNW ? 7 : 2; }
@@ -51,7 +51,9 @@ constexpr uint64_t kFtMaxPairs = 32768;            // pairs per CTA (s32 accumul
 // vector (those D rows are never read).
 template <int D, bool FIRST> struct FtGeo;
 template <> struct FtGeo<2, false> { static constexpr uint32_t TILE = 4096, BOFF = 2048, N = 64, TCOLS = 64; };
-template <> struct FtGeo<3, false> { static constexpr uint32_t TILE = 6144, BOFF = 3072, N = 96, TCOLS = 128; };
+// d = 3 fused rounds (wide): vectors 0..5 = X0 lo|hi, X2 lo|hi, Xinf lo|hi, 6..8 = Y0, Y2, Yinf; MMAs
+// (X0, X2) x (Y0 | Y2) (N = 64) and (Xinf, -) x Yinf (N = 32)
+template <> struct FtGeo<3, false> { static constexpr uint32_t TILE = 9216, BOFF = 6144, N = 64, TCOLS = 128; };
 // d = 3 round 1 ("wide"): X_t = x0(t) x1(t) UNREDUCED (512 bits = two 32-byte vectors, lo | hi), so the
 // integer pipe does 64 limb products per point instead of a Montgomery product's 136; vectors
 // 0..7 = X0 lo|hi, X1 lo|hi, X2 lo|hi, Xinf lo|hi, 8..11 = Y0, Y1, Y2, Yinf.  Two MMAs per tile into two
@@ -94,7 +96,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
     extern __shared__ uint8_t ft_raw[];
     uint8_t *base = ft_raw + ((1024 - (smem_u32(ft_raw) & 1023)) & 1023);
     BZK_ASSERT((size_t)(base - ft_raw) + (size_t)NW * (D * G::SLOT + FG::TILE) <= dyn_smem_bytes() &&
-               (size_t)(D == 3 && FIRST ? 8 : NV) * 32 * 33 * 4 <= (size_t)NW * D * G::SLOT);
+               (size_t)(D == 3 ? 2 * NV : NV) * 32 * 33 * 4 <= (size_t)NW * D * G::SLOT);
     const uint32_t b = blockIdx.y, warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint64_t h = 1ull << P.log_h;
     const uint64_t stride = (uint64_t)P.ctas * kFtCompute;
@@ -205,13 +207,17 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
                     for (int q = 0; q < 8; ++q) { lo.l[q] = X2[q]; hi.l[q] = X2[8 + q]; }
                     put(4, lo);
                     put(5, hi);
-                } else {
+                } else {   // points 0, 2, inf: X_t = x0(t) x1(t) unreduced (x_m(t) < 2p: X_t < 4p^2 < 2^512)
 #pragma unroll
                     for (int idx = 0; idx < NV; ++idx) {
-                        const fe x0 = d3_point<DERIVE>(a[0], sv[0], dl[0], idx);
-                        const fe x1 = d3_point<DERIVE>(a[1], sv[1], dl[1], idx);
-                        put(idx, mont_mul_lz(x0, x1));
-                        put(FG::BOFF / 1024 + idx, d3_point<DERIVE>(a[2], sv[2], dl[2], idx));
+                        acc17 W = acc17_zero();
+                        mul_acc(W, d3_point<DERIVE>(a[0], sv[0], dl[0], idx), d3_point<DERIVE>(a[1], sv[1], dl[1], idx));
+                        fe lo, hi;
+#pragma unroll
+                        for (int q = 0; q < 8; ++q) { lo.l[q] = W.w[q]; hi.l[q] = W.w[8 + q]; }
+                        put(2 * idx, lo);
+                        put(2 * idx + 1, hi);
+                        put(6 + idx, d3_point<DERIVE>(a[2], sv[2], dl[2], idx));
                     }
                 }
             }
@@ -245,6 +251,11 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
                         tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + 8192, 1024, 256), idesc, !first);
                         tc::mma_u8(tmem + 64, tc::desc_sw32(t0 + 4096, 1024, 256), tc::desc_sw32(t0 + 10240, 1024, 256),
                                    idesc, !first);
+                    } else if constexpr (D == 3) {     // (X0 | X2) x (Y0 | Y2), (Xinf | -) x Yinf
+                        const uint32_t idesc32 = tc::idesc_u8(128, 32, true) | (1u << 15);
+                        tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + 6144, 1024, 256), idesc, !first);
+                        tc::mma_u8(tmem + 64, tc::desc_sw32(t0 + 4096, 1024, 256), tc::desc_sw32(t0 + 8192, 1024, 256),
+                                   idesc32, !first);
                     } else {
                         tc::mma_u8(tmem, tc::desc_sw32(t0, 1024, 256), tc::desc_sw32(t0 + FG::BOFF, 1024, 256), idesc,
                                    !first);
@@ -263,8 +274,8 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
     __syncwarp();
     // anti-diagonal sums of the diagonal blocks (warp t reads TMEM lanes 32t.., columns 32t..; the wide
     // d = 3 round 1 has NB = 8 blocks: warp q reads its quadrant of both accumulators)
-    constexpr bool WIDE = D == 3 && FIRST;
-    constexpr int NB = WIDE ? 8 : NV;
+    constexpr bool WIDE = D == 3;
+    constexpr int NB = WIDE ? 2 * NV : NV;
     uint32_t *sM = reinterpret_cast<uint32_t *>(base);   // [NB][32][33] (reuses the TMA slots)
     __shared__ unsigned long long s_diag[NB][64];
     const bool any = (uint64_t)blockIdx.x * kFtCompute < h;
@@ -275,6 +286,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
         tc::fence_after();
 #pragma unroll
         for (int g = 0; g < (WIDE ? 2 : 1); ++g) {
+            if (WIDE && !FIRST && g == 1 && warp >= 2) break;   // (Xinf | -) x Yinf: lanes 0..63 only
             uint32_t v[32];
             const uint32_t col = WIDE ? g * 64 + (warp >> 1) * 32 : warp * 32;
             tc::ld_x32(tmem + ((warp * 32) << 16) + col, v);
@@ -305,7 +317,7 @@ __global__ void __launch_bounds__(ft_threads(NW), ft_minb(D, NW)) k_fused_tc(Rou
     if (threadIdx.x < NV && any) {
         fe f;
         if constexpr (WIDE) {
-            // S_t = sum_j X_t Y_t = B_lo + 2^256 B_hi (< 2^784, 25 words); partial = S_t R^-2 mod p (the
+            // S_t = sum_j X_t Y_t = B_lo + 2^256 B_hi (< 2^788, 25 words); partial = S_t R^-2 mod p (the
             // Montgomery products of the narrow path carried one R^-1 each): 16 REDC word steps
             const uint32_t Pw[8] = {BZK_P0, BZK_P1, BZK_P2, BZK_P3, BZK_P4, BZK_P5, BZK_P6, BZK_P7};
             uint32_t T[26];
