@@ -996,6 +996,21 @@ def run_sumcheck(args, rank, world, local):
                      "step_hbm_alg_frac": round(d * (1 << k) * esz * count / (ms_per_step / 1000.0) / 1e9 / hbm_peak, 4),
                      "hbm_peak_gbs": hbm_peak})
 
+    # both round kernels against the HBM roof (the dominant one is `roofline` above): round 1 reads
+    # only, so it can exceed the copy-bandwidth peak
+    per_kernel = {}
+    for pname, pkind in (("round1_eval", "round1"), ("fused_fold_eval", "fused")):
+        p_ms, p_cnt = prof.get(pname, (0.0, 0))
+        if p_cnt and kinds[dom] in ("round1", "fused"):
+            p_lps = max(1.0, p_cnt / args.steps)
+            p_avg_s = p_ms / p_cnt / 1000.0
+            p_bytes = alg_bytes_kind(d, k, pkind, esz) * count / p_lps
+            per_kernel[pname] = {"launches_per_step": p_lps, "avg_launch_ms": round(p_avg_s * 1000.0, 4),
+                                 "alg_bytes_per_launch": p_bytes, "achieved_gbs": round(p_bytes / p_avg_s / 1e9, 1),
+                                 "hbm_frac": round(p_bytes / p_avg_s / 1e9 / hbm_peak, 4)}
+    if per_kernel:
+        roofline["per_kernel_hbm"] = per_kernel
+
     kernel_ms = {n: round(v[0] / args.steps, 3) for n, v in prof.items() if v[1]}
     line = {"metric": METRIC, "value": round(value, 2), "unit": "proofs/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
